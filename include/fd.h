@@ -1,0 +1,164 @@
+/*
+ * fd.h -- C ABI of the B200-native boosted-cascade face detector.
+ *
+ * Method: Oro, Fernandez, Segura, Martorell, Hernando, "Accelerating Boosting-based Face
+ * Detection on GPUs", ICPP 2012 (PAPER.md; citations "P:Lxxx" = line of PAPER.md).
+ * Problem statement: "determine the presence of faces in arbitrary images, along with their
+ * locations and dimensions" (abstract).  The pipeline is Fig. 1:
+ * scaling -> (filtering) -> integral images -> cascade evaluation -> detections.
+ * Readings where the paper is silent are listed in DESIGN.md ("Readings", R1..R12).
+ *
+ * Conventions common to every entry point
+ *   - Every function returns fd_status; FD_OK == 0.  On failure a thread-local message is
+ *     available from fd_last_error() (valid until the next call on the same thread).
+ *   - d_* pointers are CALLER-OWNED DEVICE memory on the current CUDA device; h_* pointers
+ *     are caller-owned host memory (pinned is faster, pageable works).  The library owns
+ *     only cascade handles and an internal per-(device, stream) workspace that grows on
+ *     demand and is released by fd_release_workspaces() or at process exit.
+ *   - stream is a cudaStream_t passed as void* (NULL = legacy default stream).  Work is
+ *     stream-ordered; calls that must return a count synchronise `stream` once (noted).
+ *   - Frames are 8-bit luma ("only the luminance components"), row-major,
+ *     frame-major: byte (i, y, x) at frames[i*H*pitch + y*pitch + x].
+ *   - FD_EINVAL: W or H < 24, min_size < 24, scale_factor <= 1, step < 1, pitch < W, n < 1,
+ *     more than FD_MAX_LEVELS levels, NULL pointers, bad pitch alignment.
+ *     FD_EFORMAT: malformed cascade text.  FD_ECAPACITY: result larger than the caller's
+ *     buffer (the required count is still returned).  FD_ECUDA: CUDA error (text in
+ *     fd_last_error).  FD_ENOMEM: device or host allocation failed.
+ */
+#ifndef FD_H
+#define FD_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define FD_ABI_VERSION 1
+#define FD_MAX_LEVELS 128
+#define FD_WINDOW 24 /* fixed 24x24 sliding window, image scaled instead (Fig. 2) */
+
+typedef enum {
+    FD_OK = 0,
+    FD_EINVAL = 1,
+    FD_EFORMAT = 2,
+    FD_ECAPACITY = 3,
+    FD_ECUDA = 4,
+    FD_ENOMEM = 5
+} fd_status;
+
+/* Opaque cascade handle: library-owned, immutable after load, usable from several streams. */
+typedef struct fd_cascade_s* fd_cascade;
+
+/* One detection (40 bytes).  Detection output of fd_detect: the window at
+ * level-space origin (wx, wy) of pyramid level `level` reached the maximum depth; its
+ * original-frame rectangle is the back-projection x = floor(wx*f_k + 1/2),
+ * y = floor(wy*f_k + 1/2), w = h = floor(24*f_k + 1/2) ("multiplying the downscaling factor by
+ * the normalized dimensions").  score = sum of the last stage (the paper's
+ * "detection score"; reading R9); aux = depth (= number of stages).
+ * For fd_group output: x,y,w,h = rounded member mean, score = max member score,
+ * aux = member count, (level, wx, wy) = those of the cluster's first member. */
+typedef struct {
+    int32_t frame, level, wx, wy;
+    int32_t x, y, w, h;
+    float score;
+    int32_t aux;
+} fd_detection;
+
+/* Pyramid plan (host only).  f[k] = (min_size/24) * s^k by repeated multiplication,
+ * w[k] = floor(W/f[k]), h[k] = floor(H/f[k]) while both >= 24 (reading R1). */
+typedef struct {
+    int32_t n_levels;
+    double f[FD_MAX_LEVELS];
+    int32_t w[FD_MAX_LEVELS], h[FD_MAX_LEVELS];
+    int64_t windows[FD_MAX_LEVELS]; /* (floor((w-24)/step)+1) * (floor((h-24)/step)+1) */
+    int64_t total_windows;          /* per frame */
+} fd_plan;
+
+/* Parse a cascade in .fdc text (format in DESIGN.md "Cascade format": FDC 1 / window 24 24 /
+ * stages N / per stage "stage n T" / per stump "stump r (x y w h wt)*r theta left right").
+ * Stages of growing size evaluated in order with early rejection;
+ * stumps are GentleBoost regression stumps on Haar features.
+ * Uploads the packed cascade to the CURRENT device.  text need not be NUL-terminated.
+ * Errors: FD_EFORMAT (line number in fd_last_error): rect outside the 24x24 window,
+ * weight not an integer in [-16,16], r not in {1,2,3}, NaN/inf theta or leaves, NaN T.
+ * Ownership: *out is released with fd_free_cascade. */
+fd_status fd_load_cascade(const char* text, size_t len, fd_cascade* out);
+fd_status fd_free_cascade(fd_cascade c);
+fd_status fd_cascade_info(fd_cascade c, int32_t* n_stages, int32_t* n_stumps);
+
+/* Host-only pyramid geometry for a W x H frame (reading R1). */
+fd_status fd_pyramid_plan(int W, int H, int min_size, double scale_factor, int step, fd_plan* out);
+
+/* Scaling stage: every pyramid level of n frames, each sampled from the
+ * ORIGINAL frame with exact integer bilinear interpolation (reading R2: centre-aligned
+ * (x+1/2)f-1/2 in Q16, 8-bit weights, clamp to edge; identity filter, reading R3).
+ * d_levels: per frame sum_k w[k]*h[k] bytes, level-major, each level tight (pitch w[k]):
+ * byte (i, k, y, x) at d_levels[i*S + off_k + y*w[k] + x], S = sum_k w[k]h[k],
+ * off_k = sum_{j<k} w[j]h[j].  Asynchronous. */
+fd_status fd_build_pyramid(const uint8_t* d_frames, int n, int W, int H, int pitch, int min_size,
+                           double scale_factor, uint8_t* d_levels, void* stream);
+
+/* Integral image computation of n W x H images:
+ * ii[y][x] = sum_{y'<y, x'<x} I (uint32), sqii the same over I^2 (uint64), padded exclusive
+ * (H+1) x (W+1) (reading R4).  out_pitch (elements) >= W+1 and a multiple of 4; image i at
+ * d_ii + i*(H+1)*out_pitch.  Elements [W+1, out_pitch) of each row are written with the row
+ * total.  Asynchronous. */
+fd_status fd_integral(const uint8_t* d_img, int n, int W, int H, int pitch, uint32_t* d_ii,
+                      uint64_t* d_sqii, int out_pitch, void* stream);
+
+/* Cascade evaluation over every window of every pyramid level of n frames:
+ * per window the variance normalisation nf (reading R5), Haar features f = sum wt*R
+ * (reading R6), stump leaf ((float)f < theta*nf ? left : right) (R7), fp32 stage sums in
+ * stump order with early rejection, pass iff sum >= T (R8).  Windows reaching the maximum
+ * depth are detections, written to d_out sorted by (frame, level, wy, wx).
+ * capacity = elements of d_out.  *n_out = number of detections (host).  If
+ * *n_out > capacity returns FD_ECAPACITY and d_out is unspecified.
+ * Synchronises `stream` once (to read the count); the records in d_out are complete when
+ * `stream` next completes. */
+fd_status fd_detect(fd_cascade c, const uint8_t* d_frames, int n, int W, int H, int pitch,
+                    int min_size, double scale_factor, int step, fd_detection* d_out,
+                    int64_t capacity, int64_t* n_out, void* stream);
+
+/* fd_detect plus per-stage statistics: d_stage_counts (device, n_stages+1 int64, ADDED to):
+ * entry s = number of windows that entered stage s (entry 0 = all windows); entry N =
+ * accepted.  Stumps evaluated = sum_s entry[s] * stage_size[s]. */
+fd_status fd_detect_ex(fd_cascade c, const uint8_t* d_frames, int n, int W, int H, int pitch,
+                       int min_size, double scale_factor, int step, fd_detection* d_out,
+                       int64_t capacity, int64_t* n_out, int64_t* d_stage_counts, void* stream);
+
+/* The paper's native output: for every window, the deepest stage reached
+ * (d_depth, uint8: number of stages passed, N = face) and the sum of the last evaluated stage
+ * (d_score, float).  Layout [frame][level][wy/step][wx/step]; per-frame stride
+ * plan.total_windows.  Asynchronous. */
+fd_status fd_detect_depth(fd_cascade c, const uint8_t* d_frames, int n, int W, int H, int pitch,
+                          int min_size, double scale_factor, int step, uint8_t* d_depth,
+                          float* d_score, void* stream);
+
+/* End-to-end entry with HOST buffers: copies h_frames to the device, runs fd_detect, copies
+ * the detections back to h_out (capacity elements).  Synchronises `stream`. */
+fd_status fd_detect_host(fd_cascade c, const uint8_t* h_frames, int n, int W, int H, int pitch,
+                         int min_size, double scale_factor, int step, fd_detection* h_out,
+                         int64_t capacity, int64_t* n_out, void* stream);
+
+/* Grouping: per frame, repeatedly merge the pair of clusters with the smallest
+ * S_eyes (eq. 6) while it is < eyes_thresh (paper: 0.5), members averaged;
+ * ties -> lexicographically smallest pair (reading R10).  d_in: n detections sorted by frame
+ * (fd_detect order).  Clusters with >= min_neighbors members are written to d_out ordered by
+ * (frame, first member).  *n_out (host) = count; FD_ECAPACITY if > capacity.
+ * Synchronises `stream` once. */
+fd_status fd_group(const fd_detection* d_in, int64_t n, double eyes_thresh, int min_neighbors,
+                   fd_detection* d_out, int64_t capacity, int64_t* n_out, void* stream);
+
+/* Release every internal workspace of the current device. */
+fd_status fd_release_workspaces(void);
+
+/* Thread-local text of the last error ("" if none). */
+const char* fd_last_error(void);
+int fd_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FD_H */

@@ -1,0 +1,90 @@
+/*
+ * fd_oracle.h -- plain, slow, obviously-correct CPU oracle for the face-detection hot path
+ * of Oro et al., "Accelerating Boosting-based Face Detection on GPUs" (ICPP 2012).
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py's
+ * cpu_baseline / --impl reference legs may load this library.  It shares no code with
+ * the CUDA path (paper_conf_icpp_orofsmh12_b200/) and neither includes the other.
+ *
+ * Citations are "P:Lxxx" = line of PAPER.md, plus SURVEY.md 8(c) row ids (c1..c10) for
+ * the readings taken where the paper is silent.  Every reading is listed in DESIGN.md.
+ * Pins: tests/test_oracle.py (brute-force rect sums, closed forms, worked example,
+ * all-pass/all-reject cascades, Table I counts, grouping hand cases).
+ */
+#ifndef FD_ORACLE_H
+#define FD_ORACLE_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define FDO_MAX_LEVELS 128
+
+typedef struct { int32_t x, y, w, h, wt; } fdo_rect;
+typedef struct { int32_t nrect; fdo_rect r[3]; float theta, left, right; } fdo_stump;
+typedef struct { int32_t n, first; float T; } fdo_stage;
+typedef struct {
+    int32_t win_w, win_h, n_stages, n_stumps;
+    fdo_stage* stages;
+    fdo_stump* stumps;
+} fdo_cascade;
+
+/* same 40-byte layout as the product's fd_detection (checked in tests) */
+typedef struct {
+    int32_t frame, level, wx, wy, x, y, w, h;
+    float score;
+    int32_t aux;
+} fdo_detection;
+
+/* .fdc text -> cascade (NULL on error, message in err). */
+fdo_cascade* fdo_cascade_parse(const char* text, size_t len, char* err, int errlen);
+void fdo_cascade_free(fdo_cascade* c);
+
+/* c1: pyramid levels; returns n_levels (0 if none fit, -1 on bad args). */
+int fdo_plan(int W, int H, int min_size, double scale, int step, int max_levels,
+             double* f, int32_t* Wk, int32_t* Hk, int64_t* nwin);
+/* c2: level image (Wk x Hk, tight pitch) sampled from the frame. */
+void fdo_resample(const uint8_t* frame, int W, int H, int pitch, double f, int Wk, int Hk, uint8_t* out);
+/* c3: ii, sqii of (H+1) x (W+1), tight pitch W+1. */
+void fdo_integral(const uint8_t* img, int W, int H, int pitch, uint32_t* ii, uint64_t* sqii);
+/* c3/c6: one rectangle sum by the four-corner rule (9 accesses incl. the rect). */
+uint32_t fdo_rect_sum(const uint32_t* ii, int ii_pitch, int x, int y, int w, int h);
+/* c5: normalisation factor nf of the 24x24 window at (wx, wy). */
+float fdo_window_nf(const uint32_t* ii, const uint64_t* sqii, int ii_pitch, int wx, int wy);
+/* c6: feature response sum_r wt_r * R_r of the window at (wx, wy). */
+int32_t fdo_feature(const uint32_t* ii, int ii_pitch, int wx, int wy, const fdo_rect* r, int nrect);
+/* c6 batched for calibration tooling: wins = (wx, wy) pairs. */
+void fdo_feature_values(const uint32_t* ii, int ii_pitch, const int32_t* wins, int64_t nw,
+                        const fdo_rect* r, int nrect, int32_t* out);
+void fdo_window_nf_values(const uint32_t* ii, const uint64_t* sqii, int ii_pitch,
+                          const int32_t* wins, int64_t nw, float* out);
+/* c7/c8: evaluate one window; returns depth (stages passed); *score = last evaluated stage sum;
+ * *near = bit0 stage-sum within 1e-4 of T, bit1 stump near-tie (c11). */
+int fdo_eval_window(const fdo_cascade* c, const uint32_t* ii, const uint64_t* sqii, int ii_pitch,
+                    int wx, int wy, float* score, int* near);
+/* c7/c8 over one level's windows (row-major over (wy/step, wx/step)). */
+void fdo_eval_level(const fdo_cascade* c, const uint32_t* ii, const uint64_t* sqii, int Wk, int Hk,
+                    int step, uint8_t* depth, float* score, uint8_t* near);
+
+/* Whole path per frame batch (frames u8[n][H][pitch]).
+ * fdo_detect: c1..c9; detections sorted (frame, level, wy, wx); returns total count (writes
+ * at most cap); *n_near = windows flagged near-threshold.  nthreads: host threads. */
+int64_t fdo_detect(const fdo_cascade* c, const uint8_t* frames, int n, int W, int H, int pitch,
+                   int min_size, double scale, int step, int nthreads,
+                   fdo_detection* out, int64_t cap, int64_t* n_near);
+/* per-window depth/score/near maps, layout [frame][level][wy/step][wx/step]. */
+int fdo_detect_depth(const fdo_cascade* c, const uint8_t* frames, int n, int W, int H, int pitch,
+                     int min_size, double scale, int step, int nthreads,
+                     uint8_t* depth, float* score, uint8_t* near);
+/* c10: greedy S_eyes grouping (eq. 6).  Input sorted by frame. Returns count. */
+int64_t fdo_group(const fdo_detection* in, int64_t n, double eyes_thresh, int min_neighbors,
+                  fdo_detection* out, int64_t cap);
+/* eq. 6 between two rectangles given as doubles (for pins). */
+double fdo_s_eyes(double ax, double ay, double aw, double ah, double bx, double by, double bw, double bh);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,367 @@
+"""Pins for the CPU oracle against what the paper and the mathematics fix (CPU only).
+
+Each test names the SURVEY.md 8(c) row / paper passage it pins.  The oracle is never checked
+against itself: expected values are closed forms, brute force (numpy sums written from the
+definition in a different form), hand computations (tests/golden/), or invariants.
+"""
+import math
+import os
+
+import numpy as np
+import pytest
+
+import fdgen
+import oracle
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _golden(name):
+    rows = []
+    with open(os.path.join(GOLD, name)) as fh:
+        for line in fh:
+            line = line.strip()
+            if line and not line.startswith("#"):
+                rows.append(line.split())
+    return rows
+
+
+def cascade_text(stages):
+    """stages: list of (T, [ (rects, theta, left, right), ... ])"""
+    out = ["FDC 1", "window 24 24", f"stages {len(stages)}"]
+    for T, stumps in stages:
+        out.append(f"stage {len(stumps)} {float(T)!r}" if math.isfinite(T) else f"stage {len(stumps)} {'inf' if T > 0 else '-inf'}")
+        for rects, th, l, r in stumps:
+            rs = " ".join(" ".join(str(v) for v in rc) for rc in rects)
+            out.append(f"stump {len(rects)} {rs} {np.float32(th).item()!r} {np.float32(l).item()!r} {np.float32(r).item()!r}")
+    return "\n".join(out) + "\n"
+
+
+# ---------------------------------------------------------------- c1: pyramid geometry
+@pytest.mark.parametrize("row", [r for r in _golden("pyramid_counts.txt") if r[0][0].isdigit()])
+def test_plan_closed_form_totals(row):
+    W, H, s, step, nl, tot = int(row[0]), int(row[1]), float(row[2]), int(row[3]), int(row[4]), int(row[5])
+    lv = oracle.plan(W, H, 24, s, step)
+    assert len(lv) == nl
+    assert sum(l[3] for l in lv) == tot
+    # closed form written independently: f_k by repeated multiply, floor rule
+    f = 1.0
+    for k, (fk, wk, hk, nw) in enumerate(lv):
+        assert fk == f
+        assert wk == math.floor(W / f) and hk == math.floor(H / f)
+        assert nw == ((wk - 24) // step + 1) * ((hk - 24) // step + 1)
+        f = f * s
+    assert math.floor(W / f) < 24 or math.floor(H / f) < 24
+
+
+def test_plan_per_level_counts():
+    for row in _golden("pyramid_counts.txt"):
+        if row[0] == "levels":
+            W, H, s = int(row[1]), int(row[2]), float(row[3])
+            assert [l[3] for l in oracle.plan(W, H, 24, s, 1)] == [int(v) for v in row[4:]]
+        elif row[0] == "dims":
+            k, wk, hk, nw = (int(v) for v in row[1:])
+            lv = oracle.plan(1920, 1080, 24, 1.1, 1)[k]
+            assert (lv[1], lv[2], lv[3]) == (wk, hk, nw)
+
+
+@pytest.mark.parametrize("W,H,s", [(320, 240, 1.25), (640, 480, 1.2), (1920, 1080, 1.1), (3840, 2160, 1.1)])
+def test_backprojection_inside_frame(W, H, s):
+    # c1/c9 invariant: the last window of every level back-projects inside the frame
+    for (f, wk, hk, _n) in oracle.plan(W, H, 24, s, 1):
+        x = math.floor((wk - 24) * f + 0.5)
+        y = math.floor((hk - 24) * f + 0.5)
+        w = math.floor(24 * f + 0.5)
+        assert x + w <= W and y + w <= H
+
+
+def test_plan_rejects_bad_args():
+    with pytest.raises(ValueError):
+        oracle.plan(20, 240, 24, 1.25, 1)
+    with pytest.raises(ValueError):
+        oracle.plan(320, 240, 24, 1.0, 1)
+    with pytest.raises(ValueError):
+        oracle.plan(320, 240, 16, 1.25, 1)
+
+
+# ---------------------------------------------------------------- c2: scaling
+def _resample_naive(img, f, Wk, Hk):
+    """Second, differently written bilinear: interpolate along x then y, with exact rationals
+    for the Q16 sample position (centre-aligned (x+1/2)f - 1/2, 8-bit weights, clamp)."""
+    from fractions import Fraction
+    H, W = img.shape
+    r = Fraction(int(math.floor(f * 65536 + 0.5)), 65536)
+    out = np.zeros((Hk, Wk), np.uint8)
+    for y in range(Hk):
+        sy = (y + Fraction(1, 2)) * r - Fraction(1, 2)
+        y0 = min(math.floor(sy), H - 1)
+        wy = math.floor((sy - math.floor(sy)) * 256)
+        y1 = min(y0 + 1, H - 1)
+        for x in range(Wk):
+            sx = (x + Fraction(1, 2)) * r - Fraction(1, 2)
+            x0 = min(math.floor(sx), W - 1)
+            wx = math.floor((sx - math.floor(sx)) * 256)
+            x1 = min(x0 + 1, W - 1)
+            top = int(img[y0, x0]) * (256 - wx) + int(img[y0, x1]) * wx
+            bot = int(img[y1, x0]) * (256 - wx) + int(img[y1, x1]) * wx
+            out[y, x] = (top * (256 - wy) + bot * wy + 32768) >> 16
+    return out
+
+
+def test_resample_level0_identity():
+    fr = fdgen.background(1, 7, 320, 240)
+    f, wk, hk, _ = oracle.plan(320, 240, 24, 1.25, 1)[0]
+    assert f == 1.0 and (wk, hk) == (320, 240)
+    np.testing.assert_array_equal(oracle.resample(fr, f, wk, hk), fr)
+
+
+def test_resample_constant_frame():
+    fr = np.full((97, 131), 173, np.uint8)
+    for (f, wk, hk, _) in oracle.plan(131, 97, 24, 1.13, 1):
+        assert (oracle.resample(fr, f, wk, hk) == 173).all()
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_resample_matches_naive(seed):
+    rng = np.random.default_rng(seed)
+    fr = rng.integers(0, 256, (53, 61), dtype=np.uint8)
+    for (f, wk, hk, _) in oracle.plan(61, 53, 24, 1.17, 1):
+        np.testing.assert_array_equal(oracle.resample(fr, f, wk, hk), _resample_naive(fr, f, wk, hk))
+
+
+def test_resample_linear_ramp():
+    # bilinear reproduces a linear ramp: value ~ a*(x+1/2)f - 1/2 ... within 1 grey level
+    W, H = 200, 40
+    fr = np.tile(np.arange(W, dtype=np.int64), (H, 1)).astype(np.uint8)
+    for (f, wk, hk, _) in oracle.plan(W, H, 24, 1.3, 1)[:4]:
+        lv = oracle.resample(fr, f, wk, hk).astype(np.float64)
+        xs = (np.arange(wk) + 0.5) * f - 0.5
+        np.testing.assert_allclose(lv[hk // 2, : wk - 2], xs[: wk - 2], atol=1.01)
+
+
+# ---------------------------------------------------------------- c3: integral images
+@pytest.mark.parametrize("seed", [0, 1])
+def test_integral_brute_force_all_rects(seed):
+    rng = np.random.default_rng(seed)
+    img = rng.integers(0, 256, (9, 11), dtype=np.uint8)
+    ii, sq = oracle.integral(img)
+    I = img.astype(np.int64)
+    for y in range(10):
+        for x in range(12):
+            assert ii[y, x] == I[:y, :x].sum()
+            assert sq[y, x] == (I[:y, :x] ** 2).sum()
+    for y in range(9):
+        for x in range(11):
+            for h in range(1, 10 - y):
+                for w in range(1, 12 - x):
+                    assert oracle.rect_sum(ii, x, y, w, h) == I[y:y + h, x:x + w].sum()
+
+
+def test_integral_constant_closed_form():
+    c = 201
+    img = np.full((30, 41), c, np.uint8)
+    ii, sq = oracle.integral(img)
+    y, x = np.mgrid[0:31, 0:42]
+    np.testing.assert_array_equal(ii, (c * x * y).astype(np.uint32))
+    np.testing.assert_array_equal(sq, (c * c * x * y).astype(np.uint64))
+
+
+def test_integral_total_and_u32_range():
+    # worst case 1080p all-255: ii max 255*1920*1080 fits u32; sqii needs u64
+    img = np.full((1080, 1920), 255, np.uint8)
+    ii, sq = oracle.integral(img)
+    assert int(ii[-1, -1]) == 255 * 1920 * 1080 == 528768000
+    assert int(sq[-1, -1]) == 255 * 255 * 1920 * 1080 > 2 ** 32
+
+
+# ---------------------------------------------------------------- c5: variance normalisation
+def test_nf_constant_window():
+    ii, sq = oracle.integral(np.full((24, 24), 77, np.uint8))
+    assert oracle.window_nf(ii, sq, 0, 0) == 1.0
+
+
+@pytest.mark.parametrize("a,b", [(0, 255), (10, 20), (255, 0), (3, 200)])
+def test_nf_two_valued_windows(a, b):
+    # half/half and checkerboard with values a,b: v = (288 |a-b|)^2, nf = 288 |a-b|
+    half = np.full((24, 24), a, np.uint8)
+    half[:, 12:] = b
+    chk = np.where((np.add.outer(np.arange(24), np.arange(24)) % 2) == 0, a, b).astype(np.uint8)
+    for img in (half, chk):
+        ii, sq = oracle.integral(img)
+        assert oracle.window_nf(ii, sq, 0, 0) == 288.0 * abs(a - b)
+
+
+# ---------------------------------------------------------------- c6: features (Table I, Fig. 4)
+def test_table1_counts():
+    want = {r[0]: int(r[1]) for r in _golden("table1.txt")}
+    assert fdgen.table1_counts() == want
+
+
+def test_families_zero_on_constant_window():
+    ii, _ = oracle.integral(np.full((24, 24), 93, np.uint8))
+    rng = np.random.default_rng(5)
+    counts = fdgen.table1_counts()
+    for fam in counts:
+        for idx in rng.integers(0, counts[fam], 50):
+            assert oracle.feature(ii, 0, 0, fdgen.table1_feature(fam, int(idx))) == 0
+
+
+def test_fig4_edge_expression_unpadded_integral():
+    """Fig. 4: eval = (-1)(r[h0]+r[h1]-r[h2]-r[h3]) + 2(r[h4]+r[h5]-r[h6]-r[h7]) over the
+    576-row unpadded 24x24 integral J.  Table I features start at offset >= 1, so the
+    paper's corners J[y-1][x-1] ... equal the padded ii[y][x] ...: the oracle must agree."""
+    rng = np.random.default_rng(11)
+    img = rng.integers(0, 256, (24, 24), dtype=np.uint8)
+    J = img.astype(np.int64).cumsum(0).cumsum(1)       # unpadded inclusive integral
+    ii, _ = oracle.integral(img)
+    counts = fdgen.table1_counts()
+    for idx in rng.integers(0, counts["edge"], 200):
+        rects = fdgen.table1_feature("edge", int(idx))
+        (x0, y0, w0, h0, _), (x1, y1, w1, h1, _) = rects
+
+        def rsum(x, y, w, h):  # r[A] + r[D] - r[B] - r[C] with corners just outside the rect
+            return J[y + h - 1, x + w - 1] + J[y - 1, x - 1] - J[y - 1, x + w - 1] - J[y + h - 1, x - 1]
+        ev = -1 * rsum(x0, y0, w0, h0) + 2 * rsum(x1, y1, w1, h1)
+        assert oracle.feature(ii, 0, 0, rects) == ev
+        # and against a direct pixel sum
+        direct = -int(img[y0:y0 + h0, x0:x0 + w0].astype(np.int64).sum()) + 2 * int(img[y1:y1 + h1, x1:x1 + w1].astype(np.int64).sum())
+        assert ev == direct
+
+
+# ---------------------------------------------------------------- c7/c8: stump, stages
+def _worked_window():
+    img = np.zeros((24, 24), np.uint8)
+    img[:, 12:] = 255
+    return img
+
+
+def test_worked_example_single_stump():
+    g = {r[0]: r[1] for r in _golden("worked_example.txt")}
+    img = _worked_window()
+    ii, sq = oracle.integral(img)
+    whole, half = (1, 1, 22, 22, -1), (1, 1, 11, 22, 2)
+    assert oracle.rect_sum(ii, 1, 1, 22, 22) == int(g["R_whole"])
+    assert oracle.rect_sum(ii, 1, 1, 11, 22) == int(g["R_half"])
+    assert oracle.feature(ii, 0, 0, [whole, half]) == int(g["f"])
+    assert oracle.window_nf(ii, sq, 0, 0) == float(g["nf"])
+    casc = oracle.Cascade(cascade_text([(-10.0, [([whole, half], -0.5, 0.25, 0.75)])]))
+    d, score, near = oracle.eval_window(casc, ii, sq, 0, 0)
+    assert g["leaf"] == "left" and score == np.float32(0.25) and d == 1 and near == 0
+    # the same stump with theta = -1.0: t = -73440 < f -> right leaf
+    casc2 = oracle.Cascade(cascade_text([(-10.0, [([whole, half], -1.0, 0.25, 0.75)])]))
+    assert oracle.eval_window(casc2, ii, sq, 0, 0)[1] == np.float32(0.75)
+
+
+def test_stump_tie_goes_right():
+    # constant window: f = 0, nf = 1; theta = 0 -> t = 0, (0 < 0) false -> right leaf (c7)
+    ii, sq = oracle.integral(np.full((24, 24), 50, np.uint8))
+    casc = oracle.Cascade(cascade_text([(-10.0, [([(1, 1, 4, 4, -1), (1, 1, 2, 4, 2)], 0.0, -1.0, 1.0)])]))
+    d, score, near = oracle.eval_window(casc, ii, sq, 0, 0)
+    assert score == 1.0 and near & 2
+
+
+def test_stage_pass_on_equality_and_early_exit():
+    ii, sq = oracle.integral(_worked_window())
+    st = ([(1, 1, 22, 22, -1), (1, 1, 11, 22, 2)], -0.5, 0.25, 0.75)     # leaf 0.25
+    # stage 0 threshold exactly 0.5 = 0.25 + 0.25 -> pass (>=); stage 1 threshold 0.26 > 0.25 -> reject
+    casc = oracle.Cascade(cascade_text([(0.5, [st, st]), (0.26, [st]), (-1.0, [st])]))
+    d, score, near = oracle.eval_window(casc, ii, sq, 0, 0)
+    assert d == 1 and score == np.float32(0.25)
+
+
+def test_all_pass_and_all_reject_cascades():
+    W, H, s = 160, 120, 1.25
+    fr, _ = fdgen.frames(9, 3, 2, W, H)
+    st = ([(1, 1, 10, 10, -1), (1, 1, 5, 10, 2)], 0.1, 0.5, 0.5)
+    allpass = oracle.Cascade(cascade_text([(-math.inf, [st, st]), (-1e30, [st])]))
+    dets, _ = oracle.detect(allpass, fr, 24, s, 1, nthreads=2)
+    tot = sum(l[3] for l in oracle.plan(W, H, 24, s, 1))
+    assert len(dets) == 2 * tot
+    assert (dets["aux"] == 2).all()
+    allrej = oracle.Cascade(cascade_text([(math.inf, [st])]))
+    d, sc, nr = oracle.detect_depth(allrej, fr, 24, s, 1)
+    assert len(d) == 2 * tot and (d == 0).all() and (sc == 0.5).all()
+
+
+def test_detect_matches_depth_maps_and_order():
+    fr, _ = fdgen.frames(1, 0, 2, 320, 240)
+    casc = oracle.Cascade.from_file(os.path.join(ROOT, "cascades", "c1.fdc"))
+    dets, _ = oracle.detect(casc, fr, 24, 1.25, 1, nthreads=4)
+    d, sc, _ = oracle.detect_depth(casc, fr, 24, 1.25, 1, nthreads=4)
+    assert (d == casc.n_stages).sum() == len(dets)
+    keys = dets["frame"].astype(np.int64) << 40 | dets["level"].astype(np.int64) << 32 | dets["wy"].astype(np.int64) << 16 | dets["wx"]
+    assert (np.diff(keys) > 0).all()
+    # window step: detections only on the step grid, in range
+    d2, _, _ = oracle.detect_depth(casc, fr, 24, 1.25, 2, nthreads=4)
+    assert len(d2) == 2 * sum(l[3] for l in oracle.plan(320, 240, 24, 1.25, 2))
+
+
+def test_parse_errors():
+    with pytest.raises(ValueError):
+        oracle.Cascade("FDC 2\nwindow 24 24\nstages 1\nstage 1 0\nstump 1 0 0 1 1 1 0 0 0\n")
+    with pytest.raises(ValueError):       # rect outside the window
+        oracle.Cascade("FDC 1\nwindow 24 24\nstages 1\nstage 1 0\nstump 1 20 0 5 1 1 0 0 0\n")
+    with pytest.raises(ValueError):       # weight out of range
+        oracle.Cascade("FDC 1\nwindow 24 24\nstages 1\nstage 1 0\nstump 1 0 0 1 1 17 0 0 0\n")
+    with pytest.raises(ValueError):       # non-finite theta
+        oracle.Cascade("FDC 1\nwindow 24 24\nstages 1\nstage 1 0\nstump 1 0 0 1 1 1 nan 0 0\n")
+    c = oracle.Cascade("FDC 1\nwindow 24 24\nstages 1\nstage 1 0x1.8p-1\nstump 1 0 0 1 1 1 0x1p-2 -1 1\n")
+    assert c.n_stages == 1 and c.n_stumps == 1
+
+
+# ---------------------------------------------------------------- c9: planted faces
+@pytest.mark.parametrize("cfg,W,H,s,mfl", [(1, 320, 240, 1.25, 8), (2, 640, 480, 1.2, 12)])
+def test_planted_faces_detected_iou1(cfg, W, H, s, mfl):
+    casc = oracle.Cascade.from_file(os.path.join(ROOT, "cascades", f"c{cfg}.fdc"))
+    lv = oracle.plan(W, H, 24, s, 1)
+    fr, faces = fdgen.frames(cfg, 0, 3, W, H, lv, faces="fixed", face_param=3, max_face_level=mfl)
+    dets, _ = oracle.detect(casc, fr, 24, s, 1, nthreads=4)
+    for i, fl in enumerate(faces):
+        for (k, wx, wy, X, Y, S) in fl:
+            m = (dets["frame"] == i) & (dets["level"] == k) & (dets["wx"] == wx) & (dets["wy"] == wy)
+            assert m.sum() == 1, (i, k, wx, wy)
+            d = dets[m][0]
+            # eq. 5 S_square (IoU) of the back-projected rect vs the planted rect = 1
+            assert (d["x"], d["y"], d["w"], d["h"]) == (X, Y, S, S)
+
+
+# ---------------------------------------------------------------- c10: grouping (eq. 6)
+def _det(frame, x, y, w, score=0.0):
+    return (frame, 0, x, y, x, y, w, w, score, 1)
+
+
+def test_s_eyes_closed_form():
+    # equal-size windows offset by delta: S = 2 delta / (0.4 w) = 5 delta / w
+    assert oracle.s_eyes((0, 0, 100, 100), (9, 0, 100, 100)) == pytest.approx(0.45, abs=1e-12)
+    assert oracle.s_eyes((0, 0, 100, 100), (10, 0, 100, 100)) == 0.5
+    assert oracle.s_eyes((5, 5, 40, 40), (5, 5, 40, 40)) == 0.0
+    assert oracle.s_eyes((0, 0, 100, 100), (0, 8, 100, 100)) == pytest.approx(0.4, abs=1e-12)
+
+
+def test_group_hand_cases():
+    D = oracle.DET_DTYPE
+    # delta 9 merges, delta 10 does not (S = 0.5 exactly is not < 0.5)
+    g = oracle.group(np.array([_det(0, 0, 0, 100, 1.0), _det(0, 9, 0, 100, 2.0)], D))
+    assert len(g) == 1 and g[0]["aux"] == 2 and g[0]["score"] == 2.0 and g[0]["x"] == 5   # round(4.5) half up
+    g = oracle.group(np.array([_det(0, 0, 0, 100), _det(0, 10, 0, 100)], D))
+    assert len(g) == 2
+    # identical windows merge; far windows never; frames never mix
+    g = oracle.group(np.array([_det(0, 50, 50, 30), _det(0, 50, 50, 30), _det(0, 500, 50, 30),
+                               _det(1, 50, 50, 30)], D))
+    assert sorted(g["aux"].tolist()) == [1, 1, 2]
+    # min_neighbors filters small clusters
+    g = oracle.group(np.array([_det(0, 50, 50, 30), _det(0, 50, 50, 30), _det(0, 500, 50, 30)], D),
+                     min_neighbors=2)
+    assert len(g) == 1 and g[0]["aux"] == 2
+
+
+def test_group_greedy_closest_pair_first():
+    D = oracle.DET_DTYPE
+    # a(0), b(4), c(8) at w=100: S(a,b)=S(b,c)=0.2 tie -> (a,b) first (lexicographic);
+    # merged ab mean x=2 -> S(ab,c)=0.3 < 0.5 -> all three merge into one cluster
+    g = oracle.group(np.array([_det(0, 0, 0, 100), _det(0, 4, 0, 100), _det(0, 8, 0, 100)], D))
+    assert len(g) == 1 and g[0]["aux"] == 3 and g[0]["x"] == 4
+    # a(0), b(9), c(18): S(a,b)=S(b,c)=0.45 -> (a,b) merge first (mean 4.5), then S(ab,c)=0.675 -> stop
+    g = oracle.group(np.array([_det(0, 0, 0, 100), _det(0, 9, 0, 100), _det(0, 18, 0, 100)], D))
+    assert sorted(g["aux"].tolist()) == [1, 2]

@@ -1,0 +1,252 @@
+#!/usr/bin/env python3
+"""Write the synthetic, paper-shaped cascades cascades/c{1,2,3}.fdc.
+
+A committed script that calls only ``oracle/`` (feature responses, nf, resampling, integral
+images, partial-cascade detection for bootstrapping) and ``fdgen`` (seeded frames, template,
+Table I feature space).  The cascades are INPUTS: nothing here is an expected value.
+Recipe:
+
+* stage sizes and pass targets: c1 3 stages 2/5/10 (p=0.5); c2 20 stages
+  n_k = 12 + 4k = 1000 stumps (p=0.5); c3 25 stages n_k = 10 + 4k, last 102 = 1446 stumps (the
+  paper's own cascade size) with p1 = 0.0548, p2 = 0.270 (Fig. 7 rejection
+  profile), p>=3 = 0.5.
+* features drawn uniformly from the Table I space, kept if discriminative between
+  the background windows that reached the stage and the planted template as it appears after
+  pyramid resampling at every face level (so planted faces pass every stage with margin).
+* stump threshold theta between the background median and the template's worst variant;
+  leaves: face side +a, other side -b, a, b uniform in [0.2, 1] (GentleBoost regression
+  stump form, [6]).
+* stage threshold T_s: the achievable stage sum giving the pass rate closest to p_s on the
+  background windows that reached stage s, moved half-way to the next lower achievable sum
+  (so no window sits on a threshold), capped at the template's worst stage sum - 0.01.
+  When fewer than MIN_POOL background windows reach stage s, fresh background frames are
+  added and run through the stages built so far (bootstrapping).
+"""
+from __future__ import annotations
+
+import argparse
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import fdgen  # noqa: E402
+import oracle  # noqa: E402
+
+CONFIGS = {
+    1: dict(W=320, H=240, scale=1.25, sizes=[2, 5, 10], p=[0.5, 0.5, 0.5], bg_frames=8, max_boot=0,
+            max_face_level=8),
+    2: dict(W=640, H=480, scale=1.2, sizes=[12 + 4 * k for k in range(20)], p=[0.5] * 20, bg_frames=8,
+            max_boot=64, max_face_level=12),
+    3: dict(W=1920, H=1080, scale=1.1, sizes=[10 + 4 * k for k in range(24)] + [102],
+            p=[0.0548, 0.270] + [0.5] * 23, bg_frames=2, max_boot=48, max_face_level=30),
+}
+MIN_POOL = 1000
+N_SUB = 20_000
+FAMILIES = ["edge", "line", "center", "diagonal"]
+BG_BASE = 1_000_000_000
+
+
+def fmt_cascade(stages) -> str:
+    lines = ["FDC 1", "window 24 24", f"stages {len(stages)}"]
+    for T, stumps in stages:
+        lines.append(f"stage {len(stumps)} {float(T).hex()}")
+        for rects, theta, left, right in stumps:
+            rs = " ".join(f"{x} {y} {w} {h} {wt}" for (x, y, w, h, wt) in rects)
+            lines.append(f"stump {len(rects)} {rs} {float(theta).hex()} {float(left).hex()} {float(right).hex()}")
+    return "\n".join(lines) + "\n"
+
+
+class Pool:
+    """Background windows that reached the current stage: per (frame, level) positions."""
+
+    def __init__(self, cfg: int, c: dict):
+        self.cfg, self.c = cfg, c
+        self.levels = oracle.plan(c["W"], c["H"], 24, c["scale"], 1)
+        self.groups = []          # dicts: ii, sq, wins (n,2) int32, nf (n,)
+        self.next_frame = BG_BASE
+        self.boot = 0
+
+    def _frame(self):
+        fr, _ = fdgen.frames(self.cfg, self.next_frame, 1, self.c["W"], self.c["H"])
+        self.next_frame += 1
+        return fr[0]
+
+    def add_full_frame(self):
+        fr = self._frame()
+        for (f, wk, hk, nw) in self.levels:
+            ii, sq = oracle.integral(oracle.resample(fr, f, wk, hk))
+            nx = wk - 23
+            idx = np.arange(nw)
+            wins = np.stack([idx % nx, idx // nx], axis=1).astype(np.int32)
+            self.groups.append(dict(ii=ii, sq=sq, wins=wins, nf=oracle.window_nf_values(ii, sq, wins)))
+
+    def add_bootstrap_frame(self, partial: oracle.Cascade):
+        fr = self._frame()
+        self.boot += 1
+        dets, _ = oracle.detect(partial, fr, 24, self.c["scale"], 1, nthreads=os.cpu_count() or 1)
+        for k in np.unique(dets["level"]):
+            f, wk, hk, _nw = self.levels[int(k)]
+            d = dets[dets["level"] == k]
+            ii, sq = oracle.integral(oracle.resample(fr, f, wk, hk))
+            wins = np.stack([d["wx"], d["wy"]], axis=1).astype(np.int32)
+            self.groups.append(dict(ii=ii, sq=sq, wins=wins, nf=oracle.window_nf_values(ii, sq, wins)))
+
+    def size(self) -> int:
+        return sum(len(g["wins"]) for g in self.groups)
+
+    def sub_mosaic(self, rng, n: int):
+        """Random subsample of the pool as a 25x25-patch mosaic (+ nf)."""
+        sizes = np.array([len(g["wins"]) for g in self.groups])
+        tot = int(sizes.sum())
+        pick = np.sort(rng.choice(tot, min(n, tot), replace=False))
+        starts = np.concatenate([[0], np.cumsum(sizes)])
+        patches, nfs = [], []
+        for gi, g in enumerate(self.groups):
+            sel = pick[(pick >= starts[gi]) & (pick < starts[gi + 1])] - starts[gi]
+            for i in sel:
+                wx, wy = g["wins"][i]
+                patches.append(g["ii"][wy:wy + 25, wx:wx + 25])
+            nfs.append(g["nf"][sel])
+        return np.ascontiguousarray(np.concatenate(patches, axis=1)), np.concatenate(nfs)
+
+    def leaves(self, rects, theta, left, right):
+        out = []
+        for g in self.groups:
+            f = oracle.feature_values(g["ii"], g["wins"], rects)
+            out.append(leaf_of(f, g["nf"], theta, left, right))
+        return out
+
+    def keep(self, masks):
+        groups = []
+        for g, m in zip(self.groups, masks):
+            if m.any():
+                groups.append(dict(ii=g["ii"], sq=g["sq"], wins=g["wins"][m], nf=g["nf"][m]))
+        self.groups = groups
+
+
+def template_variants(cfg: int, c: dict):
+    """The template as the pyramid sees it after planting at each face level (oracle resample)."""
+    W, H = c["W"], c["H"]
+    levels = oracle.plan(W, H, 24, c["scale"], 1)
+    patches, nfs = [], []
+    for k, (f, wk, hk, _nw) in enumerate(levels[: c["max_face_level"]]):
+        for (wx, wy) in [(1, 1), (wk // 3, hk // 3), (wk - 25, hk - 25), (wk // 2 + 1, 2), (wk // 5 + 3, hk // 2 + 1)]:
+            if wx < 0 or wy < 0 or wx > wk - 24 or wy > hk - 24:
+                continue
+            frame = fdgen.background(cfg, 2_000_000_000 + k, W, H)
+            X, Y, S = int(np.floor(wx * f + 0.5)), int(np.floor(wy * f + 0.5)), int(np.floor(24 * f + 0.5))
+            if X + S > W or Y + S > H:
+                continue
+            fdgen.render_face(frame, X, Y, S)
+            lv = oracle.resample(frame, f, wk, hk)
+            ii, sq = oracle.integral(lv)
+            nfs.append(oracle.window_nf_values(ii, sq, np.array([[wx, wy]], np.int32)))
+            patches.append(ii[wy:wy + 25, wx:wx + 25])
+    return np.ascontiguousarray(np.concatenate(patches, axis=1)), np.concatenate(nfs)
+
+
+def mosaic_f(ii_m: np.ndarray, rects) -> np.ndarray:
+    n = ii_m.shape[1] // 25
+    wins = np.stack([np.arange(n) * 25, np.zeros(n, np.int64)], axis=1).astype(np.int32)
+    return oracle.feature_values(ii_m, wins, rects)
+
+
+def leaf_of(f: np.ndarray, nf: np.ndarray, theta, left, right):
+    t = (np.float32(theta) * nf.astype(np.float32)).astype(np.float32)
+    return np.where(f.astype(np.float32) < t, np.float32(left), np.float32(right)).astype(np.float32)
+
+
+def make(cfg: int, out_path: str, verbose: bool = True) -> None:
+    c = CONFIGS[cfg]
+    rng = np.random.default_rng(0xCA5C + cfg)
+    counts = fdgen.table1_counts()
+    fam_p = np.array([counts[k] for k in FAMILIES], np.float64)
+    fam_p /= fam_p.sum()
+    pool = Pool(cfg, c)
+    for _ in range(c["bg_frames"]):
+        pool.add_full_frame()
+    tp_ii, tp_nf = template_variants(cfg, c)
+    stages = []
+    for s, (ns, ps) in enumerate(zip(c["sizes"], c["p"])):
+        if pool.size() < MIN_POOL and stages:
+            partial = oracle.Cascade(fmt_cascade(stages))
+            while pool.size() < MIN_POOL and pool.boot < c["max_boot"]:
+                pool.add_bootstrap_frame(partial)
+        npool = pool.size()
+        if npool:
+            sub_ii, sub_nf = pool.sub_mosaic(rng, N_SUB)
+        sums = [np.zeros(len(g["wins"]), np.float32) for g in pool.groups]
+        tmpl_sum = np.zeros(tp_nf.shape[0], np.float32)
+        stumps = []
+        for j in range(ns):
+            best = None
+            for attempt in range(400):
+                fam = FAMILIES[rng.choice(4, p=fam_p)]
+                rects = fdgen.table1_feature(fam, int(rng.integers(counts[fam])))
+                g_t = mosaic_f(tp_ii, rects) / tp_nf.astype(np.float64)
+                if npool:
+                    g_bg = mosaic_f(sub_ii, rects) / sub_nf.astype(np.float64)
+                    med = float(np.median(g_bg))
+                    q1, q3 = np.percentile(g_bg, [25, 75])
+                    spread = max(float(q3 - q1), 1e-6)
+                else:
+                    med, spread = 0.0, 1.0
+                hi, lo = float(g_t.min()) - med, med - float(g_t.max())
+                score = max(hi, lo) / spread
+                if best is None or score > best[0]:
+                    best = (score, rects, hi >= lo, med, float(g_t.min()), float(g_t.max()))
+                if score > 0.75 and attempt >= 2:
+                    break
+            _score, rects, face_right, med, gmin, gmax = best
+            a = np.float32(rng.uniform(0.2, 1.0))
+            b = np.float32(rng.uniform(0.2, 1.0))
+            if face_right:      # template has large f/nf: face iff f >= theta*nf (right leaf)
+                theta = np.float32(gmin - 0.3 * (gmin - med)) if gmin > med else np.float32(gmin - 0.05)
+                left, right = np.float32(-b), np.float32(a)
+            else:
+                theta = np.float32(gmax + 0.3 * (med - gmax)) if gmax < med else np.float32(gmax + 0.05)
+                left, right = np.float32(a), np.float32(-b)
+            for i, lv in enumerate(pool.leaves(rects, theta, left, right)):
+                sums[i] = (sums[i] + lv).astype(np.float32)
+            tmpl_sum = (tmpl_sum + leaf_of(mosaic_f(tp_ii, rects), tp_nf, theta, left, right)).astype(np.float32)
+            stumps.append((rects, theta, left, right))
+        cap = float(tmpl_sum.min()) - 0.01
+        if npool:
+            allsum = np.concatenate(sums)
+            vals = np.unique(allsum)[::-1]
+            frac = 1.0 - np.searchsorted(np.sort(allsum), vals, side="left") / len(allsum)
+            iq = int(np.argmin(np.abs(frac - ps) - 1e-12 * frac))
+            # half-way to the next lower achievable sum so no window sits on the threshold
+            Tq = float(vals[iq] + vals[iq + 1]) / 2 if iq + 1 < len(vals) else float(vals[iq]) - 0.01
+            T = np.float32(min(Tq, cap))
+            masks = [sm >= T for sm in sums]
+            passed = float(np.concatenate(masks).mean())
+            pool.keep(masks)
+        else:
+            T, passed = np.float32(cap), float("nan")
+        stages.append((T, stumps))
+        if verbose:
+            print(f"cfg{cfg} stage {s:2d}: {ns:3d} stumps, pool {npool:8d} (boot frames {pool.boot:3d}), "
+                  f"pass {passed:.4f} (target {ps}), template min sum {tmpl_sum.min():.3f}, T {float(T):.3f}",
+                  flush=True)
+    with open(out_path, "w") as fh:
+        fh.write("# synthetic paper-shaped cascade written by tools/make_cascades.py (input, not a result)\n")
+        fh.write(fmt_cascade(stages))
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--cfg", type=int, nargs="*", default=[1, 2, 3])
+    ap.add_argument("--out", default=os.path.join(ROOT, "cascades"))
+    a = ap.parse_args()
+    os.makedirs(a.out, exist_ok=True)
+    for cfg in a.cfg:
+        make(cfg, os.path.join(a.out, f"c{cfg}.fdc"))
+
+
+if __name__ == "__main__":
+    main()
