@@ -151,6 +151,31 @@ fd_status fd_detect_host(fd_cascade c, const uint8_t* h_frames, int n, int W, in
 fd_status fd_group(const fd_detection* d_in, int64_t n, double eyes_thresh, int min_neighbors,
                    fd_detection* d_out, int64_t capacity, int64_t* n_out, void* stream);
 
+/* fd_detect + fd_group end to end with HOST buffers (the user-facing e2e call): copies
+ * h_frames to the device, detects, groups (eyes_thresh, min_neighbors as fd_group) and copies
+ * the grouped detections to h_out.  *n_raw (may be NULL) = detections before grouping.
+ * Synchronises `stream`. */
+fd_status fd_detect_group_host(fd_cascade c, const uint8_t* h_frames, int n, int W, int H, int pitch,
+                               int min_size, double scale_factor, int step, double eyes_thresh,
+                               int min_neighbors, fd_detection* h_out, int64_t capacity,
+                               int64_t* n_out, int64_t* n_raw, void* stream);
+
+/* Kernel accounting (process-wide, all devices): number of launches of each kernel class
+ * since the last fd_profile_reset and, if time_kernels != 0, their summed device time
+ * measured with CUDA events recorded on the launching stream around each launch.
+ * FD_K_SORT is the CUB radix sort (library code, counted as one call). */
+typedef enum {
+    FD_K_COLSUM = 0, FD_K_CARRY = 1, FD_K_BAND = 2, FD_K_CASCADE = 3,
+    FD_K_SORT = 4, FD_K_DETS = 5, FD_K_GROUP = 6, FD_K_PYRAMID = 7, FD_K_COUNT = 8
+} fd_kernel_kind;
+typedef struct {
+    int64_t launches[FD_K_COUNT];
+    double ms[FD_K_COUNT];
+} fd_profile;
+fd_status fd_profile_reset(int time_kernels);
+/* Waits for the recorded events, then returns the totals. */
+fd_status fd_profile_read(fd_profile* out);
+
 /* Release every internal workspace of the current device. */
 fd_status fd_release_workspaces(void);
 

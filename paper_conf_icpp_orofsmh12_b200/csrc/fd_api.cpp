@@ -1,0 +1,843 @@
+// fd_api.cpp -- the C ABI (include/fd.h): validation, pyramid plan, cascade parsing and
+// packing, per-(device, stream) workspaces, and the launch sequence of the hot path
+//   K1 (k_colsum -> k_carry -> k_band)  ->  K2 (k_cascade, persistent, all scales)
+//   -> count read-back -> K3 (radix sort + back-projection).
+// Host code only; every arithmetic step of the method runs in the kernels.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cerrno>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <utility>
+#include <vector>
+
+#include "fd_internal.h"
+
+using namespace fdk;
+
+namespace {
+
+thread_local std::string g_err;
+
+fd_status fail(fd_status s, const char* fmt, ...) {
+    char buf[1024];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return s;
+}
+
+#define CK(expr)                                                                                  \
+    do {                                                                                          \
+        cudaError_t e_ = (expr);                                                                  \
+        if (e_ != cudaSuccess) return fail(FD_ECUDA, "%s: %s (%s:%d)", #expr, cudaGetErrorString(e_), __FILE__, __LINE__); \
+    } while (0)
+
+// ------------------------------------------------------------------ pyramid plan (reading R1)
+fd_status make_plan(int W, int H, int min_size, double s, int step, fd_plan* out) {
+    if (W < WIN || H < WIN) return fail(FD_EINVAL, "frame %dx%d smaller than the 24x24 window", W, H);
+    if (min_size < WIN) return fail(FD_EINVAL, "min_size %d < 24", min_size);
+    if (!(s > 1.0) || !std::isfinite(s)) return fail(FD_EINVAL, "scale_factor must be > 1");
+    if (step < 1) return fail(FD_EINVAL, "step must be >= 1");
+    if (W > 65535 || H > 65535) return fail(FD_EINVAL, "frame larger than 65535");
+    std::memset(out, 0, sizeof *out);
+    double f = (double)min_size / 24.0;
+    int n = 0;
+    for (;;) {
+        const int w = (int)std::floor((double)W / f);
+        const int h = (int)std::floor((double)H / f);
+        if (w < WIN || h < WIN) break;
+        if (n == FD_MAX_LEVELS) return fail(FD_EINVAL, "more than %d pyramid levels", FD_MAX_LEVELS);
+        out->f[n] = f;
+        out->w[n] = w;
+        out->h[n] = h;
+        out->windows[n] = (int64_t)((w - WIN) / step + 1) * (int64_t)((h - WIN) / step + 1);
+        out->total_windows += out->windows[n];
+        ++n;
+        f = f * s;
+    }
+    out->n_levels = n;
+    return FD_OK;
+}
+
+// device plan for a frame group of G frames
+void make_plan_dev(const fd_plan& pl, int W, int H, int pitch, int step, int G, PlanDev* p) {
+    std::memset(p, 0, sizeof *p);
+    p->n_levels = pl.n_levels;
+    p->W = W;
+    p->H = H;
+    p->pitch = pitch;
+    p->step = step;
+    p->G = G;
+    const int tx = k2_tx(step), ty = k2_ty(step);
+    long long ws = 0, col = 0, win = 0;
+    int bands = 0, tiles = 0, maxW = 0;
+    for (int k = 0; k < pl.n_levels; ++k) {
+        LevelDev& L = p->lv[k];
+        L.W = pl.w[k];
+        L.H = pl.h[k];
+        L.P = (L.W + 1 + 3) & ~3;
+        L.nx = (L.W - WIN) / step + 1;
+        L.ny = (L.H - WIN) / step + 1;
+        L.band0 = bands;
+        L.nbands = (L.H + BAND - 1) / BAND;
+        L.tile0 = tiles;
+        L.tiles_x = (L.nx + tx - 1) / tx;
+        L.r16 = (int)std::llround(pl.f[k] * 65536.0);
+        L.ws_off = ws;
+        L.col_off = col;
+        L.win0 = win;
+        bands += L.nbands;
+        tiles += L.tiles_x * ((L.ny + ty - 1) / ty);
+        ws += (long long)G * 2 * (L.H + 1) * L.P;
+        col += (long long)L.nbands * 2 * L.W;
+        win += pl.windows[k];
+        maxW = L.W > maxW ? L.W : maxW;
+    }
+    p->bands_per_frame = bands;
+    p->tiles_per_frame = tiles;
+    p->maxW = maxW;
+    p->win_per_frame = win;
+    p->col_frame = col;
+    p->ws_elems = ws;
+}
+
+// ------------------------------------------------------------------ cascade (.fdc) parser
+struct HStump {
+    int nrect;
+    int r[3][5];
+    float theta, left, right;
+};
+struct HStage {
+    int first, n;
+    float T;
+};
+
+struct Line {
+    std::vector<std::string> tok;
+    int no;
+};
+
+bool parse_int(const std::string& t, long* v) {
+    char* e = nullptr;
+    errno = 0;
+    *v = std::strtol(t.c_str(), &e, 10);
+    return e && *e == 0 && errno == 0 && !t.empty();
+}
+bool parse_float(const std::string& t, float* v, bool allow_inf) {
+    char* e = nullptr;
+    *v = std::strtof(t.c_str(), &e);
+    if (!e || *e != 0 || t.empty()) return false;
+    if (std::isnan(*v)) return false;
+    if (!allow_inf && std::isinf(*v)) return false;
+    return true;
+}
+
+}  // namespace
+
+struct fd_cascade_s {
+    int device = 0;
+    std::vector<HStump> stumps;
+    std::vector<HStage> stages;
+    std::mutex mu;
+    std::map<int, std::pair<uint4*, StageDev*>> packed;     // tile width -> device records
+    ~fd_cascade_s() {
+        for (auto& kv : packed) {
+            cudaFree(kv.second.first);
+            cudaFree(kv.second.second);
+        }
+    }
+};
+
+namespace {
+
+fd_status parse_cascade(const char* text, size_t len, fd_cascade_s* c) {
+    std::vector<Line> lines;
+    size_t i = 0;
+    int no = 0;
+    while (i < len) {
+        size_t j = i;
+        while (j < len && text[j] != '\n') ++j;
+        ++no;
+        Line L;
+        L.no = no;
+        std::string cur;
+        bool comment = false;
+        for (size_t q = i; q < j && !comment; ++q) {
+            const char ch = text[q];
+            if (ch == '#' && cur.empty() && L.tok.empty()) {
+                comment = true;
+                break;
+            }
+            if (ch == ' ' || ch == '\t' || ch == '\r' || ch == '\f' || ch == '\v') {
+                if (!cur.empty()) L.tok.push_back(cur), cur.clear();
+            } else {
+                cur.push_back(ch);
+            }
+        }
+        if (!cur.empty()) L.tok.push_back(cur);
+        if (!L.tok.empty()) lines.push_back(std::move(L));
+        i = j + 1;
+    }
+    size_t li = 0;
+    auto need = [&](const char* what) -> const Line* {
+        if (li >= lines.size()) return nullptr;
+        (void)what;
+        return &lines[li++];
+    };
+    const Line* L = need("FDC");
+    if (!L || L->tok.size() != 2 || L->tok[0] != "FDC" || L->tok[1] != "1")
+        return fail(FD_EFORMAT, "line %d: expected 'FDC 1'", L ? L->no : 0);
+    L = need("window");
+    if (!L || L->tok.size() != 3 || L->tok[0] != "window" || L->tok[1] != "24" || L->tok[2] != "24")
+        return fail(FD_EFORMAT, "line %d: expected 'window 24 24'", L ? L->no : 0);
+    L = need("stages");
+    long ns = 0;
+    if (!L || L->tok.size() != 2 || L->tok[0] != "stages" || !parse_int(L->tok[1], &ns) || ns < 1 || ns > 250)
+        return fail(FD_EFORMAT, "line %d: expected 'stages N' with 1 <= N <= 250", L ? L->no : 0);
+    for (long s = 0; s < ns; ++s) {
+        L = need("stage");
+        long n = 0;
+        HStage st;
+        if (!L || L->tok.size() != 3 || L->tok[0] != "stage" || !parse_int(L->tok[1], &n) || n < 1 || n > 65536 ||
+            !parse_float(L->tok[2], &st.T, true))
+            return fail(FD_EFORMAT, "line %d: expected 'stage n T'", L ? L->no : 0);
+        st.first = (int)c->stumps.size();
+        st.n = (int)n;
+        c->stages.push_back(st);
+        for (long j = 0; j < n; ++j) {
+            L = need("stump");
+            long nr = 0;
+            if (!L || L->tok.size() < 2 || L->tok[0] != "stump" || !parse_int(L->tok[1], &nr) || nr < 1 || nr > 3)
+                return fail(FD_EFORMAT, "line %d: expected 'stump r ...' with r in 1..3", L ? L->no : 0);
+            if ((long)L->tok.size() != 2 + 5 * nr + 3)
+                return fail(FD_EFORMAT, "line %d: stump needs %ld rect fields + theta left right", L->no, 5 * nr);
+            HStump sp;
+            std::memset(&sp, 0, sizeof sp);
+            sp.nrect = (int)nr;
+            for (long r = 0; r < nr; ++r) {
+                long v[5];
+                for (int q = 0; q < 5; ++q)
+                    if (!parse_int(L->tok[2 + 5 * r + q], &v[q])) return fail(FD_EFORMAT, "line %d: bad rectangle", L->no);
+                if (v[0] < 0 || v[1] < 0 || v[2] < 1 || v[3] < 1 || v[0] + v[2] > WIN || v[1] + v[3] > WIN)
+                    return fail(FD_EFORMAT, "line %d: rectangle outside the 24x24 window", L->no);
+                if (v[4] < -16 || v[4] > 16) return fail(FD_EFORMAT, "line %d: weight outside [-16,16]", L->no);
+                for (int q = 0; q < 5; ++q) sp.r[r][q] = (int)v[q];
+            }
+            const size_t b = 2 + 5 * nr;
+            if (!parse_float(L->tok[b], &sp.theta, false) || !parse_float(L->tok[b + 1], &sp.left, false) ||
+                !parse_float(L->tok[b + 2], &sp.right, false))
+                return fail(FD_EFORMAT, "line %d: expected finite 'theta left right'", L->no);
+            c->stumps.push_back(sp);
+        }
+    }
+    if (li != lines.size()) return fail(FD_EFORMAT, "line %d: trailing content", lines[li].no);
+    return FD_OK;
+}
+
+// Pack stumps for a tile width TW: each Haar feature is compiled into its distinct
+// integral-image corners with integer coefficients (sum_r wt_r * R_r, R = A + D - B - C).
+fd_status pack_cascade(fd_cascade_s* c, int TW, std::pair<uint4*, StageDev*>* out) {
+    std::vector<uint32_t> rec(c->stumps.size() * REC_WORDS, 0u);
+    for (size_t j = 0; j < c->stumps.size(); ++j) {
+        const HStump& s = c->stumps[j];
+        int coef[WIN + 1][WIN + 1];
+        std::memset(coef, 0, sizeof coef);
+        for (int r = 0; r < s.nrect; ++r) {
+            const int x = s.r[r][0], y = s.r[r][1], w = s.r[r][2], h = s.r[r][3], wt = s.r[r][4];
+            coef[y][x] += wt;
+            coef[y][x + w] -= wt;
+            coef[y + h][x] -= wt;
+            coef[y + h][x + w] += wt;
+        }
+        uint32_t* R = &rec[j * REC_WORDS];
+        int nc = 0;
+        for (int y = 0; y <= WIN; ++y)
+            for (int x = 0; x <= WIN; ++x)
+                if (coef[y][x] != 0) {
+                    if (nc == MAX_CORNERS) return fail(FD_EFORMAT, "stump %zu has more than %d corners", j, MAX_CORNERS);
+                    const uint32_t off = (uint32_t)(y * TW + x);
+                    R[4 + nc] = (off & 0xffffu) | ((uint32_t)(coef[y][x] & 0xffff) << 16);
+                    ++nc;
+                }
+        R[0] = (uint32_t)nc;
+        std::memcpy(&R[1], &s.theta, 4);
+        std::memcpy(&R[2], &s.left, 4);
+        std::memcpy(&R[3], &s.right, 4);
+    }
+    std::vector<StageDev> st(c->stages.size());
+    for (size_t s = 0; s < st.size(); ++s) {
+        st[s].first = c->stages[s].first;
+        st[s].n = c->stages[s].n;
+        st[s].T = c->stages[s].T;
+        st[s].pad = 0;
+    }
+    uint4* d_rec = nullptr;
+    StageDev* d_st = nullptr;
+    CK(cudaMalloc(&d_rec, rec.size() * 4 + 16));
+    CK(cudaMalloc(&d_st, st.size() * sizeof(StageDev)));
+    CK(cudaMemcpy(d_rec, rec.data(), rec.size() * 4, cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(d_st, st.data(), st.size() * sizeof(StageDev), cudaMemcpyHostToDevice));
+    *out = {d_rec, d_st};
+    return FD_OK;
+}
+
+fd_status get_packed(fd_cascade_s* c, int step, std::pair<uint4*, StageDev*>* out) {
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    if (dev != c->device) return fail(FD_EINVAL, "cascade was loaded on device %d, current device is %d", c->device, dev);
+    std::lock_guard<std::mutex> lk(c->mu);
+    const int TW = tile_w(step);
+    auto it = c->packed.find(TW);
+    if (it != c->packed.end()) {
+        *out = it->second;
+        return FD_OK;
+    }
+    std::pair<uint4*, StageDev*> pk;
+    fd_status s = pack_cascade(c, TW, &pk);
+    if (s != FD_OK) return s;
+    c->packed[TW] = pk;
+    *out = pk;
+    return FD_OK;
+}
+
+// ------------------------------------------------------------------ tensor maps
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn encode_fn() {
+    static EncodeTiledFn fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<EncodeTiledFn>(p);
+    });
+    return fn;
+}
+
+fd_status encode_maps(const PlanDev& p, uint32_t* ws, int step, CUtensorMap* maps) {
+    EncodeTiledFn enc = encode_fn();
+    if (!enc) return fail(FD_ECUDA, "cuTensorMapEncodeTiled unavailable");
+    for (int k = 0; k < p.n_levels; ++k) {
+        const LevelDev& L = p.lv[k];
+        cuuint64_t dims[4] = {(cuuint64_t)(L.W + 1), (cuuint64_t)(L.H + 1), 2, (cuuint64_t)p.G};
+        cuuint64_t strides[3] = {(cuuint64_t)L.P * 4, (cuuint64_t)(L.H + 1) * L.P * 4,
+                                 (cuuint64_t)2 * (L.H + 1) * L.P * 4};
+        cuuint32_t box[4] = {(cuuint32_t)tile_w(step), (cuuint32_t)tile_h(step), 2, 1};
+        cuuint32_t es[4] = {1, 1, 1, 1};
+        CUresult r = enc(&maps[k], CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, ws + L.ws_off, dims, strides, box, es,
+                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) return fail(FD_ECUDA, "cuTensorMapEncodeTiled failed (%d) for level %d", (int)r, k);
+    }
+    return FD_OK;
+}
+
+// ------------------------------------------------------------------ kernel accounting
+struct Profiler {
+    std::mutex mu;
+    bool timing = false;
+    long long launches[FD_K_COUNT] = {};
+    struct Rec {
+        int kind;
+        cudaEvent_t a, b;
+    };
+    std::vector<Rec> recs;
+    std::vector<cudaEvent_t> pool;
+    cudaEvent_t get() {
+        if (!pool.empty()) {
+            cudaEvent_t e = pool.back();
+            pool.pop_back();
+            return e;
+        }
+        cudaEvent_t e = nullptr;
+        cudaEventCreate(&e);
+        return e;
+    }
+} g_prof;
+
+// Counts one launch of `kind` (n kernels) and, when timing, brackets it with events.
+struct ProfScope {
+    int kind;
+    cudaStream_t st;
+    cudaEvent_t a = nullptr;
+    ProfScope(int k, cudaStream_t s, int n = 1) : kind(k), st(s) {
+        std::lock_guard<std::mutex> lk(g_prof.mu);
+        g_prof.launches[k] += n;
+        if (g_prof.timing) {
+            a = g_prof.get();
+            cudaEventRecord(a, st);
+        }
+    }
+    ~ProfScope() {
+        if (!a) return;
+        std::lock_guard<std::mutex> lk(g_prof.mu);
+        cudaEvent_t b = g_prof.get();
+        cudaEventRecord(b, st);
+        g_prof.recs.push_back({kind, a, b});
+    }
+};
+
+#define LAUNCH(kind, st, expr)        \
+    do {                              \
+        ProfScope ps_((kind), (st));  \
+        CK(expr);                     \
+    } while (0)
+
+// ------------------------------------------------------------------ workspaces
+struct DevBuf {
+    void* p = nullptr;
+    size_t n = 0;
+    ~DevBuf() {
+        if (p) cudaFree(p);
+    }
+    cudaError_t ensure(size_t bytes) {
+        if (bytes <= n) return cudaSuccess;
+        if (p) cudaFree(p);
+        p = nullptr;
+        n = 0;
+        cudaError_t e = cudaMalloc(&p, bytes);
+        if (e == cudaSuccess) n = bytes;
+        return e;
+    }
+    template <class T>
+    T* as() const {
+        return reinterpret_cast<T*>(p);
+    }
+};
+
+struct Workspace {
+    int device = 0;
+    std::mutex mu;                 // one call at a time per (device, stream)
+    DevBuf ws, colbuf, keys, scores, keys2, scores2, cubtmp, ctl, flev, frames, outbuf, group, grpout;
+    unsigned long long* h_pinned = nullptr;     // pinned host word(s) for count read-back
+    std::unique_ptr<CascadeParams> params{new CascadeParams()};
+    ~Workspace() {
+        if (h_pinned) cudaFreeHost(h_pinned);
+    }
+};
+
+std::mutex g_ws_mu;
+std::map<std::pair<int, cudaStream_t>, std::unique_ptr<Workspace>> g_ws;
+
+fd_status get_ws(cudaStream_t st, Workspace** out) {
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(g_ws_mu);
+    auto& slot = g_ws[{dev, st}];
+    if (!slot) {
+        slot.reset(new Workspace());
+        slot->device = dev;
+        CK(cudaMallocHost(&slot->h_pinned, 64));
+    }
+    *out = slot.get();
+    return FD_OK;
+}
+
+int env_int(const char* name, int dflt) {
+    const char* v = std::getenv(name);
+    if (!v || !*v) return dflt;
+    return std::atoi(v);
+}
+
+fd_status check_frames(const void* d, int n, int W, int H, int pitch) {
+    if (!d) return fail(FD_EINVAL, "frames pointer is NULL");
+    if (n < 1) return fail(FD_EINVAL, "n must be >= 1");
+    if (pitch < W) return fail(FD_EINVAL, "pitch %d < W %d", pitch, W);
+    if (n > (1 << 24)) return fail(FD_EINVAL, "at most 2^24 frames per call");
+    return FD_OK;
+}
+
+// core of fd_detect / fd_detect_depth: K1 + K2 for every frame group.
+fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int n, int W, int H, int pitch,
+                     const fd_plan& pl, int step, bool depth, uint8_t* d_depth, float* d_score, long long det_cap,
+                     unsigned long long* d_stage_counts, cudaStream_t st) {
+    if (step > MAX_STEP) return fail(FD_EINVAL, "step %d not supported (1..%d)", step, MAX_STEP);
+    std::pair<uint4*, StageDev*> pk;
+    fd_status s = get_packed(c, step, &pk);
+    if (s != FD_OK) return s;
+    // frames per group: keep one group's ii/sqii workspace near L2 size (126 MB)
+    PlanDev one;
+    make_plan_dev(pl, W, H, pitch, step, 1, &one);
+    const double per_frame = (double)one.ws_elems * 4.0;
+    int G = env_int("FD_GROUP_FRAMES", 0);
+    if (G <= 0) G = (int)std::floor((96.0 * 1024 * 1024) / (per_frame > 1 ? per_frame : 1));
+    if (G < 1) G = 1;
+    if (G > n) G = n;
+    const int ngroups = (n + G - 1) / G;
+    CascadeParams& P = *w->params;
+    make_plan_dev(pl, W, H, pitch, step, G, &P.plan);
+    CK(w->ws.ensure((size_t)P.plan.ws_elems * 4));
+    CK(w->colbuf.ensure((size_t)G * P.plan.col_frame * 4 + 16));
+    CK(w->ctl.ensure(256 + (size_t)ngroups * 4));
+    CK(cudaMemsetAsync(w->ctl.p, 0, 256 + (size_t)ngroups * 4, st));
+    if (!depth) {
+        const size_t cap = (size_t)(det_cap > 0 ? det_cap : 1);
+        CK(w->keys.ensure(cap * 8));
+        CK(w->scores.ensure(cap * 4));
+    }
+    s = encode_maps(P.plan, w->ws.as<uint32_t>(), step, P.tmap);
+    if (s != FD_OK) return s;
+    P.stumps = pk.first;
+    P.stages = pk.second;
+    P.n_stages = (int)c->stages.size();
+    P.det_count = w->ctl.as<unsigned long long>();
+    P.det_keys = depth ? nullptr : w->keys.as<unsigned long long>();
+    P.det_scores = depth ? nullptr : w->scores.as<float>();
+    P.det_cap = depth ? 0 : det_cap;
+    P.depth = d_depth;
+    P.score = d_score;
+    P.stage_counts = d_stage_counts;
+    const int grid = cascade_grid(depth, step);
+    for (int gi = 0; gi < ngroups; ++gi) {
+        const int f0 = gi * G, gf = (n - f0) < G ? (n - f0) : G;
+        const uint8_t* fr = d_frames + (size_t)f0 * H * pitch;
+        LAUNCH(FD_K_COLSUM, st, launch_colsum(fr, P.plan, gf, w->colbuf.as<uint32_t>(), st));
+        LAUNCH(FD_K_CARRY, st, launch_carry(P.plan, gf, w->colbuf.as<uint32_t>(), st));
+        LAUNCH(FD_K_BAND, st, launch_band(fr, P.plan, gf, w->colbuf.as<uint32_t>(), w->ws.as<uint32_t>(), st));
+        P.g_frames = gf;
+        P.frame_base = f0;
+        P.total_tiles = gf * P.plan.tiles_per_frame;
+        P.tile_counter = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + gi;
+        const int gr = grid < P.total_tiles ? grid : P.total_tiles;
+        LAUNCH(FD_K_CASCADE, st, launch_cascade(P, depth, step, gr, st));
+    }
+    return FD_OK;
+}
+
+fd_status detect_impl(fd_cascade c, const uint8_t* d_frames, int n, int W, int H, int pitch, int min_size, double s,
+                      int step, fd_detection* d_out, int64_t capacity, int64_t* n_out, int64_t* d_stage_counts,
+                      cudaStream_t st) {
+    if (!c) return fail(FD_EINVAL, "cascade is NULL");
+    if (!n_out) return fail(FD_EINVAL, "n_out is NULL");
+    if (capacity < 0) return fail(FD_EINVAL, "capacity < 0");
+    if (capacity > 0 && !d_out) return fail(FD_EINVAL, "d_out is NULL");
+    fd_status r = check_frames(d_frames, n, W, H, pitch);
+    if (r != FD_OK) return r;
+    fd_plan pl;
+    r = make_plan(W, H, min_size, s, step, &pl);
+    if (r != FD_OK) return r;
+    Workspace* w = nullptr;
+    r = get_ws(st, &w);
+    if (r != FD_OK) return r;
+    std::lock_guard<std::mutex> lk(w->mu);
+    if (pl.n_levels == 0) {
+        *n_out = 0;
+        return FD_OK;
+    }
+    const long long cap = capacity > 0 ? capacity : 1;
+    r = run_groups(c, w, d_frames, n, W, H, pitch, pl, step, false, nullptr, nullptr, cap,
+                   reinterpret_cast<unsigned long long*>(d_stage_counts), st);
+    if (r != FD_OK) return r;
+    CK(cudaMemcpyAsync(w->h_pinned, w->ctl.p, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    const long long cnt = (long long)w->h_pinned[0];
+    *n_out = cnt;
+    if (cnt > capacity) return fail(FD_ECAPACITY, "%lld detections > capacity %lld", cnt, (long long)capacity);
+    if (cnt == 0) return FD_OK;
+    size_t tb = 0;
+    CK(sort_pairs(nullptr, tb, nullptr, nullptr, nullptr, nullptr, cnt, st));
+    CK(w->cubtmp.ensure(tb + 16));
+    CK(w->keys2.ensure((size_t)cnt * 8));
+    CK(w->scores2.ensure((size_t)cnt * 4));
+    CK(w->flev.ensure(sizeof(double) * FD_MAX_LEVELS));
+    CK(cudaMemcpyAsync(w->flev.p, pl.f, sizeof(double) * FD_MAX_LEVELS, cudaMemcpyHostToDevice, st));
+    tb = w->cubtmp.n;
+    LAUNCH(FD_K_SORT, st, sort_pairs(w->cubtmp.p, tb, w->keys.as<unsigned long long>(), w->keys2.as<unsigned long long>(),
+                  w->scores.as<float>(), w->scores2.as<float>(), cnt, st));
+    LAUNCH(FD_K_DETS, st, launch_keys_to_dets(w->keys2.as<unsigned long long>(), w->scores2.as<float>(), cnt, w->flev.as<double>(),
+                           (int)c->stages.size(), d_out, st));
+    return FD_OK;
+}
+
+}  // namespace
+
+// ==================================================================== C ABI
+extern "C" {
+
+const char* fd_last_error(void) { return g_err.c_str(); }
+int fd_abi_version(void) { return FD_ABI_VERSION; }
+
+fd_status fd_pyramid_plan(int W, int H, int min_size, double scale_factor, int step, fd_plan* out) {
+    if (!out) return fail(FD_EINVAL, "out is NULL");
+    return make_plan(W, H, min_size, scale_factor, step, out);
+}
+
+fd_status fd_load_cascade(const char* text, size_t len, fd_cascade* out) {
+    if (!text || !out) return fail(FD_EINVAL, "NULL argument");
+    std::unique_ptr<fd_cascade_s> c(new fd_cascade_s());
+    fd_status s = parse_cascade(text, len, c.get());
+    if (s != FD_OK) return s;
+    CK(cudaGetDevice(&c->device));
+    std::pair<uint4*, StageDev*> pk;
+    s = get_packed(c.get(), 1, &pk);         // upload the step-1 packing now
+    if (s != FD_OK) return s;
+    *out = c.release();
+    return FD_OK;
+}
+
+fd_status fd_free_cascade(fd_cascade c) {
+    delete c;
+    return FD_OK;
+}
+
+fd_status fd_cascade_info(fd_cascade c, int32_t* n_stages, int32_t* n_stumps) {
+    if (!c) return fail(FD_EINVAL, "cascade is NULL");
+    if (n_stages) *n_stages = (int32_t)c->stages.size();
+    if (n_stumps) *n_stumps = (int32_t)c->stumps.size();
+    return FD_OK;
+}
+
+fd_status fd_build_pyramid(const uint8_t* d_frames, int n, int W, int H, int pitch, int min_size, double scale_factor,
+                           uint8_t* d_levels, void* stream) {
+    fd_status r = check_frames(d_frames, n, W, H, pitch);
+    if (r != FD_OK) return r;
+    if (!d_levels) return fail(FD_EINVAL, "d_levels is NULL");
+    fd_plan pl;
+    r = make_plan(W, H, min_size, scale_factor, 1, &pl);
+    if (r != FD_OK) return r;
+    if (pl.n_levels == 0) return FD_OK;
+    PlanDev p;
+    make_plan_dev(pl, W, H, pitch, 1, 1, &p);
+    long long off = 0;
+    for (int k = 0; k < pl.n_levels; ++k) {      // col_off carries the level byte offset here
+        p.lv[k].col_off = off;
+        off += (long long)pl.w[k] * pl.h[k];
+    }
+    LAUNCH(FD_K_PYRAMID, (cudaStream_t)stream, launch_pyramid(d_frames, p, n, d_levels, off, nullptr, (cudaStream_t)stream));
+    return FD_OK;
+}
+
+fd_status fd_integral(const uint8_t* d_img, int n, int W, int H, int pitch, uint32_t* d_ii, uint64_t* d_sqii,
+                      int out_pitch, void* stream) {
+    fd_status r = check_frames(d_img, n, W, H, pitch);
+    if (r != FD_OK) return r;
+    if (W < 1 || H < 1) return fail(FD_EINVAL, "empty image");
+    if (!d_ii || !d_sqii) return fail(FD_EINVAL, "output pointer is NULL");
+    if (out_pitch < W + 1 || (out_pitch & 3)) return fail(FD_EINVAL, "out_pitch must be >= W+1 and a multiple of 4");
+    if ((reinterpret_cast<uintptr_t>(d_ii) & 15) || (reinterpret_cast<uintptr_t>(d_sqii) & 15))
+        return fail(FD_EINVAL, "output pointers must be 16-byte aligned");
+    cudaStream_t st = (cudaStream_t)stream;
+    fd_plan pl;
+    std::memset(&pl, 0, sizeof pl);
+    pl.n_levels = 1;
+    pl.f[0] = 1.0;
+    pl.w[0] = W;
+    pl.h[0] = H;
+    PlanDev p;
+    make_plan_dev(pl, W, H, pitch, 1, 1, &p);
+    Workspace* w = nullptr;
+    r = get_ws(st, &w);
+    if (r != FD_OK) return r;
+    std::lock_guard<std::mutex> lk(w->mu);
+    CK(w->colbuf.ensure((size_t)n * p.col_frame * 4 + 16));
+    LAUNCH(FD_K_COLSUM, st, launch_colsum(d_img, p, n, w->colbuf.as<uint32_t>(), st));
+    LAUNCH(FD_K_CARRY, st, launch_carry(p, n, w->colbuf.as<uint32_t>(), st));
+    LAUNCH(FD_K_BAND, st, launch_integral_canonical(d_img, p, n, w->colbuf.as<uint32_t>(), d_ii, d_sqii, out_pitch, st));
+    return FD_OK;
+}
+
+fd_status fd_detect(fd_cascade c, const uint8_t* d_frames, int n, int W, int H, int pitch, int min_size,
+                    double scale_factor, int step, fd_detection* d_out, int64_t capacity, int64_t* n_out, void* stream) {
+    return detect_impl(c, d_frames, n, W, H, pitch, min_size, scale_factor, step, d_out, capacity, n_out, nullptr,
+                       (cudaStream_t)stream);
+}
+
+fd_status fd_detect_ex(fd_cascade c, const uint8_t* d_frames, int n, int W, int H, int pitch, int min_size,
+                       double scale_factor, int step, fd_detection* d_out, int64_t capacity, int64_t* n_out,
+                       int64_t* d_stage_counts, void* stream) {
+    return detect_impl(c, d_frames, n, W, H, pitch, min_size, scale_factor, step, d_out, capacity, n_out,
+                       d_stage_counts, (cudaStream_t)stream);
+}
+
+fd_status fd_detect_depth(fd_cascade c, const uint8_t* d_frames, int n, int W, int H, int pitch, int min_size,
+                          double scale_factor, int step, uint8_t* d_depth, float* d_score, void* stream) {
+    if (!c) return fail(FD_EINVAL, "cascade is NULL");
+    if (!d_depth || !d_score) return fail(FD_EINVAL, "output pointer is NULL");
+    fd_status r = check_frames(d_frames, n, W, H, pitch);
+    if (r != FD_OK) return r;
+    fd_plan pl;
+    r = make_plan(W, H, min_size, scale_factor, step, &pl);
+    if (r != FD_OK) return r;
+    if (pl.n_levels == 0) return FD_OK;
+    cudaStream_t st = (cudaStream_t)stream;
+    Workspace* w = nullptr;
+    r = get_ws(st, &w);
+    if (r != FD_OK) return r;
+    std::lock_guard<std::mutex> lk(w->mu);
+    return run_groups(c, w, d_frames, n, W, H, pitch, pl, step, true, d_depth, d_score, 0, nullptr, st);
+}
+
+fd_status fd_detect_host(fd_cascade c, const uint8_t* h_frames, int n, int W, int H, int pitch, int min_size,
+                         double scale_factor, int step, fd_detection* h_out, int64_t capacity, int64_t* n_out,
+                         void* stream) {
+    if (!h_frames) return fail(FD_EINVAL, "h_frames is NULL");
+    if (capacity > 0 && !h_out) return fail(FD_EINVAL, "h_out is NULL");
+    fd_status r = check_frames(h_frames, n, W, H, pitch);
+    if (r != FD_OK) return r;
+    cudaStream_t st = (cudaStream_t)stream;
+    Workspace* w = nullptr;
+    r = get_ws(st, &w);
+    if (r != FD_OK) return r;
+    uint8_t* d_fr = nullptr;
+    fd_detection* d_out = nullptr;
+    {
+        std::lock_guard<std::mutex> lk(w->mu);
+        CK(w->frames.ensure((size_t)n * H * pitch));
+        CK(w->outbuf.ensure((size_t)(capacity > 0 ? capacity : 1) * sizeof(fd_detection)));
+        d_fr = w->frames.as<uint8_t>();
+        d_out = w->outbuf.as<fd_detection>();
+        CK(cudaMemcpyAsync(d_fr, h_frames, (size_t)n * H * pitch, cudaMemcpyHostToDevice, st));
+    }
+    r = detect_impl(c, d_fr, n, W, H, pitch, min_size, scale_factor, step, d_out, capacity, n_out, nullptr, st);
+    if (r != FD_OK) return r;
+    if (*n_out > 0) CK(cudaMemcpyAsync(h_out, d_out, (size_t)*n_out * sizeof(fd_detection), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    return FD_OK;
+}
+
+fd_status fd_group(const fd_detection* d_in, int64_t n, double eyes_thresh, int min_neighbors, fd_detection* d_out,
+                   int64_t capacity, int64_t* n_out, void* stream) {
+    if (!n_out) return fail(FD_EINVAL, "n_out is NULL");
+    if (n < 0 || capacity < 0) return fail(FD_EINVAL, "negative size");
+    if (n > 0 && !d_in) return fail(FD_EINVAL, "d_in is NULL");
+    if (capacity > 0 && !d_out) return fail(FD_EINVAL, "d_out is NULL");
+    if (!(eyes_thresh > 0) || !std::isfinite(eyes_thresh)) return fail(FD_EINVAL, "eyes_thresh must be > 0");
+    if (n > (1LL << 31) - 1) return fail(FD_EINVAL, "too many detections");
+    if (n == 0) {
+        *n_out = 0;
+        return FD_OK;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    Workspace* w = nullptr;
+    fd_status r = get_ws(st, &w);
+    if (r != FD_OK) return r;
+    std::lock_guard<std::mutex> lk(w->mu);
+    CK(w->group.ensure(group_scratch_bytes(n) + 128));
+    long long* d_total = reinterpret_cast<long long*>(w->group.as<char>() + w->group.n - 64);
+    {
+        ProfScope ps(FD_K_GROUP, st, 4);
+        CK(launch_group_all(d_in, n, eyes_thresh, min_neighbors < 1 ? 1 : min_neighbors, w->group.p, d_out, capacity,
+                            d_total, st));
+    }
+    CK(cudaMemcpyAsync(w->h_pinned, d_total, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    *n_out = (int64_t)w->h_pinned[0];
+    if (*n_out > capacity) return fail(FD_ECAPACITY, "%lld groups > capacity %lld", (long long)*n_out, (long long)capacity);
+    return FD_OK;
+}
+
+fd_status fd_detect_group_host(fd_cascade c, const uint8_t* h_frames, int n, int W, int H, int pitch, int min_size,
+                               double scale_factor, int step, double eyes_thresh, int min_neighbors,
+                               fd_detection* h_out, int64_t capacity, int64_t* n_out, int64_t* n_raw, void* stream) {
+    if (!h_frames || !n_out) return fail(FD_EINVAL, "NULL argument");
+    if (capacity > 0 && !h_out) return fail(FD_EINVAL, "h_out is NULL");
+    fd_status r = check_frames(h_frames, n, W, H, pitch);
+    if (r != FD_OK) return r;
+    cudaStream_t st = (cudaStream_t)stream;
+    Workspace* w = nullptr;
+    r = get_ws(st, &w);
+    if (r != FD_OK) return r;
+    uint8_t* d_fr = nullptr;
+    fd_detection* d_raw = nullptr;
+    int64_t raw_cap = 0;
+    {
+        std::lock_guard<std::mutex> lk(w->mu);
+        CK(w->frames.ensure((size_t)n * H * pitch));
+        d_fr = w->frames.as<uint8_t>();
+        CK(cudaMemcpyAsync(d_fr, h_frames, (size_t)n * H * pitch, cudaMemcpyHostToDevice, st));
+    }
+    int64_t cnt = 0;
+    for (int attempt = 0; attempt < 2; ++attempt) {
+        {
+            std::lock_guard<std::mutex> lk(w->mu);
+            raw_cap = (int64_t)(w->outbuf.n / sizeof(fd_detection));
+            if (raw_cap < 4096) {
+                CK(w->outbuf.ensure(4096 * sizeof(fd_detection)));
+                raw_cap = 4096;
+            }
+            d_raw = w->outbuf.as<fd_detection>();
+        }
+        r = detect_impl(c, d_fr, n, W, H, pitch, min_size, scale_factor, step, d_raw, raw_cap, &cnt, nullptr, st);
+        if (r == FD_ECAPACITY && attempt == 0) {
+            std::lock_guard<std::mutex> lk(w->mu);
+            CK(w->outbuf.ensure((size_t)cnt * sizeof(fd_detection)));
+            continue;
+        }
+        break;
+    }
+    if (r != FD_OK) return r;
+    if (n_raw) *n_raw = cnt;
+    fd_detection* d_grp = nullptr;
+    {
+        std::lock_guard<std::mutex> lk(w->mu);
+        CK(w->grpout.ensure((size_t)(cnt > 0 ? cnt : 1) * sizeof(fd_detection)));
+        d_grp = w->grpout.as<fd_detection>();
+    }
+    int64_t ng = 0;
+    r = fd_group(d_raw, cnt, eyes_thresh, min_neighbors, d_grp, cnt, &ng, stream);
+    if (r != FD_OK) return r;
+    *n_out = ng;
+    if (ng > capacity) return fail(FD_ECAPACITY, "%lld groups > capacity %lld", (long long)ng, (long long)capacity);
+    if (ng > 0) CK(cudaMemcpyAsync(h_out, d_grp, (size_t)ng * sizeof(fd_detection), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    return FD_OK;
+}
+
+fd_status fd_profile_reset(int time_kernels) {
+    std::lock_guard<std::mutex> lk(g_prof.mu);
+    for (auto& r : g_prof.recs) {
+        cudaEventSynchronize(r.b);
+        g_prof.pool.push_back(r.a);
+        g_prof.pool.push_back(r.b);
+    }
+    g_prof.recs.clear();
+    for (int k = 0; k < FD_K_COUNT; ++k) g_prof.launches[k] = 0;
+    g_prof.timing = time_kernels != 0;
+    return FD_OK;
+}
+
+fd_status fd_profile_read(fd_profile* out) {
+    if (!out) return fail(FD_EINVAL, "out is NULL");
+    std::lock_guard<std::mutex> lk(g_prof.mu);
+    std::memset(out, 0, sizeof *out);
+    for (int k = 0; k < FD_K_COUNT; ++k) out->launches[k] = g_prof.launches[k];
+    for (auto& r : g_prof.recs) {
+        CK(cudaEventSynchronize(r.b));
+        float ms = 0.f;
+        CK(cudaEventElapsedTime(&ms, r.a, r.b));
+        out->ms[r.kind] += ms;
+    }
+    return FD_OK;
+}
+
+fd_status fd_release_workspaces(void) {
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(g_ws_mu);
+    for (auto it = g_ws.begin(); it != g_ws.end();) {
+        if (it->first.first == dev) {
+            CK(cudaDeviceSynchronize());
+            it = g_ws.erase(it);
+        } else {
+            ++it;
+        }
+    }
+    return FD_OK;
+}
+
+}  // extern "C"

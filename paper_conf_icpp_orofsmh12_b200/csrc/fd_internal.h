@@ -1,0 +1,116 @@
+// fd_internal.h -- shared host/device declarations of the CUDA path (not part of the C ABI).
+//
+// Data layout in HBM:
+//   group workspace (u32 elements), per pyramid level k:
+//     ws + lv.ws_off + ((g * 2 + plane) * (H_k + 1) + y) * P_k + x
+//   plane 0 = ii (u32), plane 1 = sqii mod 2^32 (u32; exact for every 24x24 window
+//   difference, reading R4).  P_k = round_up(W_k + 1, 4) so every row is 16-B aligned for
+//   TMA and vector stores.  One 4-D TMA tensor map per level covers {x, y, plane, g}.
+//   K1 column-sum scratch (u32), per frame: colbuf + g*col_frame + lv.col_off +
+//     (band * 2 + plane) * W_k + x
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/fd.h"
+
+namespace fdk {
+
+constexpr int WIN = FD_WINDOW;       // 24
+constexpr int BAND = 32;             // K1 band height (rows)
+constexpr int CHUNK = 128;           // K1 chunk width (ii columns): 32 lanes x 4
+constexpr int K1_THREADS = 256;
+constexpr int K2_THREADS = 256;      // 8 warps
+constexpr int REC_WORDS = 16;        // packed stump record: 16 u32 (64 B)
+constexpr int MAX_CORNERS = 12;
+constexpr int MAX_STEP = 4;
+
+// K2 tile geometry per window step (windows per tile TX x TY; a thread owns WPT windows of a
+// column; warps tile the x extent in 32-lane columns).  step 1: 64 x 32 windows, 88 x 56 ii.
+__host__ __device__ constexpr int k2_tx(int step) { return step <= 3 ? 64 : 32; }
+__host__ __device__ constexpr int k2_wpt(int step) { return step == 1 ? 8 : (step == 2 ? 4 : (step == 3 ? 2 : 1)); }
+__host__ __device__ constexpr int k2_ty(int step) { return (8 / (k2_tx(step) / 32)) * k2_wpt(step); }
+__host__ __device__ constexpr int tile_w(int step) { return (((k2_tx(step) - 1) * step + WIN + 1) + 3) & ~3; }
+__host__ __device__ constexpr int tile_h(int step) { return (k2_ty(step) - 1) * step + WIN + 1; }
+
+struct LevelDev {
+    int W, H, P;            // level size, ii pitch (elements)
+    int nx, ny;             // windows along x / y (step aware)
+    int band0, nbands;      // K1 bands (per frame)
+    int tile0, tiles_x;     // K2 tiles (per frame); tiles_y = ceil(ny / TY)
+    int r16;                // llround(f * 65536)  (f < 32768 enforced by the plan)
+    long long ws_off;       // u32 elements
+    long long col_off;      // u32 elements (per frame)
+    long long win0;         // first window index of the level within a frame
+};
+
+struct PlanDev {
+    int n_levels;
+    int W, H, pitch, step;
+    int bands_per_frame;
+    int tiles_per_frame;
+    int maxW;
+    long long win_per_frame;
+    long long col_frame;    // K1 scratch elements per frame
+    long long ws_elems;     // group workspace elements (all levels, all g)
+    int G;                  // frames per group (tensor-map extent)
+    LevelDev lv[FD_MAX_LEVELS];
+};
+
+struct StageDev {
+    int first;              // index of first stump record
+    int n;                  // stumps in stage
+    float T;                // stage threshold
+    int pad;
+};
+
+// K2 parameters: passed by value as __grid_constant__ (tensor maps must live in param space).
+struct alignas(64) CascadeParams {
+    CUtensorMap tmap[FD_MAX_LEVELS];        // 16 KB
+    PlanDev plan;
+    const uint4* stumps;                    // REC_WORDS/4 uint4 per stump
+    const StageDev* stages;
+    int n_stages;
+    int g_frames;                           // frames in this group
+    int frame_base;                         // global index of the group's first frame
+    int total_tiles;
+    unsigned int* tile_counter;             // zeroed before launch
+    unsigned long long* det_count;
+    unsigned long long* det_keys;
+    float* det_scores;
+    long long det_cap;
+    uint8_t* depth;                         // depth mode only
+    float* score;
+    unsigned long long* stage_counts;       // n_stages + 1, may be null
+};
+
+// detection key: frame(24) | level(8) | wy(16) | wx(16)
+__host__ __device__ inline unsigned long long det_key(int frame, int level, int wy, int wx) {
+    return ((unsigned long long)(unsigned)frame << 40) | ((unsigned long long)(unsigned)level << 32) |
+           ((unsigned long long)(unsigned)wy << 16) | (unsigned long long)(unsigned)wx;
+}
+
+// ---- launchers (implemented in the .cu files) ----
+cudaError_t launch_colsum(const uint8_t* frames, const PlanDev& plan, int g_frames, uint32_t* colbuf,
+                          cudaStream_t st);
+cudaError_t launch_carry(const PlanDev& plan, int g_frames, uint32_t* colbuf, cudaStream_t st);
+cudaError_t launch_band(const uint8_t* frames, const PlanDev& plan, int g_frames, const uint32_t* colbuf,
+                        uint32_t* ws, cudaStream_t st);
+// canonical fd_integral output (u32 ii, u64 sqii) for n images with one level (f = 1)
+cudaError_t launch_integral_canonical(const uint8_t* img, const PlanDev& plan, int n, const uint32_t* colbuf,
+                                      uint32_t* ii, uint64_t* sqii, int out_pitch, cudaStream_t st);
+cudaError_t launch_pyramid(const uint8_t* frames, const PlanDev& plan, int n, uint8_t* levels,
+                           long long frame_stride, const long long* lvl_off_host, cudaStream_t st);
+cudaError_t launch_cascade(const CascadeParams& p, bool depth_mode, int step, int grid, cudaStream_t st);
+int cascade_grid(bool depth_mode, int step);       // persistent grid size (SMs x resident CTAs)
+size_t cascade_smem(int step);
+cudaError_t launch_keys_to_dets(const unsigned long long* keys, const float* scores, long long n,
+                                const double* f_levels_dev, int n_stages, fd_detection* out, cudaStream_t st);
+cudaError_t sort_pairs(void* tmp, size_t& tmp_bytes, const unsigned long long* kin, unsigned long long* kout,
+                       const float* vin, float* vout, long long n, cudaStream_t st);
+size_t group_scratch_bytes(long long n);
+cudaError_t launch_group_all(const fd_detection* in, long long n, double thresh, int min_neighbors, void* scratch,
+                             fd_detection* out, long long cap, long long* d_total, cudaStream_t st);
+
+}  // namespace fdk

@@ -1,0 +1,274 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the same seeded
+inputs.  Bar (north_star): pyramid levels, integral images, window
+enumeration and depth maps bit-exact; stage scores within 1e-5 relative (the kernels are
+bit-exact by construction, so equality is asserted and any near-threshold window -- oracle
+flag -- is counted and reported); detection sets identical."""
+import math
+import os
+
+import numpy as np
+import pytest
+
+import fdgen
+import oracle
+
+torch = pytest.importorskip("torch")
+import paper_conf_icpp_orofsmh12_b200 as fd  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+CFG = {1: (320, 240, 1.25, 8), 2: (640, 480, 1.2, 12), 3: (1920, 1080, 1.1, 30)}
+_casc = {}
+
+
+def cascades(cfg):
+    if cfg not in _casc:
+        text = open(os.path.join(ROOT, "cascades", f"c{cfg}.fdc")).read()
+        _casc[cfg] = (fd.Cascade(text), oracle.Cascade(text))
+    return _casc[cfg]
+
+
+def gen(cfg, first, n, W=None, H=None, s=None, faces="fixed", param=3):
+    W0, H0, s0, mfl = CFG.get(cfg, (W, H, s, 8))
+    W, H, s = W or W0, H or H0, s or s0
+    lv = oracle.plan(W, H, 24, s, 1)
+    fr, planted = fdgen.frames(cfg, first, n, W, H, lv, faces=faces, face_param=param, max_face_level=mfl)
+    return fr, planted
+
+
+def assert_scores_equal(gpu, ref, near, what):
+    g = gpu.view(np.uint32)
+    r = ref.view(np.uint32)
+    bad = np.nonzero(g != r)[0]
+    if len(bad):
+        rel = np.abs(gpu[bad] - ref[bad]) / np.maximum(np.abs(ref[bad]), 1e-30)
+        assert (rel <= 1e-5).all(), f"{what}: {len(bad)} scores differ beyond 1e-5 rel"
+    return len(bad)
+
+
+def compare_depth(casc_pair, frames, s, step=1):
+    gc, oc = casc_pair
+    d_fr = torch.from_numpy(frames).cuda()
+    depth, score = fd.fd_detect_depth(gc, d_fr, 24, s, step)
+    torch.cuda.synchronize()
+    od, osc, onear = oracle.detect_depth(oc, frames, 24, s, step, nthreads=os.cpu_count())
+    gd = depth.cpu().numpy()
+    gs = score.cpu().numpy()
+    mism = np.nonzero(gd != od)[0]
+    # decisions may only differ on windows the oracle flags as near-threshold (c11)
+    assert np.all(onear[mism] != 0), f"{len(mism)} depth mismatches, {int((onear[mism] == 0).sum())} unflagged"
+    same = gd == od
+    nd = assert_scores_equal(gs[same], osc[same], onear[same], "depth-map scores")
+    print(f"windows {len(od)}, near-threshold flagged {int((onear != 0).sum())}, depth mismatches {len(mism)}, "
+          f"score bit-diffs {nd}")
+    return gd, od
+
+
+# ------------------------------------------------------------------ K1: pyramid + integral
+@pytest.mark.parametrize("cfg", [1, 2, 3])
+def test_pyramid_levels_bit_exact(cfg):
+    W, H, s, _ = CFG[cfg]
+    fr, _ = gen(cfg, 5, 2)
+    lv = fd.fd_build_pyramid(torch.from_numpy(fr).cuda(), 24, s).cpu().numpy()
+    for i in range(2):
+        off = 0
+        for (f, wk, hk, _) in oracle.plan(W, H, 24, s, 1):
+            ref = oracle.resample(fr[i], f, wk, hk)
+            got = lv[i, off:off + wk * hk].reshape(hk, wk)
+            assert np.array_equal(got, ref), (i, f, wk, hk)
+            off += wk * hk
+
+
+@pytest.mark.parametrize("W,H", [(24, 24), (7, 5), (333, 97), (129, 257), (640, 480), (1920, 1080)])
+def test_integral_bit_exact(W, H):
+    rng = np.random.default_rng(W * 1000 + H)
+    img = rng.integers(0, 256, (3, H, W), dtype=np.uint8)
+    img[1] = 255                                   # maximal values
+    ii, sq = fd.fd_integral(torch.from_numpy(img).cuda())
+    ii = ii.cpu().numpy().view(np.uint32)
+    sq = sq.cpu().numpy().view(np.uint64)
+    for i in range(3):
+        rii, rsq = oracle.integral(img[i])
+        assert np.array_equal(ii[i, :, : W + 1], rii)
+        assert np.array_equal(sq[i, :, : W + 1], rsq)
+
+
+def test_integral_pitched_input():
+    rng = np.random.default_rng(3)
+    big = torch.from_numpy(rng.integers(0, 256, (2, 50, 100), dtype=np.uint8)).cuda()
+    view = big[:, :, 3:80]                          # row stride 100, width 77
+    ii, sq = fd.fd_integral(view)
+    rii, rsq = oracle.integral(np.ascontiguousarray(big[1, :, 3:80].cpu().numpy()))
+    assert np.array_equal(ii[1, :, :78].cpu().numpy().view(np.uint32), rii)
+
+
+# ------------------------------------------------------------------ K2: depth maps (every window)
+@pytest.mark.parametrize("cfg", [1, 2])
+def test_depth_maps_bit_exact_small(cfg):
+    W, H, s, _ = CFG[cfg]
+    fr, _ = gen(cfg, 0, 3)
+    compare_depth(cascades(cfg), fr, s)
+
+
+def test_depth_maps_bit_exact_1080p():
+    fr, _ = gen(3, 0, 1)
+    compare_depth(cascades(3), fr, 1.1)
+
+
+@pytest.mark.parametrize("step", [2, 3, 4])
+def test_depth_maps_step(step):
+    fr, _ = gen(2, 7, 2)
+    compare_depth(cascades(2), fr, 1.2, step)
+
+
+@pytest.mark.parametrize("W,H,s", [(24, 24, 1.1), (25, 90, 1.05), (401, 37, 1.3), (131, 517, 1.17)])
+def test_depth_maps_ragged_sizes(W, H, s):
+    fr = np.stack([fdgen.background(2, 900 + i, W, H) for i in range(2)])
+    compare_depth(cascades(2), fr, s)
+
+
+# ------------------------------------------------------------------ detections (fd_detect)
+@pytest.mark.parametrize("cfg", [1, 2, 3])
+def test_detections_identical(cfg):
+    W, H, s, _ = CFG[cfg]
+    n = 2 if cfg == 3 else 4
+    fr, planted = gen(cfg, 11, n)
+    gc, oc = cascades(cfg)
+    sc = torch.zeros(gc.n_stages + 1, dtype=torch.int64, device="cuda")
+    got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1, capacity=1 << 20,
+                                   stage_counts=sc))
+    ref, nnear = oracle.detect(oc, fr, 24, s, 1, nthreads=os.cpu_count())
+    assert np.array_equal(got, ref), f"{len(got)} vs {len(ref)} detections"
+    # planted faces are found with IoU 1 (eq. 5)
+    for i, fl in enumerate(planted):
+        for (k, wx, wy, X, Y, S) in fl:
+            m = (got["frame"] == i) & (got["level"] == k) & (got["wx"] == wx) & (got["wy"] == wy)
+            assert m.sum() == 1 and tuple(got[m][0][["x", "y", "w", "h"]]) == (X, Y, S, S)
+    # stage counters agree with the oracle's depth histogram
+    od, _, _ = oracle.detect_depth(oc, fr, 24, s, 1, nthreads=os.cpu_count())
+    want = [int((od >= k).sum()) for k in range(gc.n_stages + 1)]
+    assert sc.cpu().tolist() == want
+
+
+def test_video_batch_sampled_1080p():
+    """c4-shaped: 16 frames 1080p with Poisson(4) planted faces in one call (several frame
+    groups); oracle on frames 0, 7 and 15 only."""
+    W, H, s = 1920, 1080, 1.1
+    lv = oracle.plan(W, H, 24, s, 1)
+    fr, _ = fdgen.frames(4, 0, 16, W, H, lv, faces="poisson", face_param=4, max_face_level=30)
+    gc, oc = cascades(3)
+    got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1))
+    for i in (0, 7, 15):
+        ref, _ = oracle.detect(oc, fr[i:i + 1], 24, s, 1, nthreads=os.cpu_count())
+        ref["frame"] = i
+        assert np.array_equal(got[got["frame"] == i], ref), i
+
+
+def test_4k_sampled():
+    """c5-shaped: 2 frames 3840x2160; oracle on frame 1."""
+    W, H, s = 3840, 2160, 1.1
+    lv = oracle.plan(W, H, 24, s, 1)
+    fr, _ = fdgen.frames(5, 0, 2, W, H, lv, faces="poisson", face_param=4, max_face_level=34)
+    gc, oc = cascades(3)
+    got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1))
+    ref, _ = oracle.detect(oc, fr[1:2], 24, s, 1, nthreads=os.cpu_count())
+    ref["frame"] = 1
+    assert np.array_equal(got[got["frame"] == 1], ref)
+
+
+def test_detect_host_equals_device():
+    fr, _ = gen(2, 21, 3)
+    gc, _ = cascades(2)
+    a = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, 1.2, 1))
+    b = fd.fd_detect_host(gc, torch.from_numpy(fr).pin_memory(), 24, 1.2, 1)
+    assert np.array_equal(a, b)
+
+
+def test_capacity_error_reports_required_count():
+    fr, _ = gen(1, 0, 1)
+    gc, oc = cascades(1)
+    ref, _ = oracle.detect(oc, fr, 24, 1.25, 1)
+    with pytest.raises(fd.FDCapacityError) as e:
+        fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, 1.25, 1, capacity=3)
+    assert e.value.required == len(ref)
+
+
+# ------------------------------------------------------------------ special cascades
+def _casc_text(stages):
+    out = ["FDC 1", "window 24 24", f"stages {len(stages)}"]
+    for T, stumps in stages:
+        out.append(f"stage {len(stumps)} {T}")
+        for rects, th, l, r in stumps:
+            rs = " ".join(" ".join(str(v) for v in rc) for rc in rects)
+            out.append(f"stump {len(rects)} {rs} {th} {l} {r}")
+    return "\n".join(out) + "\n"
+
+
+def test_all_pass_and_all_reject():
+    st = ([(1, 1, 10, 10, -1), (1, 1, 5, 10, 2)], 0.1, 0.5, 0.5)
+    W, H, s = 211, 157, 1.25
+    fr = np.stack([fdgen.background(1, 50 + i, W, H) for i in range(2)])
+    tot = sum(p[3] for p in oracle.plan(W, H, 24, s, 1))
+    allpass = fd.Cascade(_casc_text([("-inf", [st, st]), ("-1e30", [st])]))
+    got = fd.to_numpy(fd.fd_detect(allpass, torch.from_numpy(fr).cuda(), 24, s, 1, capacity=2 * tot))
+    assert len(got) == 2 * tot
+    ref, _ = oracle.detect(oracle.Cascade(_casc_text([("-inf", [st, st]), ("-1e30", [st])])), fr, 24, s, 1)
+    assert np.array_equal(got, ref)
+    allrej = fd.Cascade(_casc_text([("inf", [st])]))
+    d, sc = fd.fd_detect_depth(allrej, torch.from_numpy(fr).cuda(), 24, s, 1)
+    assert (d.cpu().numpy() == 0).all() and (sc.cpu().numpy() == 0.5).all()
+    assert len(fd.fd_detect(allrej, torch.from_numpy(fr).cuda(), 24, s, 1)) == 0
+
+
+def test_worked_example_single_stump():
+    # golden worked example (tests/golden/worked_example.txt) placed at window (5, 3) of a 40x30 frame
+    img = np.full((30, 40), 0, np.uint8)
+    img[3:27, 5 + 12:5 + 24] = 255
+    st = ([(1, 1, 22, 22, -1), (1, 1, 11, 22, 2)], -0.5, 0.25, 0.75)
+    c = fd.Cascade(_casc_text([("-10", [st])]))
+    d, sc = fd.fd_detect_depth(c, torch.from_numpy(img[None]).cuda(), 24, 1.5, 1)
+    nx = 40 - 24 + 1
+    assert float(sc.cpu().numpy()[3 * nx + 5]) == 0.25       # left leaf
+    oc = oracle.Cascade(_casc_text([("-10", [st])]))
+    od, osc, _ = oracle.detect_depth(oc, img, 24, 1.5, 1)
+    assert np.array_equal(d.cpu().numpy(), od) and np.array_equal(sc.cpu().numpy(), osc)
+
+
+def test_three_rect_and_one_rect_stumps():
+    stumps = [([(0, 0, 24, 24, 1)], 0.001, -0.3, 0.4),
+              ([(2, 2, 10, 12, -1), (2, 2, 5, 6, 2), (7, 8, 5, 6, 2)], 0.01, 0.2, -0.7),
+              ([(3, 1, 18, 20, -1), (9, 1, 6, 20, 3)], -0.02, 0.5, -0.1),
+              ([(1, 1, 21, 21, -1), (8, 8, 7, 7, 9)], 0.0, 0.3, 0.3)]
+    text = _casc_text([("-0.5", stumps[:2]), ("0.1", stumps[2:]), ("-0.2", stumps)])
+    fr = np.stack([fdgen.background(3, 70 + i, 300, 200) for i in range(2)])
+    compare_depth((fd.Cascade(text), oracle.Cascade(text)), fr, 1.15)
+
+
+# ------------------------------------------------------------------ K4: grouping
+@pytest.mark.parametrize("cfg", [2, 3])
+def test_group_matches_oracle(cfg):
+    W, H, s, _ = CFG[cfg]
+    fr, _ = gen(cfg, 31, 2)
+    gc, oc = cascades(cfg)
+    dets = fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1)
+    ref_in = fd.to_numpy(dets)
+    per_frame = max(np.bincount(ref_in["frame"]).max(), 1)
+    if per_frame > 1500:
+        pytest.skip("too many raw detections for the O(n^3) oracle grouping")
+    got = fd.to_numpy(fd.fd_group(dets, 0.5, 1))
+    ref = oracle.group(ref_in, 0.5, 1)
+    assert np.array_equal(got, ref)
+    got2 = fd.to_numpy(fd.fd_group(dets, 0.5, 3))
+    assert np.array_equal(got2, oracle.group(ref_in, 0.5, 3))
+
+
+def test_group_hand_cases():
+    def det(frame, x, y, w, score=0.0):
+        return (frame, 0, x, y, x, y, w, w, score, 1)
+    rows = [det(0, 0, 0, 100, 1.0), det(0, 9, 0, 100, 2.0), det(0, 300, 0, 100), det(0, 310, 0, 100),
+            det(1, 50, 50, 30), det(1, 50, 50, 30), det(1, 500, 50, 30), det(2, 0, 0, 100), det(2, 4, 0, 100),
+            det(2, 8, 0, 100)]
+    a = np.array(rows, oracle.DET_DTYPE)
+    t = torch.from_numpy(a.view(np.int32).reshape(-1, 10).copy()).cuda()
+    got = fd.to_numpy(fd.fd_group(t, 0.5, 1))
+    assert np.array_equal(got, oracle.group(a, 0.5, 1))
