@@ -150,14 +150,21 @@ struct fd_cascade_s {
     std::vector<HStump> stumps;
     std::vector<HStage> stages;
     std::mutex mu;
-    std::map<int, std::pair<uint4*, StageDev*>> packed;     // tile width -> device records
+    struct Packed {
+        uint4* d_rec = nullptr;             // device records (REC_WORDS u32 per stump)
+        StageDev* d_st = nullptr;
+        std::vector<uint32_t> h_rec;        // host copy (first PREC_MAX go to the parameter bank)
+        std::vector<StageDev> h_st;         // host copy (first PSTAGE_MAX go to the parameter bank)
+    };
+    std::map<int, Packed> packed;           // tile width -> packed records
     ~fd_cascade_s() {
         for (auto& kv : packed) {
-            cudaFree(kv.second.first);
-            cudaFree(kv.second.second);
+            cudaFree(kv.second.d_rec);
+            cudaFree(kv.second.d_st);
         }
     }
 };
+using Packed = fd_cascade_s::Packed;
 
 namespace {
 
@@ -247,7 +254,7 @@ fd_status parse_cascade(const char* text, size_t len, fd_cascade_s* c) {
 
 // Pack stumps for a tile width TW: each Haar feature is compiled into its distinct
 // integral-image corners with integer coefficients (sum_r wt_r * R_r, R = A + D - B - C).
-fd_status pack_cascade(fd_cascade_s* c, int TW, std::pair<uint4*, StageDev*>* out) {
+fd_status pack_cascade(fd_cascade_s* c, int TW, Packed* out) {
     std::vector<uint32_t> rec(c->stumps.size() * REC_WORDS, 0u);
     for (size_t j = 0; j < c->stumps.size(); ++j) {
         const HStump& s = c->stumps[j];
@@ -266,8 +273,9 @@ fd_status pack_cascade(fd_cascade_s* c, int TW, std::pair<uint4*, StageDev*>* ou
             for (int x = 0; x <= WIN; ++x)
                 if (coef[y][x] != 0) {
                     if (nc == MAX_CORNERS) return fail(FD_EFORMAT, "stump %zu has more than %d corners", j, MAX_CORNERS);
-                    const uint32_t off = (uint32_t)(y * TW + x);
-                    R[4 + nc] = (off & 0xffffu) | ((uint32_t)(coef[y][x] & 0xffff) << 16);
+                    const uint32_t off = (uint32_t)(y * TW + x) * 4u;     // byte offset in the smem tile
+                    if (off > 0xffffu) return fail(FD_EINVAL, "tile too wide for 16-bit corner offsets");
+                    R[4 + nc] = off | ((uint32_t)(coef[y][x] & 0xffff) << 16);
                     ++nc;
                 }
         R[0] = (uint32_t)nc;
@@ -280,7 +288,10 @@ fd_status pack_cascade(fd_cascade_s* c, int TW, std::pair<uint4*, StageDev*>* ou
         st[s].first = c->stages[s].first;
         st[s].n = c->stages[s].n;
         st[s].T = c->stages[s].T;
-        st[s].pad = 0;
+        int mc = 1;
+        for (int j = st[s].first; j < st[s].first + st[s].n; ++j)
+            mc = (int)rec[(size_t)j * REC_WORDS] > mc ? (int)rec[(size_t)j * REC_WORDS] : mc;
+        st[s].mc = mc;
     }
     uint4* d_rec = nullptr;
     StageDev* d_st = nullptr;
@@ -288,11 +299,14 @@ fd_status pack_cascade(fd_cascade_s* c, int TW, std::pair<uint4*, StageDev*>* ou
     CK(cudaMalloc(&d_st, st.size() * sizeof(StageDev)));
     CK(cudaMemcpy(d_rec, rec.data(), rec.size() * 4, cudaMemcpyHostToDevice));
     CK(cudaMemcpy(d_st, st.data(), st.size() * sizeof(StageDev), cudaMemcpyHostToDevice));
-    *out = {d_rec, d_st};
+    out->d_rec = d_rec;
+    out->d_st = d_st;
+    out->h_rec = std::move(rec);
+    out->h_st = std::move(st);
     return FD_OK;
 }
 
-fd_status get_packed(fd_cascade_s* c, int step, std::pair<uint4*, StageDev*>* out) {
+fd_status get_packed(fd_cascade_s* c, int step, const Packed** out) {
     int dev = 0;
     CK(cudaGetDevice(&dev));
     if (dev != c->device) return fail(FD_EINVAL, "cascade was loaded on device %d, current device is %d", c->device, dev);
@@ -300,14 +314,13 @@ fd_status get_packed(fd_cascade_s* c, int step, std::pair<uint4*, StageDev*>* ou
     const int TW = tile_w(step);
     auto it = c->packed.find(TW);
     if (it != c->packed.end()) {
-        *out = it->second;
+        *out = &it->second;
         return FD_OK;
     }
-    std::pair<uint4*, StageDev*> pk;
+    Packed pk;
     fd_status s = pack_cascade(c, TW, &pk);
     if (s != FD_OK) return s;
-    c->packed[TW] = pk;
-    *out = pk;
+    *out = &(c->packed[TW] = std::move(pk));
     return FD_OK;
 }
 
@@ -423,9 +436,13 @@ struct DevBuf {
 struct Workspace {
     int device = 0;
     std::mutex mu;                 // one call at a time per (device, stream)
-    DevBuf ws, colbuf, keys, scores, keys2, scores2, cubtmp, ctl, flev, frames, outbuf, group, grpout;
+    DevBuf ws, colbuf, keys, scores, keys2, scores2, cubtmp, ctl, flev, frames, outbuf, group, grpout, tmaps, lvbuf;
     unsigned long long* h_pinned = nullptr;     // pinned host word(s) for count read-back
     std::unique_ptr<CascadeParams> params{new CascadeParams()};
+    std::unique_ptr<PlanDev> plan{new PlanDev()};
+    // host staging of tensor maps + level table (kept alive until the async copies run)
+    std::unique_ptr<CUtensorMap[]> h_geo{new CUtensorMap[FD_MAX_LEVELS + (sizeof(LevelDev) * FD_MAX_LEVELS +
+                                                                          sizeof(CUtensorMap) - 1) / sizeof(CUtensorMap)]};
     ~Workspace() {
         if (h_pinned) cudaFreeHost(h_pinned);
     }
@@ -467,22 +484,24 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
                      const fd_plan& pl, int step, bool depth, uint8_t* d_depth, float* d_score, long long det_cap,
                      unsigned long long* d_stage_counts, cudaStream_t st) {
     if (step > MAX_STEP) return fail(FD_EINVAL, "step %d not supported (1..%d)", step, MAX_STEP);
-    std::pair<uint4*, StageDev*> pk;
+    const Packed* pk = nullptr;
     fd_status s = get_packed(c, step, &pk);
     if (s != FD_OK) return s;
-    // frames per group: keep one group's ii/sqii workspace near L2 size (126 MB)
+    // frames per group: one K2 launch per group; larger groups amortise the launch tail
+    // (FD_GROUP_MB workspace budget, default 1536 MB = 16 frames of 1080p; FD_GROUP_FRAMES overrides)
     PlanDev one;
     make_plan_dev(pl, W, H, pitch, step, 1, &one);
     const double per_frame = (double)one.ws_elems * 4.0;
     int G = env_int("FD_GROUP_FRAMES", 0);
-    if (G <= 0) G = (int)std::floor((96.0 * 1024 * 1024) / (per_frame > 1 ? per_frame : 1));
+    const double budget = (double)env_int("FD_GROUP_MB", 1536) * 1024.0 * 1024.0;
+    if (G <= 0) G = (int)std::floor(budget / (per_frame > 1 ? per_frame : 1));
     if (G < 1) G = 1;
     if (G > n) G = n;
     const int ngroups = (n + G - 1) / G;
-    CascadeParams& P = *w->params;
-    make_plan_dev(pl, W, H, pitch, step, G, &P.plan);
-    CK(w->ws.ensure((size_t)P.plan.ws_elems * 4));
-    CK(w->colbuf.ensure((size_t)G * P.plan.col_frame * 4 + 16));
+    PlanDev& PD = *w->plan;
+    make_plan_dev(pl, W, H, pitch, step, G, &PD);
+    CK(w->ws.ensure((size_t)PD.ws_elems * 4));
+    CK(w->colbuf.ensure((size_t)G * PD.col_frame * 4 + 16));
     CK(w->ctl.ensure(256 + (size_t)ngroups * 4));
     CK(cudaMemsetAsync(w->ctl.p, 0, 256 + (size_t)ngroups * 4, st));
     if (!depth) {
@@ -490,11 +509,31 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         CK(w->keys.ensure(cap * 8));
         CK(w->scores.ensure(cap * 4));
     }
-    s = encode_maps(P.plan, w->ws.as<uint32_t>(), step, P.tmap);
+    // tensor maps + level table for K2 (global memory, copied in stream order)
+    std::vector<CUtensorMap> maps((size_t)PD.n_levels);
+    s = encode_maps(PD, w->ws.as<uint32_t>(), step, maps.data());
     if (s != FD_OK) return s;
-    P.stumps = pk.first;
-    P.stages = pk.second;
+    CK(w->tmaps.ensure(sizeof(CUtensorMap) * FD_MAX_LEVELS));
+    CK(w->lvbuf.ensure(sizeof(LevelDev) * FD_MAX_LEVELS));
+    std::memcpy(w->h_geo.get(), maps.data(), sizeof(CUtensorMap) * PD.n_levels);
+    std::memcpy(reinterpret_cast<char*>(w->h_geo.get()) + sizeof(CUtensorMap) * FD_MAX_LEVELS, PD.lv,
+                sizeof(LevelDev) * PD.n_levels);
+    CK(cudaMemcpyAsync(w->tmaps.p, w->h_geo.get(), sizeof(CUtensorMap) * PD.n_levels, cudaMemcpyHostToDevice, st));
+    CK(cudaMemcpyAsync(w->lvbuf.p, reinterpret_cast<char*>(w->h_geo.get()) + sizeof(CUtensorMap) * FD_MAX_LEVELS,
+                       sizeof(LevelDev) * PD.n_levels, cudaMemcpyHostToDevice, st));
+    CascadeParams& P = *w->params;
+    P.tmaps = w->tmaps.as<CUtensorMap>();
+    P.lv = w->lvbuf.as<LevelDev>();
+    P.n_levels = PD.n_levels;
+    P.tiles_per_frame = PD.tiles_per_frame;
+    P.win_per_frame = PD.win_per_frame;
+    P.stumps = pk->d_rec;
+    P.stages = pk->d_st;
     P.n_stages = (int)c->stages.size();
+    P.n_pstumps = (int)std::min<size_t>(c->stumps.size(), (size_t)PREC_MAX);
+    std::memcpy(P.prec, pk->h_rec.data(), (size_t)P.n_pstumps * REC_WORDS * 4);
+    P.n_pstages = (int)std::min<size_t>(c->stages.size(), (size_t)PSTAGE_MAX);
+    std::memcpy(P.pstages, pk->h_st.data(), (size_t)P.n_pstages * sizeof(StageDev));
     P.det_count = w->ctl.as<unsigned long long>();
     P.det_keys = depth ? nullptr : w->keys.as<unsigned long long>();
     P.det_scores = depth ? nullptr : w->scores.as<float>();
@@ -502,16 +541,17 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     P.depth = d_depth;
     P.score = d_score;
     P.stage_counts = d_stage_counts;
+    P.lane_min = env_int("FD_LANE_MIN", 32);
     const int grid = cascade_grid(depth, step);
     for (int gi = 0; gi < ngroups; ++gi) {
         const int f0 = gi * G, gf = (n - f0) < G ? (n - f0) : G;
         const uint8_t* fr = d_frames + (size_t)f0 * H * pitch;
-        LAUNCH(FD_K_COLSUM, st, launch_colsum(fr, P.plan, gf, w->colbuf.as<uint32_t>(), st));
-        LAUNCH(FD_K_CARRY, st, launch_carry(P.plan, gf, w->colbuf.as<uint32_t>(), st));
-        LAUNCH(FD_K_BAND, st, launch_band(fr, P.plan, gf, w->colbuf.as<uint32_t>(), w->ws.as<uint32_t>(), st));
+        LAUNCH(FD_K_COLSUM, st, launch_colsum(fr, PD, gf, w->colbuf.as<uint32_t>(), st));
+        LAUNCH(FD_K_CARRY, st, launch_carry(PD, gf, w->colbuf.as<uint32_t>(), st));
+        LAUNCH(FD_K_BAND, st, launch_band(fr, PD, gf, w->colbuf.as<uint32_t>(), w->ws.as<uint32_t>(), st));
         P.g_frames = gf;
         P.frame_base = f0;
-        P.total_tiles = gf * P.plan.tiles_per_frame;
+        P.total_tiles = gf * PD.tiles_per_frame;
         P.tile_counter = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + gi;
         const int gr = grid < P.total_tiles ? grid : P.total_tiles;
         LAUNCH(FD_K_CASCADE, st, launch_cascade(P, depth, step, gr, st));
@@ -583,7 +623,7 @@ fd_status fd_load_cascade(const char* text, size_t len, fd_cascade* out) {
     fd_status s = parse_cascade(text, len, c.get());
     if (s != FD_OK) return s;
     CK(cudaGetDevice(&c->device));
-    std::pair<uint4*, StageDev*> pk;
+    const Packed* pk = nullptr;
     s = get_packed(c.get(), 1, &pk);         // upload the step-1 packing now
     if (s != FD_OK) return s;
     *out = c.release();

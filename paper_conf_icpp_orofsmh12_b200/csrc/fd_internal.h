@@ -62,19 +62,28 @@ struct StageDev {
     int first;              // index of first stump record
     int n;                  // stumps in stage
     float T;                // stage threshold
-    int pad;
+    int mc;                 // largest corner count of the stage's stumps (records are zero-padded)
 };
 
-// K2 parameters: passed by value as __grid_constant__ (tensor maps must live in param space).
-struct alignas(64) CascadeParams {
-    CUtensorMap tmap[FD_MAX_LEVELS];        // 16 KB
-    PlanDev plan;
-    const uint4* stumps;                    // REC_WORDS/4 uint4 per stump
+// K2 parameters: passed by value as __grid_constant__.  Tensor maps and the level table live
+// in global memory; the parameter block (constant bank 0, <= 32 KB) carries a copy of the first
+// n_pstumps stump records so warp-uniform record reads use the uniform datapath.
+constexpr int PREC_MAX = 440;               // stump records held in parameter space (27.5 KB)
+constexpr int PSTAGE_MAX = 64;              // stage descriptors held in parameter space (1 KB)
+struct alignas(16) CascadeParams {
+    const CUtensorMap* tmaps;               // [n_levels], 64-B aligned, global
+    const LevelDev* lv;                     // [n_levels], global
+    int n_levels;
+    int tiles_per_frame;
+    long long win_per_frame;
+    const uint4* stumps;                    // REC_WORDS/4 uint4 per stump (all stumps)
     const StageDev* stages;
     int n_stages;
+    int n_pstumps;                          // records [0, n_pstumps) are also in prec
     int g_frames;                           // frames in this group
     int frame_base;                         // global index of the group's first frame
     int total_tiles;
+    int lane_min;                           // deep stages with fewer survivors use GL lanes per window
     unsigned int* tile_counter;             // zeroed before launch
     unsigned long long* det_count;
     unsigned long long* det_keys;
@@ -83,6 +92,10 @@ struct alignas(64) CascadeParams {
     uint8_t* depth;                         // depth mode only
     float* score;
     unsigned long long* stage_counts;       // n_stages + 1, may be null
+    int n_pstages;                          // stages [0, n_pstages) are also in pstages
+    int pad0;
+    StageDev pstages[PSTAGE_MAX];
+    uint4 prec[PREC_MAX * (REC_WORDS / 4)];
 };
 
 // detection key: frame(24) | level(8) | wy(16) | wx(16)

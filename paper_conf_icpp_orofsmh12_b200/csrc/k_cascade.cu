@@ -3,18 +3,21 @@
 // Paper: each integral image is cut into n x m chunks, one thread block per
 // chunk, one thread per window; each block stages its chunk (2n x 2m values, eqs. 1-4) in
 // shared memory, then every thread walks the stages with early exit; feature attributes sit
-// in constant memory for warp-uniform broadcast.  B200 design (DESIGN.md "K2"):
+// in constant memory for warp-uniform broadcast (P:L573-594).  B200 design (DESIGN.md "K2"):
 //   * one persistent launch covers every (frame, level, tile) of a frame group -- replaces
 //     the paper's one-kernel-per-scale streams;
 //   * a tile of TX x TY windows needs a (TX+24) x (TY+24) block of ii and sqii: one 4-D TMA
-//     (cp.async.bulk.tensor) per tile, double buffered with mbarriers, prefetching the next
-//     tile while the current one is evaluated;
-//   * stage 1 (94.5% of windows stop there) is evaluated densely: each thread
-//     owns 8 windows of a column, stump records are warp-uniform loads, and each Haar
-//     feature is pre-compiled on the host into its distinct integral-image corners with
-//     integer coefficients (sum_r wt_r*R_r == sum_c coef_c*ii_c exactly, mod 2^32);
-//   * survivors are compacted with warp ballots into a shared-memory queue after every stage
-//     so deeper stages run on full warps (the divergence problem of P:L1228-1258);
+//     (cp.async.bulk.tensor) per tile completing on an mbarrier (optionally double buffered);
+//   * stump records of the first stages live in the kernel-parameter constant bank, so the
+//     warp-uniform record reads go through the uniform datapath (the paper's constant-memory
+//     broadcast); each Haar feature is pre-compiled on the host into its distinct
+//     integral-image corners with integer coefficients (sum_r wt_r*R_r == sum_c coef_c*ii_c
+//     exactly, mod 2^32);
+//   * stage 1 (94.5% of windows stop there) is evaluated densely, each thread
+//     owning WPT windows of a column; survivors are compacted with warp ballots into a
+//     shared-memory queue after every stage so deeper stages run on full warps (the
+//     divergence problem of P:L1228-1258); when few windows survive, GL lanes share a window
+//     (one stump per lane) and the leaves are added in stump order;
 //   * fp32 arithmetic matches the oracle bit for bit: __fmul_rn/__fadd_rn (no FMA
 //     contraction), __int2float_rn, __ll2float_rn, IEEE __fsqrt_rn.
 #include "fd_internal.h"
@@ -59,38 +62,109 @@ __device__ __forceinline__ int corner_word(const uint4& a, const uint4& b, const
     return (int)(j == 0 ? v.x : (j == 1 ? v.y : (j == 2 ? v.z : v.w)));
 }
 
-// One stage for one window: sum_j leaf_j in stump order (oracle c7/c8).
-template <int STEP>
-__device__ __forceinline__ float eval_stage(const uint32_t* __restrict__ T, int b, float nf, const uint4* __restrict__ rec,
-                                            int n) {
-    float sum = 0.0f;
-    for (int j = 0; j < n; ++j) {
-        const uint4 h = __ldg(rec + 4 * j);
-        const uint4 c0 = __ldg(rec + 4 * j + 1), c1 = __ldg(rec + 4 * j + 2), c2 = __ldg(rec + 4 * j + 3);
-        const int nc = (int)h.x;
-        uint32_t f = 0;
+// Record accessors: word4 i of the packed stump records (4 x uint4 per stump).
+struct GlobalRec {                 // global memory, read-only path (lane-varying indices)
+    const uint4* s;
+    __device__ __forceinline__ uint4 operator()(int i) const { return __ldg(s + i); }
+};
+struct ParamRec {                  // kernel-parameter constant bank (warp-uniform indices)
+    const CascadeParams& p;
+    __device__ __forceinline__ uint4 operator()(int i) const { return p.prec[i]; }
+};
+
+// One stump for one window with a compile-time corner count MC >= the stump's corners: the
+// unused corner words are zero (offset 0, coefficient 0), so the loop is branch-free.
+template <int MC, class R>
+__device__ __forceinline__ float eval_stump_mc(const uint32_t* __restrict__ T, int b, float nf, const R& rec, int j) {
+    const uint4 h = rec(4 * j);
+    const uint4 c0 = rec(4 * j + 1);
+    const uint4 c1 = MC > 4 ? rec(4 * j + 2) : make_uint4(0, 0, 0, 0);
+    const uint4 c2 = MC > 8 ? rec(4 * j + 3) : make_uint4(0, 0, 0, 0);
+    uint32_t f = 0;
 #pragma unroll
-        for (int c = 0; c < MAX_CORNERS; ++c) {
-            if (c < nc) {
-                const int w = corner_word(c0, c1, c2, c);
-                f += (uint32_t)(w >> 16) * T[b + (w & 0xffff)];
-            }
-        }
-        const float t = __fmul_rn(__int_as_float((int)h.y), nf);
-        const float leaf = (__int2float_rn((int)f) < t) ? __int_as_float((int)h.z) : __int_as_float((int)h.w);
-        sum = __fadd_rn(sum, leaf);
+    for (int c = 0; c < MC; ++c) {
+        const int w = corner_word(c0, c1, c2, c);
+        f += (uint32_t)(w >> 16) * *reinterpret_cast<const uint32_t*>(reinterpret_cast<const char*>(T + b) + (w & 0xffff));
     }
+    const float t = __fmul_rn(__int_as_float((int)h.y), nf);
+    return (__int2float_rn((int)f) < t) ? __int_as_float((int)h.z) : __int_as_float((int)h.w);
+}
+
+// One stage for one window: sum_j leaf_j in stump order (oracle c7/c8).  Stumps are
+// independent until the ordered fp32 additions, so four are evaluated per iteration.
+template <int MC, class R>
+__device__ __forceinline__ float eval_stage_mc(const uint32_t* __restrict__ T, int b, float nf, const R& rec, int first,
+                                               int n) {
+    float sum = 0.0f;
+    int j = 0;
+    for (; j + 4 <= n; j += 4) {
+        const float l0 = eval_stump_mc<MC>(T, b, nf, rec, first + j);
+        const float l1 = eval_stump_mc<MC>(T, b, nf, rec, first + j + 1);
+        const float l2 = eval_stump_mc<MC>(T, b, nf, rec, first + j + 2);
+        const float l3 = eval_stump_mc<MC>(T, b, nf, rec, first + j + 3);
+        sum = __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(sum, l0), l1), l2), l3);
+    }
+    for (; j < n; ++j) sum = __fadd_rn(sum, eval_stump_mc<MC>(T, b, nf, rec, first + j));
     return sum;
 }
 
-// below this many surviving windows a deep stage runs warp-per-window / lane-per-stump
-constexpr int LANE_MODE_MIN = 64;
-
-__device__ __forceinline__ int find_level_tile(const PlanDev& p, int r) {
-    int k = 0;
-    while (k + 1 < p.n_levels && p.lv[k + 1].tile0 <= r) ++k;
-    return k;
+// mc = the stage's largest corner count (StageDev::mc); dispatch to a padded, unrolled body
+template <class R>
+__device__ __forceinline__ float eval_stage(const uint32_t* __restrict__ T, int b, float nf, const R& rec, int first, int n,
+                                            int mc) {
+    if (mc <= 4) return eval_stage_mc<4>(T, b, nf, rec, first, n);
+    if (mc <= 6) return eval_stage_mc<6>(T, b, nf, rec, first, n);
+    if (mc <= 8) return eval_stage_mc<8>(T, b, nf, rec, first, n);
+    if (mc <= 9) return eval_stage_mc<9>(T, b, nf, rec, first, n);
+    return eval_stage_mc<MAX_CORNERS>(T, b, nf, rec, first, n);
 }
+
+// Dense first stage: each thread owns WPT windows of one column (stride STEP*TW words in
+// shared memory).  The corner count nc is warp-uniform; common counts get a fully unrolled,
+// branch-free body.
+template <int NC, int WPT, int STRIDE>
+__device__ __forceinline__ void dense_corners(const uint32_t* __restrict__ T, int base, const uint4& c0, const uint4& c1,
+                                              const uint4& c2, int nc, uint32_t* f) {
+#pragma unroll
+    for (int c = 0; c < (NC > 0 ? NC : MAX_CORNERS); ++c) {
+        if (NC > 0 || c < nc) {
+            const int w = corner_word(c0, c1, c2, c);
+            const uint32_t coef = (uint32_t)(w >> 16);
+            const uint32_t* src = reinterpret_cast<const uint32_t*>(reinterpret_cast<const char*>(T + base) + (w & 0xffff));
+#pragma unroll
+            for (int i = 0; i < WPT; ++i) f[i] += coef * src[i * STRIDE];
+        }
+    }
+}
+
+template <int WPT, int STRIDE, class R>
+__device__ __forceinline__ void dense_stage(const uint32_t* __restrict__ T, int base, const float* nf, float* sm,
+                                            const R& rec, int first, int n) {
+    for (int j = first; j < first + n; ++j) {
+        const uint4 h = rec(4 * j);
+        const uint4 c0 = rec(4 * j + 1), c1 = rec(4 * j + 2), c2 = rec(4 * j + 3);
+        const int nc = (int)h.x;
+        uint32_t f[WPT];
+#pragma unroll
+        for (int i = 0; i < WPT; ++i) f[i] = 0;
+        switch (nc) {      // Table I features compile to 6 (edge), 8 (line, centre) or 9 (diagonal) corners
+            case 6: dense_corners<6, WPT, STRIDE>(T, base, c0, c1, c2, nc, f); break;
+            case 8: dense_corners<8, WPT, STRIDE>(T, base, c0, c1, c2, nc, f); break;
+            case 9: dense_corners<9, WPT, STRIDE>(T, base, c0, c1, c2, nc, f); break;
+            default: dense_corners<0, WPT, STRIDE>(T, base, c0, c1, c2, nc, f); break;
+        }
+        const float th = __int_as_float((int)h.y), lf = __int_as_float((int)h.z), rt = __int_as_float((int)h.w);
+#pragma unroll
+        for (int i = 0; i < WPT; ++i) {
+            const float tt = __fmul_rn(th, nf[i]);
+            sm[i] = __fadd_rn(sm[i], (__int2float_rn((int)f[i]) < tt) ? lf : rt);
+        }
+    }
+}
+
+constexpr int GL = 8;                        // lanes per window in the sparse deep mode
+constexpr int WPW = 32 / GL;                 // windows per warp in the sparse deep mode
+constexpr int LEAF_CHUNK = 64;               // leaves parked per window before the ordered sum
 
 template <int STEP>
 struct TileGeo {
@@ -104,69 +178,74 @@ struct TileGeo {
     static constexpr int BOX = 2 * PLANE;          // ii + sqii (one TMA box)
     static constexpr int BUF = (BOX + 255) & ~255; // buffer stride: keeps every TMA destination 1 KB aligned
     static constexpr int NW = TX * TY;             // windows per tile
-    static constexpr size_t SMEM = (size_t)2 * BUF * 4 + (size_t)NW * 4 * 2 + (size_t)NW * 2 * 2;
+    static constexpr size_t LEAVES = (size_t)(K2_THREADS / 32) * WPW * LEAF_CHUNK;   // floats
+    static constexpr size_t smem(int nst) {
+        return (size_t)nst * BUF * 4 + (size_t)NW * 4 * 2 + LEAVES * 4 + (size_t)NW * 2 * 2;
+    }
 };
 
-template <int STEP, bool DEPTH>
-__global__ void __launch_bounds__(K2_THREADS, 2) k_cascade(const __grid_constant__ CascadeParams p) {
+// NST = TMA stages: 2 = double-buffered tiles (prefetch the next tile during evaluation),
+// 1 = single buffer with one more resident CTA per SM.
+template <int STEP, bool DEPTH, int NST>
+__global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const __grid_constant__ CascadeParams p) {
     using G = TileGeo<STEP>;
     constexpr int TW = G::TW, TX = G::TX, TY = G::TY, WPT = G::WPT;
     extern __shared__ __align__(1024) uint8_t smem_raw[];
-    uint32_t* tiles = reinterpret_cast<uint32_t*>(smem_raw);               // [2][2][TH][TW]
-    float* nfs = reinterpret_cast<float*>(tiles + 2 * G::BUF);              // [NW] per-window nf
+    uint32_t* tiles = reinterpret_cast<uint32_t*>(smem_raw);               // [NST][2][TH][TW]
+    float* nfs = reinterpret_cast<float*>(tiles + NST * G::BUF);            // [NW] per-window nf
     float* sums = nfs + G::NW;                                              // [NW] last stage sum
-    uint16_t* lists = reinterpret_cast<uint16_t*>(sums + G::NW);            // [2][NW]
+    float* leaves = sums + G::NW;                                           // [8 warps][WPW][LEAF_CHUNK]
+    uint16_t* lists = reinterpret_cast<uint16_t*>(leaves + G::LEAVES);      // [2][NW]
     __shared__ __align__(8) uint64_t mbar[2];
-    __shared__ int s_tile[2];
+    __shared__ int s_tile[2], s_lvl[2], s_tl[2];
     __shared__ int s_cnt[3];
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int N = p.n_stages;
-    const StageDev st0 = p.stages[0];
+    const StageDev& st0 = p.pstages[0];     // parameter bank: warp-uniform (n_pstages >= 1)
+    const ParamRec prec{p};
+    const GlobalRec grec{p.stumps};
 
+    // thread 0: claim a tile from the work counter, decode it and start its TMA into buffer b
+    auto fetch = [&](int b) {
+        const int tn = (int)atomicAdd(p.tile_counter, 1u);
+        s_tile[b] = tn;
+        if (tn < p.total_tiles) {
+            const int g = tn / p.tiles_per_frame, r = tn % p.tiles_per_frame;
+            int k = 0;
+            while (k + 1 < p.n_levels && __ldg(&p.lv[k + 1].tile0) <= r) ++k;
+            const int tl = r - __ldg(&p.lv[k].tile0);
+            const int tx = __ldg(&p.lv[k].tiles_x);
+            s_lvl[b] = k;
+            s_tl[b] = tl;
+            mbar_expect_tx(&mbar[b], G::BOX * 4);
+            tma_load_4d(tiles + b * G::BUF, p.tmaps + k, (tl % tx) * TX * STEP, (tl / tx) * TY * STEP, 0, g, &mbar[b]);
+        }
+    };
     if (tid == 0) {
         mbar_init(&mbar[0], 1);
         mbar_init(&mbar[1], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        const int t0 = (int)atomicAdd(p.tile_counter, 1u);
-        s_tile[0] = t0;
-        if (t0 < p.total_tiles) {
-            const int g = t0 / p.plan.tiles_per_frame, r = t0 % p.plan.tiles_per_frame;
-            const int k = find_level_tile(p.plan, r);
-            const LevelDev& L = p.plan.lv[k];
-            const int tl = r - L.tile0;
-            mbar_expect_tx(&mbar[0], G::BOX * 4);
-            tma_load_4d(tiles, &p.tmap[k], (tl % L.tiles_x) * TX * STEP, (tl / L.tiles_x) * TY * STEP, 0, g, &mbar[0]);
-        }
+        if (NST == 2) fetch(0);
     }
     uint32_t phase0 = 0, phase1 = 0;
 
     for (int it = 0;; ++it) {
-        const int buf = it & 1;
-        __syncthreads();                      // previous tile fully consumed (buf^1 free, counters free)
+        const int buf = NST == 2 ? (it & 1) : 0;
+        __syncthreads();                      // previous tile fully consumed (buffers and counters free)
         if (tid == 0) {
             s_cnt[0] = 0;
             s_cnt[1] = 0;
             s_cnt[2] = 0;
-            const int tn = (int)atomicAdd(p.tile_counter, 1u);
-            s_tile[buf ^ 1] = tn;
-            if (tn < p.total_tiles) {
-                const int g = tn / p.plan.tiles_per_frame, r = tn % p.plan.tiles_per_frame;
-                const int k = find_level_tile(p.plan, r);
-                const LevelDev& L = p.plan.lv[k];
-                const int tl = r - L.tile0;
-                mbar_expect_tx(&mbar[buf ^ 1], G::BOX * 4);
-                tma_load_4d(tiles + (buf ^ 1) * G::BUF, &p.tmap[k], (tl % L.tiles_x) * TX * STEP,
-                            (tl / L.tiles_x) * TY * STEP, 0, g, &mbar[buf ^ 1]);
-            }
+            fetch(NST == 2 ? (buf ^ 1) : 0);  // double buffer: prefetch the next tile; single: this one
         }
         __syncthreads();
         const int t = s_tile[buf];
         if (t >= p.total_tiles) break;
-        const int g = t / p.plan.tiles_per_frame, r = t % p.plan.tiles_per_frame;
-        const int k = find_level_tile(p.plan, r);
-        const LevelDev& L = p.plan.lv[k];
-        const int tl = r - L.tile0;
+        const int g = t / p.tiles_per_frame;
+        const int k = s_lvl[buf];
+        const LevelDev L = p.lv[k];
+        const int tl = s_tl[buf];
         const int wx0 = (tl % L.tiles_x) * TX, wy0 = (tl / L.tiles_x) * TY;
         const int frame = p.frame_base + g;
         if (buf == 0) {
@@ -179,7 +258,7 @@ __global__ void __launch_bounds__(K2_THREADS, 2) k_cascade(const __grid_constant
         const uint32_t* T = tiles + buf * G::BUF;      // ii plane
         const uint32_t* Q = T + G::PLANE;              // sqii plane (mod 2^32)
 
-        // ---------------- stage 1, dense: 8 windows per thread down a column
+        // ---------------- stage 1, dense: WPT windows per thread down a column
         const int lx = lane + 32 * (warp % G::WARPS_X);
         const int ly0 = (warp / G::WARPS_X) * WPT;
         const int base = ly0 * STEP * TW + lx * STEP;
@@ -195,33 +274,11 @@ __global__ void __launch_bounds__(K2_THREADS, 2) k_cascade(const __grid_constant
             nfs[(ly0 + i) * TX + lx] = nf[i];
             sm[i] = 0.0f;
         }
-        {
-            const uint4* rec = p.stumps + 4 * st0.first;
-            for (int j = 0; j < st0.n; ++j) {
-                const uint4 h = __ldg(rec + 4 * j);
-                const uint4 c0 = __ldg(rec + 4 * j + 1), c1 = __ldg(rec + 4 * j + 2), c2 = __ldg(rec + 4 * j + 3);
-                const int nc = (int)h.x;
-                uint32_t f[WPT];
-#pragma unroll
-                for (int i = 0; i < WPT; ++i) f[i] = 0;
-#pragma unroll
-                for (int c = 0; c < MAX_CORNERS; ++c) {
-                    if (c < nc) {
-                        const int w = corner_word(c0, c1, c2, c);
-                        const uint32_t coef = (uint32_t)(w >> 16);
-                        const uint32_t* src = T + base + (w & 0xffff);
-#pragma unroll
-                        for (int i = 0; i < WPT; ++i) f[i] += coef * src[i * STEP * TW];
-                    }
-                }
-                const float th = __int_as_float((int)h.y), lf = __int_as_float((int)h.z), rt = __int_as_float((int)h.w);
-#pragma unroll
-                for (int i = 0; i < WPT; ++i) {
-                    const float tt = __fmul_rn(th, nf[i]);
-                    sm[i] = __fadd_rn(sm[i], (__int2float_rn((int)f[i]) < tt) ? lf : rt);
-                }
-            }
-        }
+        if (st0.first + st0.n <= p.n_pstumps)
+            dense_stage<WPT, STEP * TW>(T, base, nf, sm, prec, st0.first, st0.n);
+        else
+            dense_stage<WPT, STEP * TW>(T, base, nf, sm, grec, st0.first, st0.n);
+
         // compaction of stage-1 survivors into lists[1] (count s_cnt[1])
 #pragma unroll
         for (int i = 0; i < WPT; ++i) {
@@ -230,7 +287,7 @@ __global__ void __launch_bounds__(K2_THREADS, 2) k_cascade(const __grid_constant
             const bool pass = valid && (sm[i] >= st0.T);
             const int idx = (ly0 + i) * TX + lx;
             if (DEPTH && valid && !pass) {
-                const long long o = (long long)frame * p.plan.win_per_frame + L.win0 + (long long)wy * L.nx + (wx0 + lx);
+                const long long o = (long long)frame * p.win_per_frame + L.win0 + (long long)wy * L.nx + (wx0 + lx);
                 p.depth[o] = 0;
                 p.score[o] = sm[i];
             }
@@ -255,47 +312,50 @@ __global__ void __launch_bounds__(K2_THREADS, 2) k_cascade(const __grid_constant
 
         // ---------------- deeper stages over the compacted queue
         int s = 1;
-        for (; s < N; ++s) {
-            const int n = s_cnt[s % 3];
-            if (tid == 0 && p.stage_counts && n) atomicAdd(p.stage_counts + s, (unsigned long long)n);
-            if (n == 0) break;
-            if (tid == 0) s_cnt[(s + 2) % 3] = 0;
-            const StageDev sd = p.stages[s];
+        // one deep stage; sd is a parameter-bank (uniform) or global stage descriptor
+        auto deep_stage = [&](const StageDev& sd, int n) {
             const uint16_t* lin = lists + (s & 1) * G::NW;
             uint16_t* lout = lists + ((s + 1) & 1) * G::NW;
-            const uint4* rec = p.stumps + 4 * sd.first;
-            if (n < LANE_MODE_MIN) {
-                // few survivors: one warp per window, one lane per stump (params and corners
-                // fetched in parallel), then the leaves are added in stump order (exact fp32
-                // sequence of the definition) by every lane redundantly via shuffles.
-                for (int e = warp; e < n; e += K2_THREADS / 32) {
-                    const int idx = lin[e];
+            if (n < p.lane_min) {
+                // few survivors: GL lanes per window (WPW windows per warp), the group's lanes
+                // evaluate different stumps in parallel and park the leaves in shared memory;
+                // the group leader then adds them in stump order (the exact fp32 sequence of
+                // the definition).
+                const int grp = lane / GL, q = lane % GL;
+                float* lv = leaves + (warp * WPW + grp) * LEAF_CHUNK;
+                for (int e0 = warp * WPW; e0 < n; e0 += (K2_THREADS / 32) * WPW) {
+                    const int e = e0 + grp;
+                    const bool act = e < n;
+                    const int idx = act ? lin[e] : 0;
                     const int wlx = idx % TX, wly = idx / TX;
                     const int b = wly * STEP * TW + wlx * STEP;
                     const float nfw = nfs[idx];
                     float sum = 0.0f;
-                    for (int c0 = 0; c0 < sd.n; c0 += 32) {
-                        const int j = c0 + lane;
-                        float leaf = 0.0f;
-                        if (j < sd.n) leaf = eval_stage<STEP>(T, b, nfw, rec + 4 * j, 1);
-                        const int m = min(32, sd.n - c0);
-                        for (int t = 0; t < m; ++t) sum = __fadd_rn(sum, __shfl_sync(0xffffffffu, leaf, t));
+                    for (int c0 = 0; c0 < sd.n; c0 += LEAF_CHUNK) {
+                        const int cn = min(LEAF_CHUNK, sd.n - c0);
+                        if (act)
+                            for (int j = q; j < cn; j += GL)
+                                lv[j] = eval_stage(T, b, nfw, grec, sd.first + c0 + j, 1, sd.mc);
+                        __syncwarp();
+                        if (act && q == 0)
+                            for (int t2 = 0; t2 < cn; ++t2) sum = __fadd_rn(sum, lv[t2]);
+                        __syncwarp();
                     }
-                    if (lane == 0) {
+                    if (act && q == 0) {
                         if (sum >= sd.T) {
                             lout[atomicAdd(&s_cnt[(s + 1) % 3], 1)] = (uint16_t)idx;
                             sums[idx] = sum;
                         } else if (DEPTH) {
-                            const long long o = (long long)frame * p.plan.win_per_frame + L.win0 +
+                            const long long o = (long long)frame * p.win_per_frame + L.win0 +
                                                 (long long)(wy0 + wly) * L.nx + (wx0 + wlx);
                             p.depth[o] = (uint8_t)(s < 255 ? s : 255);
                             p.score[o] = sum;
                         }
                     }
                 }
-                __syncthreads();
-                continue;
+                return;
             }
+            const bool in_param = sd.first + sd.n <= p.n_pstumps;
             for (int e0 = warp * 32; e0 < n; e0 += K2_THREADS) {
                 const int e = e0 + lane;
                 const bool act = e < n;
@@ -304,12 +364,14 @@ __global__ void __launch_bounds__(K2_THREADS, 2) k_cascade(const __grid_constant
                 if (act) {
                     idx = lin[e];
                     const int wlx = idx % TX, wly = idx / TX;
-                    sum = eval_stage<STEP>(T, wly * STEP * TW + wlx * STEP, nfs[idx], rec, sd.n);
+                    const int b = wly * STEP * TW + wlx * STEP;
+                    sum = in_param ? eval_stage(T, b, nfs[idx], prec, sd.first, sd.n, sd.mc)
+                                   : eval_stage(T, b, nfs[idx], grec, sd.first, sd.n, sd.mc);
                 }
                 const bool pass = act && (sum >= sd.T);
                 if (DEPTH && act && !pass) {
                     const int wlx = idx % TX, wly = idx / TX;
-                    const long long o = (long long)frame * p.plan.win_per_frame + L.win0 +
+                    const long long o = (long long)frame * p.win_per_frame + L.win0 +
                                         (long long)(wy0 + wly) * L.nx + (wx0 + wlx);
                     p.depth[o] = (uint8_t)(s < 255 ? s : 255);
                     p.score[o] = sum;
@@ -325,6 +387,16 @@ __global__ void __launch_bounds__(K2_THREADS, 2) k_cascade(const __grid_constant
                     }
                 }
             }
+        };
+        for (; s < N; ++s) {
+            const int n = s_cnt[s % 3];
+            if (tid == 0 && p.stage_counts && n) atomicAdd(p.stage_counts + s, (unsigned long long)n);
+            if (n == 0) break;
+            if (tid == 0) s_cnt[(s + 2) % 3] = 0;
+            if (s < p.n_pstages)
+                deep_stage(p.pstages[s], n);
+            else
+                deep_stage(p.stages[s], n);
             __syncthreads();
         }
         if (s == N) {                               // accepted windows: depth N
@@ -338,7 +410,7 @@ __global__ void __launch_bounds__(K2_THREADS, 2) k_cascade(const __grid_constant
                 const int wlx = idx % TX, wly = idx / TX;
                 if (DEPTH) {
                     if (act) {
-                        const long long o = (long long)frame * p.plan.win_per_frame + L.win0 +
+                        const long long o = (long long)frame * p.win_per_frame + L.win0 +
                                             (long long)(wy0 + wly) * L.nx + (wx0 + wlx);
                         p.depth[o] = (uint8_t)(N < 255 ? N : 255);
                         p.score[o] = sums[idx];
@@ -361,50 +433,70 @@ __global__ void __launch_bounds__(K2_THREADS, 2) k_cascade(const __grid_constant
     }
 }
 
-template <int STEP, bool DEPTH>
+// TMA stages (FD_K2_STAGES=1|2, default 1: measured faster, 3 CTAs/SM hide more latency)
+static int k2_stages() {
+    static int v = [] {
+        const char* e = getenv("FD_K2_STAGES");
+        return (e && e[0] == '2') ? 2 : 1;
+    }();
+    return v;
+}
+
+template <int STEP, bool DEPTH, int NST>
 static cudaError_t launch_one(const CascadeParams& p, int grid, cudaStream_t st) {
-    const size_t smem = TileGeo<STEP>::SMEM;
-    cudaError_t e = cudaFuncSetAttribute(k_cascade<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const size_t smem = TileGeo<STEP>::smem(NST);
+    cudaError_t e = cudaFuncSetAttribute(k_cascade<STEP, DEPTH, NST>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    k_cascade<STEP, DEPTH><<<grid, K2_THREADS, smem, st>>>(p);
+    k_cascade<STEP, DEPTH, NST><<<grid, K2_THREADS, smem, st>>>(p);
     return cudaGetLastError();
 }
 
-template <int STEP, bool DEPTH>
+template <int STEP, bool DEPTH, int NST>
 static int grid_one() {
-    const size_t smem = TileGeo<STEP>::SMEM;
-    cudaFuncSetAttribute(k_cascade<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const size_t smem = TileGeo<STEP>::smem(NST);
+    cudaFuncSetAttribute(k_cascade<STEP, DEPTH, NST>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int dev = 0, sms = 0, per = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_cascade<STEP, DEPTH>, K2_THREADS, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_cascade<STEP, DEPTH, NST>, K2_THREADS, smem);
     return sms * (per > 0 ? per : 1);
 }
 
+template <int STEP, bool DEPTH>
+static int grid_step() {
+    return k2_stages() == 1 ? grid_one<STEP, DEPTH, 1>() : grid_one<STEP, DEPTH, 2>();
+}
+
+template <int STEP, bool DEPTH>
+static cudaError_t launch_step(const CascadeParams& p, int grid, cudaStream_t st) {
+    return k2_stages() == 1 ? launch_one<STEP, DEPTH, 1>(p, grid, st) : launch_one<STEP, DEPTH, 2>(p, grid, st);
+}
+
 size_t cascade_smem(int step) {
+    const int n = k2_stages();
     switch (step) {
-        case 1: return TileGeo<1>::SMEM;
-        case 2: return TileGeo<2>::SMEM;
-        case 3: return TileGeo<3>::SMEM;
-        default: return TileGeo<4>::SMEM;
+        case 1: return TileGeo<1>::smem(n);
+        case 2: return TileGeo<2>::smem(n);
+        case 3: return TileGeo<3>::smem(n);
+        default: return TileGeo<4>::smem(n);
     }
 }
 
 int cascade_grid(bool depth, int step) {
     switch (step) {
-        case 1: return depth ? grid_one<1, true>() : grid_one<1, false>();
-        case 2: return depth ? grid_one<2, true>() : grid_one<2, false>();
-        case 3: return depth ? grid_one<3, true>() : grid_one<3, false>();
-        default: return depth ? grid_one<4, true>() : grid_one<4, false>();
+        case 1: return depth ? grid_step<1, true>() : grid_step<1, false>();
+        case 2: return depth ? grid_step<2, true>() : grid_step<2, false>();
+        case 3: return depth ? grid_step<3, true>() : grid_step<3, false>();
+        default: return depth ? grid_step<4, true>() : grid_step<4, false>();
     }
 }
 
 cudaError_t launch_cascade(const CascadeParams& p, bool depth, int step, int grid, cudaStream_t st) {
     switch (step) {
-        case 1: return depth ? launch_one<1, true>(p, grid, st) : launch_one<1, false>(p, grid, st);
-        case 2: return depth ? launch_one<2, true>(p, grid, st) : launch_one<2, false>(p, grid, st);
-        case 3: return depth ? launch_one<3, true>(p, grid, st) : launch_one<3, false>(p, grid, st);
-        case 4: return depth ? launch_one<4, true>(p, grid, st) : launch_one<4, false>(p, grid, st);
+        case 1: return depth ? launch_step<1, true>(p, grid, st) : launch_step<1, false>(p, grid, st);
+        case 2: return depth ? launch_step<2, true>(p, grid, st) : launch_step<2, false>(p, grid, st);
+        case 3: return depth ? launch_step<3, true>(p, grid, st) : launch_step<3, false>(p, grid, st);
+        case 4: return depth ? launch_step<4, true>(p, grid, st) : launch_step<4, false>(p, grid, st);
         default: return cudaErrorInvalidValue;
     }
 }
