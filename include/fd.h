@@ -147,7 +147,7 @@ fd_status fd_detect_host(fd_cascade c, const uint8_t* h_frames, int n, int W, in
  * ties -> lexicographically smallest pair (reading R10).  d_in: n detections sorted by frame
  * (fd_detect order).  Clusters with >= min_neighbors members are written to d_out ordered by
  * (frame, first member).  *n_out (host) = count; FD_ECAPACITY if > capacity.
- * Synchronises `stream` once. */
+ * Synchronises `stream` once (to read the count). */
 fd_status fd_group(const fd_detection* d_in, int64_t n, double eyes_thresh, int min_neighbors,
                    fd_detection* d_out, int64_t capacity, int64_t* n_out, void* stream);
 

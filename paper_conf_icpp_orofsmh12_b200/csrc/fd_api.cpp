@@ -770,8 +770,9 @@ fd_status fd_group(const fd_detection* d_in, int64_t n, double eyes_thresh, int 
     CK(w->group.ensure(group_scratch_bytes(n) + 128));
     long long* d_total = reinterpret_cast<long long*>(w->group.as<char>() + w->group.n - 64);
     {
-        ProfScope ps(FD_K_GROUP, st, 4);
-        CK(launch_group_all(d_in, n, eyes_thresh, min_neighbors < 1 ? 1 : min_neighbors, w->group.p, d_out, capacity,
+        ProfScope ps(FD_K_GROUP, st, 5);
+        CK(launch_group_plan(d_in, n, w->group.p, st));
+        CK(launch_group_run(d_in, n, eyes_thresh, min_neighbors < 1 ? 1 : min_neighbors, w->group.p, d_out, capacity,
                             d_total, st));
     }
     CK(cudaMemcpyAsync(w->h_pinned, d_total, 8, cudaMemcpyDeviceToHost, st));

@@ -123,7 +123,8 @@ cudaError_t launch_keys_to_dets(const unsigned long long* keys, const float* sco
 cudaError_t sort_pairs(void* tmp, size_t& tmp_bytes, const unsigned long long* kin, unsigned long long* kout,
                        const float* vin, float* vout, long long n, cudaStream_t st);
 size_t group_scratch_bytes(long long n);
-cudaError_t launch_group_all(const fd_detection* in, long long n, double thresh, int min_neighbors, void* scratch,
+cudaError_t launch_group_plan(const fd_detection* in, long long n, void* scratch, cudaStream_t st);
+cudaError_t launch_group_run(const fd_detection* in, long long n, double thresh, int min_neighbors, void* scratch,
                              fd_detection* out, long long cap, long long* d_total, cudaStream_t st);
 
 }  // namespace fdk

@@ -154,6 +154,11 @@ __device__ PairKey block_min(PairKey v, PairKey* red) {
 }
 
 // Segments = runs of equal frame in the sorted input. seg_start[s], n_seg on device.
+// Only pairs with S_eyes < thresh can ever be merged, so nearest neighbours are kept over those
+// pairs only (the greedy order of the definition is unchanged: the global minimum pair is the
+// same whenever it is below the threshold, and the loop stops otherwise).  A pair whose left-
+// or right-eye coordinate gap alone already forces S_eyes >= thresh is skipped without the
+// square roots and the division.
 __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ in, long long n,
                                               const long long* __restrict__ seg_start, const int* __restrict__ n_seg_p,
                                               double thresh, int min_neighbors, GroupScratch gs, int* seg_next,
@@ -163,6 +168,7 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
     __shared__ int s_nlist;
     __shared__ int s_list[GLIST];
     const int n_seg = *n_seg_p;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     for (;;) {
         __syncthreads();
         if (threadIdx.x == 0) s_seg = atomicAdd(seg_next, 1);
@@ -183,7 +189,44 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
             g.eyes[i] = eyes_of((double)d.x, (double)d.y, (double)d.w, (double)d.h);
         }
         __syncthreads();
-        for (int i = threadIdx.x; i < m; i += GT) nn_full(g, m, i);
+        // S_eyes of clusters kk, j, or +inf when a single coordinate gap proves S >= thresh:
+        // S = (d_le + d_re)/min(d) >= |gap|/min(d); the 2^-40 margin keeps every skipped pair's
+        // rounded S above thresh.
+        const double tguard = thresh * (1.0 + 0x1p-40);
+        auto dist = [&](int kk, int j) -> double {
+            const Eyes& a = g.eyes[kk];
+            const Eyes& b = g.eyes[j];
+            const double lim = tguard * (a.d < b.d ? a.d : b.d);
+            if (fabs(a.lex - b.lex) > lim || fabs(a.ley - b.ley) > lim || fabs(a.rex - b.rex) > lim) return CUDART_INF;
+            return s_eyes(a, b);
+        };
+        // warp-parallel nearest neighbour of cluster kk (lowest index on ties)
+        auto warp_nn = [&](int kk) {
+            double bs = CUDART_INF;
+            int bj = 0x7fffffff;
+            for (int j = lane; j < m; j += 32) {
+                if (j == kk || g.cnt[j] == 0) continue;
+                const double s = dist(kk, j);
+                if (s < bs) {        // j increases per lane: first minimum = lowest index
+                    bs = s;
+                    bj = j;
+                }
+            }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                const double os = __shfl_xor_sync(0xffffffffu, bs, o);
+                const int oj = __shfl_xor_sync(0xffffffffu, bj, o);
+                if (os < bs || (os == bs && oj < bj)) {
+                    bs = os;
+                    bj = oj;
+                }
+            }
+            if (lane == 0) {
+                g.nn[kk] = bj == 0x7fffffff ? -1 : bj;
+                g.nnd[kk] = bs;
+            }
+        };
+        for (int i = warp; i < m; i += GT / 32) warp_nn(i);
         __syncthreads();
         for (;;) {
             PairKey best;
@@ -220,7 +263,7 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
                     if (pos < GLIST) s_list[pos] = kk;
                     else nn_full(g, m, kk);
                 } else {
-                    const double s = s_eyes(g.eyes[kk], g.eyes[a]);
+                    const double s = dist(kk, a);
                     if (s < g.nnd[kk] || (s == g.nnd[kk] && a < nk)) {
                         g.nnd[kk] = s;
                         g.nn[kk] = a;
@@ -229,35 +272,8 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
             }
             __syncthreads();
             {
-                const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
                 const int nl = min(s_nlist, GLIST);
-                for (int e = warp; e < nl; e += GT / 32) {
-                    const int kk = s_list[e];
-                    const Eyes ek = g.eyes[kk];
-                    double bs = CUDART_INF;
-                    int bj = 0x7fffffff;
-                    for (int j = lane; j < m; j += 32) {
-                        if (j == kk || g.cnt[j] == 0) continue;
-                        const double s = s_eyes(ek, g.eyes[j]);
-                        if (s < bs) {        // j increases per lane: first minimum = lowest index
-                            bs = s;
-                            bj = j;
-                        }
-                    }
-#pragma unroll
-                    for (int o = 16; o > 0; o >>= 1) {
-                        const double os = __shfl_xor_sync(0xffffffffu, bs, o);
-                        const int oj = __shfl_xor_sync(0xffffffffu, bj, o);
-                        if (os < bs || (os == bs && oj < bj)) {
-                            bs = os;
-                            bj = oj;
-                        }
-                    }
-                    if (lane == 0) {
-                        g.nn[kk] = bj == 0x7fffffff ? -1 : bj;
-                        g.nnd[kk] = bs;
-                    }
-                }
+                for (int e = warp; e < nl; e += GT / 32) warp_nn(s_list[e]);
             }
             __syncthreads();
         }
@@ -336,48 +352,64 @@ __global__ void k_seg_copy(const int* __restrict__ n_seg_p, const long long* __r
     }
 }
 
-// scratch layout helper: returns bytes needed for n detections
+struct GroupLayout {
+    GroupScratch g;
+    long long* seg_start;
+    int* seg_count;
+    long long* seg_off;
+    fd_detection* tmp;
+    int* misc;                 // [0] n_seg, [1] seg_next
+    GroupLayout(void* scratch, long long n) {
+        char* p = reinterpret_cast<char*>(scratch);
+        auto take = [&](size_t bytes) {
+            char* r = p;
+            p += (bytes + 255) & ~size_t(255);
+            return r;
+        };
+        const size_t a = (size_t)(n > 0 ? n : 1);
+        g.sx = reinterpret_cast<long long*>(take(a * 8));
+        g.sy = reinterpret_cast<long long*>(take(a * 8));
+        g.sw = reinterpret_cast<long long*>(take(a * 8));
+        g.sh = reinterpret_cast<long long*>(take(a * 8));
+        g.cnt = reinterpret_cast<int*>(take(a * 4));
+        g.smax = reinterpret_cast<float*>(take(a * 4));
+        g.nn = reinterpret_cast<int*>(take(a * 4));
+        g.nnd = reinterpret_cast<double*>(take(a * 8));
+        g.eyes = reinterpret_cast<Eyes*>(take(a * sizeof(Eyes)));
+        seg_start = reinterpret_cast<long long*>(take(a * 8));
+        seg_count = reinterpret_cast<int*>(take(a * 4));
+        seg_off = reinterpret_cast<long long*>(take(a * 8));
+        tmp = reinterpret_cast<fd_detection*>(take(a * sizeof(fd_detection)));
+        misc = reinterpret_cast<int*>(take(256));
+    }
+};
+
 size_t group_scratch_bytes(long long n) {
     const size_t a = (size_t)(n > 0 ? n : 1);
-    return a * (4 * 8 + 4 + 4 + 4 + 8 + sizeof(Eyes)) + a * 8 /*seg_start*/ + a * 4 /*seg_count*/ +
-           a * 8 /*seg_off*/ + a * sizeof(fd_detection) /*tmp*/ + 8192;
+    return a * (4 * 8 + 4 + 4 + 4 + 8 + sizeof(Eyes) + 8 + 4 + 8 + sizeof(fd_detection)) + 20 * 256;
 }
 
-cudaError_t launch_group_all(const fd_detection* in, long long n, double thresh, int min_neighbors, void* scratch,
+// phase 1: frame segments (runs of equal frame index)
+cudaError_t launch_group_plan(const fd_detection* in, long long n, void* scratch, cudaStream_t st) {
+    GroupLayout L(scratch, n);
+    cudaError_t e = cudaMemsetAsync(L.misc, 0, 256, st);
+    if (e != cudaSuccess || n <= 0) return e;
+    k_seg_starts<<<1, 1024, 0, st>>>(in, n, L.seg_start, L.misc);
+    return cudaGetLastError();
+}
+
+// phase 2: greedy grouping per segment, then ordered compaction into out
+cudaError_t launch_group_run(const fd_detection* in, long long n, double thresh, int min_neighbors, void* scratch,
                              fd_detection* out, long long cap, long long* d_total, cudaStream_t st) {
-    char* p = reinterpret_cast<char*>(scratch);
-    auto take = [&](size_t bytes) {
-        char* r = p;
-        p += (bytes + 255) & ~size_t(255);
-        return r;
-    };
-    const size_t a = (size_t)(n > 0 ? n : 1);
-    GroupScratch g;
-    g.sx = reinterpret_cast<long long*>(take(a * 8));
-    g.sy = reinterpret_cast<long long*>(take(a * 8));
-    g.sw = reinterpret_cast<long long*>(take(a * 8));
-    g.sh = reinterpret_cast<long long*>(take(a * 8));
-    g.cnt = reinterpret_cast<int*>(take(a * 4));
-    g.smax = reinterpret_cast<float*>(take(a * 4));
-    g.nn = reinterpret_cast<int*>(take(a * 4));
-    g.nnd = reinterpret_cast<double*>(take(a * 8));
-    g.eyes = reinterpret_cast<Eyes*>(take(a * sizeof(Eyes)));
-    long long* seg_start = reinterpret_cast<long long*>(take(a * 8));
-    int* seg_count = reinterpret_cast<int*>(take(a * 4));
-    long long* seg_off = reinterpret_cast<long long*>(take(a * 8));
-    fd_detection* tmp = reinterpret_cast<fd_detection*>(take(a * sizeof(fd_detection)));
-    int* misc = reinterpret_cast<int*>(take(256));     // [0] n_seg, [1] seg_next
-    cudaError_t e = cudaMemsetAsync(misc, 0, 256, st);
-    if (e != cudaSuccess) return e;
+    GroupLayout L(scratch, n);
     if (n <= 0) return cudaMemsetAsync(d_total, 0, sizeof(long long), st);
-    k_seg_starts<<<1, 1024, 0, st>>>(in, n, seg_start, misc);
     int dev = 0, sms = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int grid = (int)(n < (long long)sms * 4 ? n : (long long)sms * 4);
-    k_group<<<grid, GT, 0, st>>>(in, n, seg_start, misc, thresh, min_neighbors, g, misc + 1, seg_count, tmp);
-    k_seg_offsets<<<1, 32, 0, st>>>(misc, seg_count, seg_off, d_total);
-    k_seg_copy<<<grid, 256, 0, st>>>(misc, seg_start, seg_count, seg_off, tmp, out, cap);
+    k_group<<<grid, GT, 0, st>>>(in, n, L.seg_start, L.misc, thresh, min_neighbors, L.g, L.misc + 1, L.seg_count, L.tmp);
+    k_seg_offsets<<<1, 32, 0, st>>>(L.misc, L.seg_count, L.seg_off, d_total);
+    k_seg_copy<<<grid, 256, 0, st>>>(L.misc, L.seg_start, L.seg_count, L.seg_off, L.tmp, out, cap);
     return cudaGetLastError();
 }
 

@@ -1,0 +1,81 @@
+"""Multi-process host logic of the frame-sharded path on CPU with gloo,
+world_size 2: contiguous frame shards, local->global frame indices, and the count + padded
+all_gather of detection lists, whose rank-order concatenation must equal the single-process
+list (computed here with the CPU oracle on the same seeded frames)."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import fdgen
+import oracle
+from paper_conf_icpp_orofsmh12_b200 import dist as fdd
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+W, H, S = 160, 120, 1.25
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def test_shard_covers_frames_contiguously():
+    for n in (1, 7, 512, 513):
+        for world in (1, 2, 4, 8):
+            r = [fdd.shard(n, k, world) for k in range(world)]
+            assert r[0][0] == 0 and r[-1][1] == n
+            assert all(a[1] == b[0] for a, b in zip(r, r[1:]))
+            assert max(e - s for s, e in r) - min(e - s for s, e in r) <= 1
+
+
+def _worker(rank, world, port, n_frames, out_q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        casc = oracle.Cascade.from_file(os.path.join(ROOT, "cascades", "c1.fdc"))
+        lo, hi = fdd.shard(n_frames, rank, world)
+        frames, _ = fdgen.frames(1, lo, hi - lo, W, H)          # global frame indices lo..hi-1
+        dets, _ = oracle.detect(casc, frames, 24, S, 1)
+        grp = oracle.group(dets)
+        t = torch.from_numpy(grp.view(np.int32).reshape(-1, 10).copy())
+        gathered = fdd.gather_detections(fdd.globalize(t, lo))
+        if rank == 0:
+            out_q.put(gathered.numpy().copy())
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2])
+def test_gather_equals_single_process(world):
+    n = 5
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, n, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    got = q.get(timeout=120)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    casc = oracle.Cascade.from_file(os.path.join(ROOT, "cascades", "c1.fdc"))
+    frames, _ = fdgen.frames(1, 0, n, W, H)
+    dets, _ = oracle.detect(casc, frames, 24, S, 1)
+    ref = oracle.group(dets)
+    assert np.array_equal(got.view(oracle.DET_DTYPE).reshape(-1), ref)
+
+
+def test_gather_handles_empty_ranks():
+    # a rank with zero detections contributes nothing; padding never leaks into the result
+    a = torch.zeros((0, 10), dtype=torch.int32)
+    b = torch.arange(30, dtype=torch.int32).reshape(3, 10)
+    assert fdd.globalize(a, 5).shape == (0, 10)
+    g = fdd.globalize(b, 4)
+    assert g[:, 0].tolist() == [4, 14, 24] and b[0, 0] == 0
