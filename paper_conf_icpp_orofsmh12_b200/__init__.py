@@ -18,7 +18,8 @@ import threading
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-_SO = os.path.join(_PKG, "libfd.so")
+# FD_LIB_VARIANT=timing loads the diagnostic build libfd_timing.so (same ABI + K2 phase counters)
+_SO = os.path.join(_PKG, f"libfd_{os.environ['FD_LIB_VARIANT']}.so" if os.environ.get("FD_LIB_VARIANT") else "libfd.so")
 _lock = threading.Lock()
 _lib = None
 

@@ -26,8 +26,11 @@ def _nvcc() -> str:
     raise RuntimeError("nvcc not found")
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, variant: str = "") -> str:
+    """variant "timing" builds libfd_timing.so with -DFD_K2_TIMING (K2 phase counters)."""
     nvcc = _nvcc()
+    if variant:
+        return _build_variant(nvcc, variant, verbose)
     os.makedirs(OBJ, exist_ok=True)
     hdr_t = max(os.path.getmtime(h) for h in HEADERS)
     objs = []
@@ -49,5 +52,23 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return OUT
 
 
+def _build_variant(nvcc: str, variant: str, verbose: bool) -> str:
+    defs = {"timing": ["-DFD_K2_TIMING"]}[variant]
+    odir = os.path.join(OBJ, variant)
+    os.makedirs(odir, exist_ok=True)
+    objs = []
+    for src in SOURCES:
+        o = os.path.join(odir, src + ".o")
+        cmd = [nvcc, *ARCH, *NVFLAGS, *defs, "-c", os.path.join(CSRC, src), "-o", o]
+        if verbose:
+            print(" ".join(cmd), file=sys.stderr)
+        subprocess.check_call(cmd)
+        objs.append(o)
+    out = os.path.join(PKG, f"libfd_{variant}.so")
+    subprocess.check_call([nvcc, *ARCH, "-shared", "-cudart", "static", "-o", out, *objs, "-ldl"])
+    return out
+
+
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose=True))
+    v = [a.split("=", 1)[1] for a in sys.argv if a.startswith("--variant=")]
+    print(build(force="--force" in sys.argv, verbose=True, variant=v[0] if v else ""))

@@ -24,6 +24,20 @@
 
 namespace fdk {
 
+#ifdef FD_K2_TIMING
+// [0] tiles, [1] TMA-wait cycles, [2] stage-1 cycles, [3] deep-stage cycles, [4+s] tiles whose
+// deepest stage loop ended at s (diagnostic build only: -DFD_K2_TIMING)
+__device__ unsigned long long g_k2_timing[16];
+extern "C" int fd_debug_k2_timing(unsigned long long* out, int reset) {
+    if (cudaMemcpyFromSymbol(out, g_k2_timing, sizeof(g_k2_timing)) != cudaSuccess) return -1;
+    if (reset) {
+        unsigned long long z[16] = {};
+        cudaMemcpyToSymbol(g_k2_timing, z, sizeof(z));
+    }
+    return 0;
+}
+#endif
+
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
@@ -248,6 +262,9 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
         const int tl = s_tl[buf];
         const int wx0 = (tl % L.tiles_x) * TX, wy0 = (tl / L.tiles_x) * TY;
         const int frame = p.frame_base + g;
+#ifdef FD_K2_TIMING
+        const long long tm0 = clock64();
+#endif
         if (buf == 0) {
             mbar_wait(&mbar[0], phase0);
             phase0 ^= 1;
@@ -255,6 +272,9 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
             mbar_wait(&mbar[1], phase1);
             phase1 ^= 1;
         }
+#ifdef FD_K2_TIMING
+        const long long tm1 = clock64();
+#endif
         const uint32_t* T = tiles + buf * G::BUF;      // ii plane
         const uint32_t* Q = T + G::PLANE;              // sqii plane (mod 2^32)
 
@@ -310,6 +330,9 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
         }
         __syncthreads();
 
+#ifdef FD_K2_TIMING
+        const long long tm2 = clock64();
+#endif
         // ---------------- deeper stages over the compacted queue
         int s = 1;
         // one deep stage; sd is a parameter-bank (uniform) or global stage descriptor
@@ -337,8 +360,16 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
                             for (int j = q; j < cn; j += GL)
                                 lv[j] = eval_stage(T, b, nfw, grec, sd.first + c0 + j, 1, sd.mc);
                         __syncwarp();
-                        if (act && q == 0)
-                            for (int t2 = 0; t2 < cn; ++t2) sum = __fadd_rn(sum, lv[t2]);
+                        if (act && q == 0) {
+                            int t2 = 0;
+                            for (; t2 + 8 <= cn; t2 += 8) {         // loads batched, additions in order
+                                const float4 a = *reinterpret_cast<const float4*>(lv + t2);
+                                const float4 c = *reinterpret_cast<const float4*>(lv + t2 + 4);
+                                sum = __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(sum, a.x), a.y), a.z), a.w);
+                                sum = __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(sum, c.x), c.y), c.z), c.w);
+                            }
+                            for (; t2 < cn; ++t2) sum = __fadd_rn(sum, lv[t2]);
+                        }
                         __syncwarp();
                     }
                     if (act && q == 0) {
@@ -388,18 +419,100 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
                 }
             }
         };
+        bool tail_done = false;
         for (; s < N; ++s) {
             const int n = s_cnt[s % 3];
             if (tid == 0 && p.stage_counts && n) atomicAdd(p.stage_counts + s, (unsigned long long)n);
             if (n == 0) break;
+            if (n <= K2_THREADS / 32) {
+                // tail: at most one window per warp left -- each warp walks its window through
+                // all remaining stages on its own (one stump per lane, leaves added in stump
+                // order via shuffles), so no block barrier is paid per stage.
+                if (warp < n) {
+                    const int idx = lists[(s & 1) * G::NW + warp];
+                    const int wlx = idx % TX, wly = idx / TX;
+                    const int b = wly * STEP * TW + wlx * STEP;
+                    const float nfw = nfs[idx];
+                    int s2 = s;
+                    float sum = 0.0f;
+                    for (; s2 < N; ++s2) {
+                        StageDev sd;
+                        if (s2 < p.n_pstages) {
+                            sd.first = p.pstages[s2].first;
+                            sd.n = p.pstages[s2].n;
+                            sd.T = p.pstages[s2].T;
+                            sd.mc = p.pstages[s2].mc;
+                        } else {
+                            sd = p.stages[s2];
+                        }
+                        if (s2 > s && lane == 0 && p.stage_counts) atomicAdd(p.stage_counts + s2, 1ull);
+                        sum = 0.0f;
+                        for (int c0 = 0; c0 < sd.n; c0 += 32) {
+                            const int j = c0 + lane;
+                            float leaf = 0.0f;
+                            if (j < sd.n) leaf = eval_stage(T, b, nfw, grec, sd.first + j, 1, sd.mc);
+                            const int m = min(32, sd.n - c0);
+                            // ordered sum of the lanes' leaves: independent shuffles, serial adds
+#pragma unroll
+                            for (int t2 = 0; t2 < 32; ++t2) {
+                                const float v = __shfl_sync(0xffffffffu, leaf, t2);
+                                if (t2 < m) sum = __fadd_rn(sum, v);
+                            }
+                        }
+                        if (!(sum >= sd.T)) break;
+                    }
+                    if (lane == 0) {
+                        const long long o = (long long)frame * p.win_per_frame + L.win0 +
+                                            (long long)(wy0 + wly) * L.nx + (wx0 + wlx);
+                        if (s2 < N) {
+                            if (DEPTH) {
+                                p.depth[o] = (uint8_t)(s2 < 255 ? s2 : 255);
+                                p.score[o] = sum;
+                            }
+                        } else {
+                            if (p.stage_counts) atomicAdd(p.stage_counts + N, 1ull);
+                            if (DEPTH) {
+                                p.depth[o] = (uint8_t)(N < 255 ? N : 255);
+                                p.score[o] = sum;
+                            } else {
+                                const unsigned long long at = atomicAdd(p.det_count, 1ull);
+                                if ((long long)at < p.det_cap) {
+                                    p.det_keys[at] = det_key(frame, k, (wy0 + wly) * STEP, (wx0 + wlx) * STEP);
+                                    p.det_scores[at] = sum;
+                                }
+                            }
+                        }
+                    }
+                }
+                tail_done = true;
+                break;
+            }
             if (tid == 0) s_cnt[(s + 2) % 3] = 0;
-            if (s < p.n_pstages)
-                deep_stage(p.pstages[s], n);
-            else
-                deep_stage(p.stages[s], n);
+            {
+                StageDev sd;                  // one call site keeps deep_stage inlined
+                if (s < p.n_pstages) {
+                    sd.first = p.pstages[s].first;
+                    sd.n = p.pstages[s].n;
+                    sd.T = p.pstages[s].T;
+                    sd.mc = p.pstages[s].mc;
+                } else {
+                    sd = p.stages[s];
+                }
+                deep_stage(sd, n);
+            }
             __syncthreads();
         }
-        if (s == N) {                               // accepted windows: depth N
+#ifdef FD_K2_TIMING
+        if (tid == 0) {
+            const long long tm3 = clock64();
+            atomicAdd(&g_k2_timing[0], 1ull);
+            atomicAdd(&g_k2_timing[1], (unsigned long long)(tm1 - tm0));
+            atomicAdd(&g_k2_timing[2], (unsigned long long)(tm2 - tm1));
+            atomicAdd(&g_k2_timing[3], (unsigned long long)(tm3 - tm2));
+            atomicAdd(&g_k2_timing[4 + (s < 11 ? s : 11)], 1ull);
+        }
+#endif
+        if (s == N && !tail_done) {                 // accepted windows: depth N
             const int nacc = s_cnt[N % 3];
             if (tid == 0 && p.stage_counts && nacc) atomicAdd(p.stage_counts + N, (unsigned long long)nacc);
             const uint16_t* lacc = lists + (N & 1) * G::NW;
