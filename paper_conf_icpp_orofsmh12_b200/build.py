@@ -12,8 +12,8 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 OUT = os.path.join(PKG, "libfd.so")
 OBJ = os.path.join(PKG, "build")
-SOURCES = ["k_integral.cu", "k_cascade.cu", "k_output.cu", "fd_api.cpp"]
-HEADERS = [os.path.join(CSRC, "fd_internal.h"), os.path.join(ROOT, "include", "fd.h")]
+SOURCES = ["k_integral.cu", "k_cascade.cu", "k_cascade_ws.cu", "k_output.cu", "fd_api.cpp"]
+HEADERS = [os.path.join(CSRC, "fd_internal.h"), os.path.join(CSRC, "k_common.cuh"), os.path.join(ROOT, "include", "fd.h")]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 # --fmad=false: no FMA contraction anywhere (the kernels also use explicit __fmul_rn/__fadd_rn)
 NVFLAGS = ["-O3", "-lineinfo", "-std=c++17", "--fmad=false", "-Xcompiler", "-fPIC,-O2", "-I", os.path.join(ROOT, "include")]

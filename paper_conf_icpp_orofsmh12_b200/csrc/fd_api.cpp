@@ -80,8 +80,8 @@ void make_plan_dev(const fd_plan& pl, int W, int H, int pitch, int step, int G, 
     p->step = step;
     p->G = G;
     const int tx = k2_tx(step), ty = k2_ty(step);
-    long long ws = 0, col = 0, win = 0;
-    int bands = 0, tiles = 0, maxW = 0;
+    long long ws = 0, col = 0, win = 0, row = 0, cor = 0, lvl = 0;
+    int bands = 0, tiles = 0, maxW = 0, k1t = 0;
     for (int k = 0; k < pl.n_levels; ++k) {
         LevelDev& L = p->lv[k];
         L.W = pl.w[k];
@@ -94,21 +94,34 @@ void make_plan_dev(const fd_plan& pl, int W, int H, int pitch, int step, int G, 
         L.tile0 = tiles;
         L.tiles_x = (L.nx + tx - 1) / tx;
         L.r16 = (int)std::llround(pl.f[k] * 65536.0);
+        L.nchunks = (L.P + CHUNK - 1) / CHUNK;
+        L.k1t0 = k1t;
         L.ws_off = ws;
         L.col_off = col;
+        L.row_off = row;
+        L.cor_off = cor;
+        L.lvl_off = lvl;
         L.win0 = win;
+        lvl += (long long)L.H * L.P;
         bands += L.nbands;
+        k1t += L.nbands * L.nchunks;
         tiles += L.tiles_x * ((L.ny + ty - 1) / ty);
         ws += (long long)G * 2 * (L.H + 1) * L.P;
         col += (long long)L.nbands * 2 * L.W;
+        row += (long long)L.nbands * L.nchunks * 2 * BAND;
+        cor += (long long)L.nbands * L.nchunks * 2;
         win += pl.windows[k];
         maxW = L.W > maxW ? L.W : maxW;
     }
     p->bands_per_frame = bands;
     p->tiles_per_frame = tiles;
+    p->k1tiles_per_frame = k1t;
     p->maxW = maxW;
     p->win_per_frame = win;
     p->col_frame = col;
+    p->row_frame = row;
+    p->cor_frame = cor;
+    p->lvl_frame = lvl;
     p->ws_elems = ws;
 }
 
@@ -342,7 +355,8 @@ EncodeTiledFn encode_fn() {
     return fn;
 }
 
-fd_status encode_maps(const PlanDev& p, uint32_t* ws, int step, CUtensorMap* maps) {
+// box_planes: 2 = one TMA brings ii and sqii (k_cascade), 1 = one TMA per plane (k_cascade_ws)
+fd_status encode_maps(const PlanDev& p, uint32_t* ws, int step, int box_planes, CUtensorMap* maps) {
     EncodeTiledFn enc = encode_fn();
     if (!enc) return fail(FD_ECUDA, "cuTensorMapEncodeTiled unavailable");
     for (int k = 0; k < p.n_levels; ++k) {
@@ -350,7 +364,7 @@ fd_status encode_maps(const PlanDev& p, uint32_t* ws, int step, CUtensorMap* map
         cuuint64_t dims[4] = {(cuuint64_t)(L.W + 1), (cuuint64_t)(L.H + 1), 2, (cuuint64_t)p.G};
         cuuint64_t strides[3] = {(cuuint64_t)L.P * 4, (cuuint64_t)(L.H + 1) * L.P * 4,
                                  (cuuint64_t)2 * (L.H + 1) * L.P * 4};
-        cuuint32_t box[4] = {(cuuint32_t)tile_w(step), (cuuint32_t)tile_h(step), 2, 1};
+        cuuint32_t box[4] = {(cuuint32_t)tile_w(step), (cuuint32_t)tile_h(step), (cuuint32_t)box_planes, 1};
         cuuint32_t es[4] = {1, 1, 1, 1};
         CUresult r = enc(&maps[k], CU_TENSOR_MAP_DATA_TYPE_UINT32, 4, ws + L.ws_off, dims, strides, box, es,
                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -436,7 +450,20 @@ struct DevBuf {
 struct Workspace {
     int device = 0;
     std::mutex mu;                 // one call at a time per (device, stream)
-    DevBuf ws, colbuf, keys, scores, keys2, scores2, cubtmp, ctl, flev, frames, outbuf, group, grpout, tmaps, lvbuf;
+    DevBuf ws, colbuf, rowbuf, corbuf, lvlbuf, keys, scores, keys2, scores2, cubtmp, ctl, flev, frames, outbuf, group, grpout,
+        tmaps, lvbuf;
+    // K1 scratch for g frames of plan p
+    cudaError_t k1_scratch(const PlanDev& p, int g, K1Scratch* s) {
+        cudaError_t e = colbuf.ensure((size_t)g * p.col_frame * 4 + 16);
+        if (e == cudaSuccess) e = rowbuf.ensure((size_t)g * p.row_frame * 4 + 16);
+        if (e == cudaSuccess) e = corbuf.ensure((size_t)g * p.cor_frame * 8 + 16);
+        if (e == cudaSuccess) e = lvlbuf.ensure((size_t)g * p.lvl_frame + 16);
+        s->lvl = lvlbuf.as<uint8_t>();
+        s->col = colbuf.as<uint32_t>();
+        s->row = rowbuf.as<uint32_t>();
+        s->cor = corbuf.as<unsigned long long>();
+        return e;
+    }
     unsigned long long* h_pinned = nullptr;     // pinned host word(s) for count read-back
     std::unique_ptr<CascadeParams> params{new CascadeParams()};
     std::unique_ptr<PlanDev> plan{new PlanDev()};
@@ -501,7 +528,8 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     PlanDev& PD = *w->plan;
     make_plan_dev(pl, W, H, pitch, step, G, &PD);
     CK(w->ws.ensure((size_t)PD.ws_elems * 4));
-    CK(w->colbuf.ensure((size_t)G * PD.col_frame * 4 + 16));
+    K1Scratch k1s;
+    CK(w->k1_scratch(PD, G, &k1s));
     CK(w->ctl.ensure(256 + (size_t)ngroups * 4));
     CK(cudaMemsetAsync(w->ctl.p, 0, 256 + (size_t)ngroups * 4, st));
     if (!depth) {
@@ -510,8 +538,10 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         CK(w->scores.ensure(cap * 4));
     }
     // tensor maps + level table for K2 (global memory, copied in stream order)
+    // K2 variant: warp-specialised pipeline for step 1 (FD_K2_WS=1; experimental, off by default)
+    const bool use_ws = step == 1 && env_int("FD_K2_WS", 0) != 0;
     std::vector<CUtensorMap> maps((size_t)PD.n_levels);
-    s = encode_maps(PD, w->ws.as<uint32_t>(), step, maps.data());
+    s = encode_maps(PD, w->ws.as<uint32_t>(), step, use_ws ? 1 : 2, maps.data());
     if (s != FD_OK) return s;
     CK(w->tmaps.ensure(sizeof(CUtensorMap) * FD_MAX_LEVELS));
     CK(w->lvbuf.ensure(sizeof(LevelDev) * FD_MAX_LEVELS));
@@ -546,15 +576,21 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     for (int gi = 0; gi < ngroups; ++gi) {
         const int f0 = gi * G, gf = (n - f0) < G ? (n - f0) : G;
         const uint8_t* fr = d_frames + (size_t)f0 * H * pitch;
-        LAUNCH(FD_K_COLSUM, st, launch_colsum(fr, PD, gf, w->colbuf.as<uint32_t>(), st));
-        LAUNCH(FD_K_CARRY, st, launch_carry(PD, gf, w->colbuf.as<uint32_t>(), st));
-        LAUNCH(FD_K_BAND, st, launch_band(fr, PD, gf, w->colbuf.as<uint32_t>(), w->ws.as<uint32_t>(), st));
+        LAUNCH(FD_K_COLSUM, st, launch_k1_marg(fr, PD, gf, k1s, st));
+        {
+            ProfScope ps(FD_K_CARRY, st, 2);
+            CK(launch_k1_carry(PD, gf, k1s, st));
+        }
+        LAUNCH(FD_K_BAND, st, launch_k1_tiles(fr, PD, gf, k1s, w->ws.as<uint32_t>(), st));
         P.g_frames = gf;
         P.frame_base = f0;
         P.total_tiles = gf * PD.tiles_per_frame;
         P.tile_counter = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + gi;
         const int gr = grid < P.total_tiles ? grid : P.total_tiles;
-        LAUNCH(FD_K_CASCADE, st, launch_cascade(P, depth, step, gr, st));
+        if (use_ws)
+            LAUNCH(FD_K_CASCADE, st, launch_cascade_ws(P, depth, st));
+        else
+            LAUNCH(FD_K_CASCADE, st, launch_cascade(P, depth, step, gr, st));
     }
     return FD_OK;
 }
@@ -684,10 +720,14 @@ fd_status fd_integral(const uint8_t* d_img, int n, int W, int H, int pitch, uint
     r = get_ws(st, &w);
     if (r != FD_OK) return r;
     std::lock_guard<std::mutex> lk(w->mu);
-    CK(w->colbuf.ensure((size_t)n * p.col_frame * 4 + 16));
-    LAUNCH(FD_K_COLSUM, st, launch_colsum(d_img, p, n, w->colbuf.as<uint32_t>(), st));
-    LAUNCH(FD_K_CARRY, st, launch_carry(p, n, w->colbuf.as<uint32_t>(), st));
-    LAUNCH(FD_K_BAND, st, launch_integral_canonical(d_img, p, n, w->colbuf.as<uint32_t>(), d_ii, d_sqii, out_pitch, st));
+    K1Scratch k1s;
+    CK(w->k1_scratch(p, n, &k1s));
+    LAUNCH(FD_K_COLSUM, st, launch_k1_marg(d_img, p, n, k1s, st));
+    {
+        ProfScope ps(FD_K_CARRY, st, 2);
+        CK(launch_k1_carry(p, n, k1s, st));
+    }
+    LAUNCH(FD_K_BAND, st, launch_k1_tiles_canonical(d_img, p, n, k1s, d_ii, d_sqii, out_pitch, st));
     return FD_OK;
 }
 

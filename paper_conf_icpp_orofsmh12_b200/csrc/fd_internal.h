@@ -40,8 +40,13 @@ struct LevelDev {
     int band0, nbands;      // K1 bands (per frame)
     int tile0, tiles_x;     // K2 tiles (per frame); tiles_y = ceil(ny / TY)
     int r16;                // llround(f * 65536)  (f < 32768 enforced by the plan)
+    int nchunks;            // K1 128-column chunks (ceil(P / 128))
+    int k1t0;               // first K1 tile (band x chunk) of the level (per frame)
     long long ws_off;       // u32 elements
-    long long col_off;      // u32 elements (per frame)
+    long long col_off;      // u32 elements (per frame): column sums/carries [band][2][W]
+    long long row_off;      // u32 elements (per frame): row sums/carries [band][chunk][2][BAND]
+    long long cor_off;      // u64 elements (per frame): tile corners [band][chunk][2]
+    long long lvl_off;      // bytes (per frame): level image [H][P] written by K1a, read by K1b
     long long win0;         // first window index of the level within a frame
 };
 
@@ -53,6 +58,10 @@ struct PlanDev {
     int maxW;
     long long win_per_frame;
     long long col_frame;    // K1 scratch elements per frame
+    long long row_frame;    // K1 row-carry elements per frame
+    long long cor_frame;    // K1 corner elements (u64) per frame
+    long long lvl_frame;    // K1 level-image bytes per frame
+    int k1tiles_per_frame;  // K1 tiles (band x chunk) per frame
     long long ws_elems;     // group workspace elements (all levels, all g)
     int G;                  // frames per group (tensor-map extent)
     LevelDev lv[FD_MAX_LEVELS];
@@ -105,19 +114,32 @@ __host__ __device__ inline unsigned long long det_key(int frame, int level, int 
 }
 
 // ---- launchers (implemented in the .cu files) ----
-cudaError_t launch_colsum(const uint8_t* frames, const PlanDev& plan, int g_frames, uint32_t* colbuf,
-                          cudaStream_t st);
-cudaError_t launch_carry(const PlanDev& plan, int g_frames, uint32_t* colbuf, cudaStream_t st);
-cudaError_t launch_band(const uint8_t* frames, const PlanDev& plan, int g_frames, const uint32_t* colbuf,
-                        uint32_t* ws, cudaStream_t st);
-// canonical fd_integral output (u32 ii, u64 sqii) for n images with one level (f = 1)
-cudaError_t launch_integral_canonical(const uint8_t* img, const PlanDev& plan, int n, const uint32_t* colbuf,
+// K1 scratch for one launch of g_frames frames
+struct K1Scratch {
+    uint32_t* col;          // g_frames * col_frame
+    uint32_t* row;          // g_frames * row_frame
+    unsigned long long* cor;// g_frames * cor_frame
+    uint8_t* lvl;           // g_frames * lvl_frame (resampled level images, pitch P_k)
+};
+// K1 marginals: per (band, chunk) tile column sums and row sums of p and p^2
+cudaError_t launch_k1_marg(const uint8_t* frames, const PlanDev& plan, int g_frames, const K1Scratch& s,
+                           cudaStream_t st);
+// K1 carries: exclusive scans of the marginals over bands (columns) and chunks (rows), tile corners
+cudaError_t launch_k1_carry(const PlanDev& plan, int g_frames, const K1Scratch& s, cudaStream_t st);
+// K1 tiles: internal workspace (u32 ii + u32 sqii mod 2^32)
+cudaError_t launch_k1_tiles(const uint8_t* frames, const PlanDev& plan, int g_frames, const K1Scratch& s,
+                            uint32_t* ws, cudaStream_t st);
+// K1 tiles: canonical fd_integral output (u32 ii, u64 sqii) for n images with one level (f = 1)
+cudaError_t launch_k1_tiles_canonical(const uint8_t* img, const PlanDev& plan, int n, const K1Scratch& s,
                                       uint32_t* ii, uint64_t* sqii, int out_pitch, cudaStream_t st);
 cudaError_t launch_pyramid(const uint8_t* frames, const PlanDev& plan, int n, uint8_t* levels,
                            long long frame_stride, const long long* lvl_off_host, cudaStream_t st);
 cudaError_t launch_cascade(const CascadeParams& p, bool depth_mode, int step, int grid, cudaStream_t st);
 int cascade_grid(bool depth_mode, int step);       // persistent grid size (SMs x resident CTAs)
 size_t cascade_smem(int step);
+// warp-specialised K2 (step 1 only; one CTA per SM; tensor maps with a one-plane box)
+cudaError_t launch_cascade_ws(const CascadeParams& p, bool depth_mode, cudaStream_t st);
+size_t cascade_ws_smem();
 cudaError_t launch_keys_to_dets(const unsigned long long* keys, const float* scores, long long n,
                                 const double* f_levels_dev, int n_stages, fd_detection* out, cudaStream_t st);
 cudaError_t sort_pairs(void* tmp, size_t& tmp_bytes, const unsigned long long* kin, unsigned long long* kout,

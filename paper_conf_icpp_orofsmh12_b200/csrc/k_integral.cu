@@ -4,14 +4,13 @@
 // frame ... tex2D linear interpolation"; "integral images are computed ... with a
 // combination of parallel prefix sum [17][18] and matrix transposition operations [19]"
 // (P:L368-384).  B200 design: no level image and no transpose
-// is materialised.  Each level is cut into 32-row bands; a band CTA resamples its pixels
-// straight from the frame (exact integer bilinear, reading R2), does warp-shuffle row scans,
-// stages the row prefixes in shared memory and runs a coalesced, vectorised (uint4) column
-// scan that adds the carry of all rows above.  The carry comes from two light kernels
-// (per-band column sums, then an exclusive scan over bands), so ii/sqii are written to HBM
-// exactly once.
-#include <cub/cub.cuh>
-
+// is materialised.  Each level is cut into tiles of 32 rows x 128 ii columns.  A tile CTA
+// resamples its pixels straight from the frame (exact integer bilinear, reading R2), runs
+// warp-shuffle row scans, stages the row prefixes in shared memory and runs a coalesced,
+// vectorised (uint4) column scan.  Every tile is independent: its row carries (pixels left of
+// the tile), column carries (pixels above) and corner (ii at its top-left) come from three
+// light kernels over per-tile marginal sums, so ii/sqii are written to HBM exactly once and all
+// tiles of all levels of all frames of a group run in parallel.
 #include "fd_internal.h"
 
 namespace fdk {
@@ -67,63 +66,183 @@ __device__ __forceinline__ uint32_t level_pixel(const uint8_t* frame, int pitch,
     return bilinear(r, col_sample(srcW, r16, x));
 }
 
-__device__ __forceinline__ int find_level_band(const PlanDev& p, int b) {
+// The 4 pixels of row y at columns x0+4*lane .. +3 of a tile (0 beyond the level width).
+__device__ __forceinline__ void tile_row_pixels(const uint8_t* frame, const PlanDev& p, const LevelDev& L, int y, int x,
+                                                const ColSample* cs, uint32_t* pv) {
+    if (L.r16 == 65536) {
+        const uint8_t* row = frame + (size_t)y * p.pitch;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) pv[j] = x + j < L.W ? __ldg(row + x + j) : 0u;
+    } else {
+        const RowSample rs = row_sample(frame, p.pitch, p.H, L.r16, y);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) pv[j] = x + j < L.W ? bilinear(rs, cs[j]) : 0u;
+    }
+}
+
+__device__ __forceinline__ int find_level_k1(const PlanDev& p, int t) {
     int k = 0;
-    while (k + 1 < p.n_levels && p.lv[k + 1].band0 <= b) ++k;
+    while (k + 1 < p.n_levels && p.lv[k + 1].k1t0 <= t) ++k;
     return k;
 }
 
-// ---------------------------------------------------------------- K1a: per-band column sums
-__global__ void __launch_bounds__(K1_THREADS) k_colsum(const uint8_t* __restrict__ frames,
-                                                       const __grid_constant__ PlanDev p,
-                                                       uint32_t* __restrict__ colbuf) {
+// ---------------------------------------------------------------- K1a: per-tile marginals
+// colsum[band][plane][x] = sum over the tile's rows of p (plane 0) / p^2 (plane 1)
+// rowsum[band][chunk][plane][r] = sum over the tile's columns
+__global__ void __launch_bounds__(K1_THREADS) k_marg(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
+                                                     K1Scratch s) {
+    __shared__ uint32_t red_s[8][CHUNK], red_q[8][CHUNK];
     const int g = blockIdx.y;
-    const int k = find_level_band(p, blockIdx.x);
+    const int k = find_level_k1(p, blockIdx.x);
     const LevelDev& L = p.lv[k];
-    const int b = blockIdx.x - L.band0;
+    const int tl = blockIdx.x - L.k1t0;
+    const int b = tl / L.nchunks, c = tl % L.nchunks;
     const int y0 = b * BAND, rows = min(BAND, L.H - y0);
+    const int x0 = c * CHUNK;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint8_t* frame = frames + (size_t)g * p.H * p.pitch;
-    uint32_t* col = colbuf + (size_t)g * p.col_frame + L.col_off + (size_t)b * 2 * L.W;
-    for (int x = threadIdx.x; x < L.W; x += K1_THREADS) {
-        uint32_t s = 0, q = 0;
-        if (L.r16 == 65536) {
-            for (int r = 0; r < rows; ++r) {
-                const uint32_t v = __ldg(frame + (size_t)(y0 + r) * p.pitch + x);
-                s += v;
-                q += v * v;
+    const int x = x0 + 4 * lane;
+    ColSample cs[4];
+    if (L.r16 != 65536) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) cs[j] = col_sample(p.W, L.r16, min(x + j, L.W - 1));
+    }
+    uint32_t cols[4] = {0, 0, 0, 0}, colq[4] = {0, 0, 0, 0};
+    uint32_t* rowsum = s.row + (size_t)g * p.row_frame + L.row_off + (size_t)(b * L.nchunks + c) * 2 * BAND;
+    uint8_t* lvl = s.lvl + (size_t)g * p.lvl_frame + L.lvl_off;
+#pragma unroll
+    for (int i = 0; i < BAND / 8; ++i) {
+        const int r = warp + 8 * i;
+        if (r < rows) {
+            uint32_t pv[4];
+            tile_row_pixels(frame, p, L, y0 + r, x, cs, pv);
+            if (x < L.P)       // level image row, 4 pixels per lane as one aligned word (0 past W)
+                *reinterpret_cast<uint32_t*>(lvl + (size_t)(y0 + r) * L.P + x) =
+                    pv[0] | (pv[1] << 8) | (pv[2] << 16) | (pv[3] << 24);
+            uint32_t rs = 0, rq = 0;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                rs += pv[j];
+                rq += pv[j] * pv[j];
+                cols[j] += pv[j];
+                colq[j] += pv[j] * pv[j];
             }
-        } else {
-            const ColSample c = col_sample(p.W, L.r16, x);
-            for (int r = 0; r < rows; ++r) {
-                const uint32_t v = bilinear(row_sample(frame, p.pitch, p.H, L.r16, y0 + r), c);
-                s += v;
-                q += v * v;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                rs += __shfl_xor_sync(0xffffffffu, rs, o);
+                rq += __shfl_xor_sync(0xffffffffu, rq, o);
+            }
+            if (lane == 0) {
+                rowsum[r] = rs;
+                rowsum[BAND + r] = rq;
             }
         }
-        col[x] = s;
-        col[L.W + x] = q;
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        red_s[warp][4 * lane + j] = cols[j];
+        red_q[warp][4 * lane + j] = colq[j];
+    }
+    __syncthreads();
+    if (threadIdx.x < CHUNK) {
+        const int xx = x0 + threadIdx.x;
+        if (xx < L.W) {
+            uint32_t ts = 0, tq = 0;
+#pragma unroll
+            for (int w = 0; w < 8; ++w) {
+                ts += red_s[w][threadIdx.x];
+                tq += red_q[w][threadIdx.x];
+            }
+            uint32_t* col = s.col + (size_t)g * p.col_frame + L.col_off + (size_t)b * 2 * L.W;
+            col[xx] = ts;
+            col[L.W + xx] = tq;
+        }
     }
 }
 
-// ---------------------------------------------------------------- K1s: exclusive carry over bands
-__global__ void __launch_bounds__(K1_THREADS) k_carry(const __grid_constant__ PlanDev p, uint32_t* __restrict__ colbuf) {
-    const int k = blockIdx.y, g = blockIdx.z;
+// ---------------------------------------------------------------- K1s: exclusive carries
+// blockIdx.y <  n_levels: column carries of level y (exclusive over bands)
+// blockIdx.y >= n_levels: row carries of level y - n_levels (exclusive over chunks)
+__global__ void __launch_bounds__(K1_THREADS) k_carry(const __grid_constant__ PlanDev p, K1Scratch s) {
+    const int g = blockIdx.z;
+    const int i = blockIdx.x * K1_THREADS + threadIdx.x;
+    // exclusive scan of n strided pairs (plane 0 at v[0], plane 1 at v[off]); loads are batched
+    // 16 at a time so the latency is paid once per batch, not once per element
+    auto scan_pairs = [](uint32_t* v, int n, size_t stride, size_t off) {
+        uint32_t rs = 0, rq = 0;
+        for (int b0 = 0; b0 < n; b0 += 16) {
+            uint32_t a[16], q[16];
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+                if (b0 + j < n) {
+                    a[j] = v[(size_t)(b0 + j) * stride];
+                    q[j] = v[(size_t)(b0 + j) * stride + off];
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+                if (b0 + j < n) {
+                    v[(size_t)(b0 + j) * stride] = rs;
+                    v[(size_t)(b0 + j) * stride + off] = rq;
+                    rs += a[j];
+                    rq += q[j];
+                }
+            }
+        }
+    };
+    if ((int)blockIdx.y < p.n_levels) {
+        const LevelDev& L = p.lv[blockIdx.y];
+        if (i >= L.W) return;
+        scan_pairs(s.col + (size_t)g * p.col_frame + L.col_off + i, L.nbands, (size_t)2 * L.W, (size_t)L.W);
+    } else {
+        const LevelDev& L = p.lv[blockIdx.y - p.n_levels];
+        const int b = i / BAND, r = i % BAND;
+        if (b >= L.nbands) return;
+        scan_pairs(s.row + (size_t)g * p.row_frame + L.row_off + (size_t)b * L.nchunks * 2 * BAND + r, L.nchunks,
+                   (size_t)2 * BAND, (size_t)BAND);
+    }
+}
+
+// ---------------------------------------------------------------- K1c: tile corners
+// corner[band][chunk][plane] = ii at (y0, x0) = sum_{x < x0} colcarry_band[x]  (u64: exact for
+// the canonical u64 sqii; the internal workspace keeps its low 32 bits)
+__global__ void __launch_bounds__(K1_THREADS) k_corner(const __grid_constant__ PlanDev p, K1Scratch s) {
+    const int g = blockIdx.y;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int gb = blockIdx.x * (K1_THREADS / 32) + warp;      // band index within the frame
+    if (gb >= p.bands_per_frame) return;
+    int k = 0;
+    while (k + 1 < p.n_levels && p.lv[k + 1].band0 <= gb) ++k;
     const LevelDev& L = p.lv[k];
-    const int x = blockIdx.x * K1_THREADS + threadIdx.x;
-    if (x >= L.W) return;
-    uint32_t* col = colbuf + (size_t)g * p.col_frame + L.col_off + x;
-    uint32_t cs = 0, cq = 0;
-    for (int b = 0; b < L.nbands; ++b) {
-        uint32_t* c = col + (size_t)b * 2 * L.W;
-        const uint32_t s = c[0], q = c[L.W];
-        c[0] = cs;
-        c[L.W] = cq;
-        cs += s;
-        cq += q;
+    const int b = gb - L.band0;
+    const uint32_t* col = s.col + (size_t)g * p.col_frame + L.col_off + (size_t)b * 2 * L.W;
+    unsigned long long* cor = s.cor + (size_t)g * p.cor_frame + L.cor_off + (size_t)b * L.nchunks * 2;
+    unsigned long long run_s = 0, run_q = 0;
+    for (int c = 0; c < L.nchunks; ++c) {
+        unsigned long long ts = 0, tq = 0;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int x = c * CHUNK + 4 * lane + j;
+            if (x < L.W) {
+                ts += col[x];
+                tq += col[L.W + x];
+            }
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            ts += __shfl_xor_sync(0xffffffffu, ts, o);
+            tq += __shfl_xor_sync(0xffffffffu, tq, o);
+        }
+        if (lane == 0) {
+            cor[2 * c] = run_s;
+            cor[2 * c + 1] = run_q;
+        }
+        run_s += ts;
+        run_q += tq;
     }
 }
 
-// ---------------------------------------------------------------- K1b: band integral
+// ---------------------------------------------------------------- K1b: tile integral
 // CANON = false: internal layout (u32 ii + u32 sqii mod 2^32 in the group workspace planes)
 // CANON = true : fd_integral output (u32 ii, u64 sqii, caller pitch)
 template <bool CANON>
@@ -138,8 +257,8 @@ struct BandOut<true> {
 };
 
 template <bool CANON>
-__global__ void __launch_bounds__(K1_THREADS) k_band(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
-                                                     const uint32_t* __restrict__ colbuf, uint32_t* __restrict__ ws,
+__global__ void __launch_bounds__(K1_THREADS) k_tile(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
+                                                     K1Scratch s, uint32_t* __restrict__ ws,
                                                      uint32_t* __restrict__ out_ii,
                                                      unsigned long long* __restrict__ out_sq, int out_pitch) {
     using QT = typename BandOut<CANON>::QT;
@@ -151,15 +270,18 @@ __global__ void __launch_bounds__(K1_THREADS) k_band(const uint8_t* __restrict__
     __shared__ __align__(16) QT top_q[CHUNK];
 
     const int g = blockIdx.y;
-    const int k = find_level_band(p, blockIdx.x);
+    const int k = find_level_k1(p, blockIdx.x);
     const LevelDev& L = p.lv[k];
-    const int b = blockIdx.x - L.band0;
+    const int tl = blockIdx.x - L.k1t0;
+    const int b = tl / L.nchunks, c = tl % L.nchunks;
     const int y0 = b * BAND, rows = min(BAND, L.H - y0);
+    const int x0 = c * CHUNK;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint8_t* frame = frames + (size_t)g * p.H * p.pitch;
-    const uint32_t* carry = colbuf + (size_t)g * p.col_frame + L.col_off + (size_t)b * 2 * L.W;
+    const uint32_t* carry = s.col + (size_t)g * p.col_frame + L.col_off + (size_t)b * 2 * L.W;
+    const uint32_t* rowc = s.row + (size_t)g * p.row_frame + L.row_off + (size_t)(b * L.nchunks + c) * 2 * BAND;
+    const unsigned long long* cor = s.cor + (size_t)g * p.cor_frame + L.cor_off + (size_t)(b * L.nchunks + c) * 2;
 
-    // output addressing
     const int P = CANON ? out_pitch : L.P;
     uint32_t* o_ii;
     QT* o_sq;
@@ -172,172 +294,146 @@ __global__ void __launch_bounds__(K1_THREADS) k_band(const uint8_t* __restrict__
         o_sq = reinterpret_cast<QT*>(o_ii + plane);
     }
 
-    uint32_t rc_s[4] = {0, 0, 0, 0}, rc_q[4] = {0, 0, 0, 0};   // row carries (pixels < x0)
-    uint32_t tc_s = 0;                                          // top-row carry (warp 0)
-    QT tc_q = 0;
-
-    const int q4 = threadIdx.x & 31;        // column-phase: column group (4 ii columns)
-    const int sg = threadIdx.x >> 5;        // column-phase: 4-row segment
-
-    for (int x0 = 0; x0 < P; x0 += CHUNK) {
-        // ---- row phase: warp-shuffle scans of 4 rows per warp (+ the carry row for warp 0)
-        ColSample cs[4];
-        if (L.r16 != 65536) {
+    // ---- row phase: warp-shuffle exclusive scans of 4 rows per warp, plus the row carries;
+    // pixels come from the level image K1a wrote (one aligned 4-pixel word per lane)
+    const int x = x0 + 4 * lane;
+    const uint8_t* lvl = s.lvl + (size_t)g * p.lvl_frame + L.lvl_off;
+    (void)frame;
 #pragma unroll
-            for (int j = 0; j < 4; ++j) cs[j] = col_sample(p.W, L.r16, min(x0 + 4 * lane + j, L.W - 1));
-        }
+    for (int i = 0; i < BAND / 8; ++i) {
+        const int r = warp + 8 * i;
+        if (r < rows) {
+            uint32_t pv[4];
+            const uint32_t wv = x < L.P ? __ldg(reinterpret_cast<const uint32_t*>(lvl + (size_t)(y0 + r) * L.P + x)) : 0u;
 #pragma unroll
-        for (int i = 0; i < 4; ++i) {
-            const int r = warp + 8 * i;
-            if (r < rows) {
-                const int y = y0 + r;
-                uint32_t pv[4];
-                if (L.r16 == 65536) {
-                    const uint8_t* row = frame + (size_t)y * p.pitch;
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) {
-                        const int x = x0 + 4 * lane + j;
-                        pv[j] = x < L.W ? __ldg(row + x) : 0u;
-                    }
-                } else {
-                    const RowSample rs = row_sample(frame, p.pitch, p.H, L.r16, y);
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) pv[j] = (x0 + 4 * lane + j < L.W) ? bilinear(rs, cs[j]) : 0u;
-                }
-                uint32_t es[4], eq[4], ts = 0, tq = 0;
-#pragma unroll
-                for (int j = 0; j < 4; ++j) {
-                    es[j] = ts;
-                    eq[j] = tq;
-                    ts += pv[j];
-                    tq += pv[j] * pv[j];
-                }
-                uint32_t is = ts, iq = tq;    // warp inclusive scan of lane totals
-#pragma unroll
-                for (int d = 1; d < 32; d <<= 1) {
-                    const uint32_t a = __shfl_up_sync(0xffffffffu, is, d);
-                    const uint32_t c = __shfl_up_sync(0xffffffffu, iq, d);
-                    if (lane >= d) {
-                        is += a;
-                        iq += c;
-                    }
-                }
-                const uint32_t bs = rc_s[i] + is - ts, bq = rc_q[i] + iq - tq;
-                *reinterpret_cast<uint4*>(&rp_s[r][4 * lane]) = make_uint4(bs + es[0], bs + es[1], bs + es[2], bs + es[3]);
-                *reinterpret_cast<uint4*>(&rp_q[r][4 * lane]) = make_uint4(bq + eq[0], bq + eq[1], bq + eq[2], bq + eq[3]);
-                rc_s[i] += __shfl_sync(0xffffffffu, is, 31);
-                rc_q[i] += __shfl_sync(0xffffffffu, iq, 31);
-            }
-        }
-        if (warp == 0) {     // top row ii[y0][X] = sum_{x<X} carry[x]
-            uint32_t cv[4];
-            QT cq[4];
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                const int x = x0 + 4 * lane + j;
-                cv[j] = x < L.W ? carry[x] : 0u;
-                cq[j] = x < L.W ? (QT)carry[L.W + x] : (QT)0;
-            }
-            uint32_t es[4], ts = 0;
-            QT eq[4], tq = 0;
+            for (int j = 0; j < 4; ++j) pv[j] = (wv >> (8 * j)) & 255u;
+            uint32_t es[4], eq[4], ts = 0, tq = 0;
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
                 es[j] = ts;
                 eq[j] = tq;
-                ts += cv[j];
-                tq += cq[j];
+                ts += pv[j];
+                tq += pv[j] * pv[j];
             }
-            uint32_t is = ts;
-            QT iq = tq;
+            uint32_t is = ts, iq = tq;    // warp inclusive scan of lane totals
 #pragma unroll
             for (int d = 1; d < 32; d <<= 1) {
                 const uint32_t a = __shfl_up_sync(0xffffffffu, is, d);
-                const QT c = __shfl_up_sync(0xffffffffu, iq, d);
+                const uint32_t q = __shfl_up_sync(0xffffffffu, iq, d);
                 if (lane >= d) {
                     is += a;
-                    iq += c;
+                    iq += q;
                 }
             }
-            const uint32_t bs = tc_s + is - ts;
-            const QT bq = tc_q + iq - tq;
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                top_s[4 * lane + j] = bs + es[j];
-                top_q[4 * lane + j] = bq + eq[j];
-            }
-            tc_s += __shfl_sync(0xffffffffu, is, 31);
-            tc_q += __shfl_sync(0xffffffffu, iq, 31);
+            const uint32_t bs = rowc[r] + is - ts, bq = rowc[BAND + r] + iq - tq;
+            *reinterpret_cast<uint4*>(&rp_s[r][4 * lane]) = make_uint4(bs + es[0], bs + es[1], bs + es[2], bs + es[3]);
+            *reinterpret_cast<uint4*>(&rp_q[r][4 * lane]) = make_uint4(bq + eq[0], bq + eq[1], bq + eq[2], bq + eq[3]);
         }
-        __syncthreads();
+    }
+    if (warp == 0) {     // top row ii[y0][X] = corner + sum_{x0 <= x < X} carry[x]
+        uint32_t cv[4];
+        QT cq[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            cv[j] = x + j < L.W ? carry[x + j] : 0u;
+            cq[j] = x + j < L.W ? (QT)carry[L.W + x + j] : (QT)0;
+        }
+        uint32_t es[4], ts = 0;
+        QT eq[4], tq = 0;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            es[j] = ts;
+            eq[j] = tq;
+            ts += cv[j];
+            tq += cq[j];
+        }
+        uint32_t is = ts;
+        QT iq = tq;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            const uint32_t a = __shfl_up_sync(0xffffffffu, is, d);
+            const QT q = __shfl_up_sync(0xffffffffu, iq, d);
+            if (lane >= d) {
+                is += a;
+                iq += q;
+            }
+        }
+        const uint32_t bs = (uint32_t)cor[0] + is - ts;
+        const QT bq = (QT)cor[1] + iq - tq;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            top_s[4 * lane + j] = bs + es[j];
+            top_q[4 * lane + j] = bq + eq[j];
+        }
+    }
+    __syncthreads();
 
-        // ---- column phase: thread (q4, sg) owns ii columns x0+4q4.. and rows 4sg..4sg+3
-        {
-            uint32_t ss[4] = {0, 0, 0, 0};
-            QT sq[4] = {0, 0, 0, 0};
+    // ---- column phase: thread (q4, sg) owns ii columns x0+4q4.. and rows 4sg..4sg+3
+    const int q4 = threadIdx.x & 31;
+    const int sg = threadIdx.x >> 5;
+    {
+        uint32_t ss[4] = {0, 0, 0, 0};
+        QT sq[4] = {0, 0, 0, 0};
 #pragma unroll
-            for (int rr = 0; rr < 4; ++rr) {
-                const int r = 4 * sg + rr;
-                if (r < rows) {
-                    const uint4 a = *reinterpret_cast<const uint4*>(&rp_s[r][4 * q4]);
-                    const uint4 c = *reinterpret_cast<const uint4*>(&rp_q[r][4 * q4]);
-                    ss[0] += a.x; ss[1] += a.y; ss[2] += a.z; ss[3] += a.w;
-                    sq[0] += c.x; sq[1] += c.y; sq[2] += c.z; sq[3] += c.w;
-                }
-            }
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                seg_s[sg][4 * q4 + j] = ss[j];
-                seg_q[sg][4 * q4 + j] = sq[j];
+        for (int rr = 0; rr < 4; ++rr) {
+            const int r = 4 * sg + rr;
+            if (r < rows) {
+                const uint4 a = *reinterpret_cast<const uint4*>(&rp_s[r][4 * q4]);
+                const uint4 q = *reinterpret_cast<const uint4*>(&rp_q[r][4 * q4]);
+                ss[0] += a.x; ss[1] += a.y; ss[2] += a.z; ss[3] += a.w;
+                sq[0] += q.x; sq[1] += q.y; sq[2] += q.z; sq[3] += q.w;
             }
         }
-        __syncthreads();
-        {
-            uint32_t os[4];
-            QT oq[4];
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                os[j] = top_s[4 * q4 + j];
-                oq[j] = top_q[4 * q4 + j];
-            }
-            for (int s2 = 0; s2 < sg; ++s2) {
+        for (int j = 0; j < 4; ++j) {
+            seg_s[sg][4 * q4 + j] = ss[j];
+            seg_q[sg][4 * q4 + j] = sq[j];
+        }
+    }
+    __syncthreads();
+    uint32_t os[4];
+    QT oq[4];
 #pragma unroll
-                for (int j = 0; j < 4; ++j) {
-                    os[j] += seg_s[s2][4 * q4 + j];
-                    oq[j] += seg_q[s2][4 * q4 + j];
-                }
-            }
-            const int X = x0 + 4 * q4;
-            if (b == 0 && sg == 0 && X < P) {       // ii row 0 is zero
-                *reinterpret_cast<uint4*>(o_ii + X) = make_uint4(0, 0, 0, 0);
+    for (int j = 0; j < 4; ++j) {
+        os[j] = top_s[4 * q4 + j];
+        oq[j] = top_q[4 * q4 + j];
+    }
+    for (int s2 = 0; s2 < sg; ++s2) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            os[j] += seg_s[s2][4 * q4 + j];
+            oq[j] += seg_q[s2][4 * q4 + j];
+        }
+    }
+    const int X = x0 + 4 * q4;
+    if (b == 0 && sg == 0 && X < P) {       // ii row 0 is zero
+        *reinterpret_cast<uint4*>(o_ii + X) = make_uint4(0, 0, 0, 0);
+        if constexpr (CANON) {
+            *reinterpret_cast<ulonglong2*>(o_sq + X) = make_ulonglong2(0, 0);
+            *reinterpret_cast<ulonglong2*>(o_sq + X + 2) = make_ulonglong2(0, 0);
+        } else {
+            *reinterpret_cast<uint4*>(o_sq + X) = make_uint4(0, 0, 0, 0);
+        }
+    }
+#pragma unroll
+    for (int rr = 0; rr < 4; ++rr) {
+        const int r = 4 * sg + rr;
+        if (r < rows) {
+            const uint4 a = *reinterpret_cast<const uint4*>(&rp_s[r][4 * q4]);
+            const uint4 q = *reinterpret_cast<const uint4*>(&rp_q[r][4 * q4]);
+            os[0] += a.x; os[1] += a.y; os[2] += a.z; os[3] += a.w;
+            oq[0] += q.x; oq[1] += q.y; oq[2] += q.z; oq[3] += q.w;
+            if (X < P) {
+                const size_t o = (size_t)(y0 + r + 1) * P + X;
+                *reinterpret_cast<uint4*>(o_ii + o) = make_uint4(os[0], os[1], os[2], os[3]);
                 if constexpr (CANON) {
-                    *reinterpret_cast<ulonglong2*>(o_sq + X) = make_ulonglong2(0, 0);
-                    *reinterpret_cast<ulonglong2*>(o_sq + X + 2) = make_ulonglong2(0, 0);
+                    *reinterpret_cast<ulonglong2*>(o_sq + o) = make_ulonglong2(oq[0], oq[1]);
+                    *reinterpret_cast<ulonglong2*>(o_sq + o + 2) = make_ulonglong2(oq[2], oq[3]);
                 } else {
-                    *reinterpret_cast<uint4*>(o_sq + X) = make_uint4(0, 0, 0, 0);
-                }
-            }
-#pragma unroll
-            for (int rr = 0; rr < 4; ++rr) {
-                const int r = 4 * sg + rr;
-                if (r < rows) {
-                    const uint4 a = *reinterpret_cast<const uint4*>(&rp_s[r][4 * q4]);
-                    const uint4 c = *reinterpret_cast<const uint4*>(&rp_q[r][4 * q4]);
-                    os[0] += a.x; os[1] += a.y; os[2] += a.z; os[3] += a.w;
-                    oq[0] += c.x; oq[1] += c.y; oq[2] += c.z; oq[3] += c.w;
-                    if (X < P) {
-                        const size_t o = (size_t)(y0 + r + 1) * P + X;
-                        *reinterpret_cast<uint4*>(o_ii + o) = make_uint4(os[0], os[1], os[2], os[3]);
-                        if constexpr (CANON) {
-                            *reinterpret_cast<ulonglong2*>(o_sq + o) = make_ulonglong2(oq[0], oq[1]);
-                            *reinterpret_cast<ulonglong2*>(o_sq + o + 2) = make_ulonglong2(oq[2], oq[3]);
-                        } else {
-                            *reinterpret_cast<uint4*>(o_sq + o) = make_uint4(oq[0], oq[1], oq[2], oq[3]);
-                        }
-                    }
+                    *reinterpret_cast<uint4*>(o_sq + o) = make_uint4(oq[0], oq[1], oq[2], oq[3]);
                 }
             }
         }
-        __syncthreads();
     }
 }
 
@@ -356,30 +452,37 @@ __global__ void __launch_bounds__(256) k_pyramid(const uint8_t* __restrict__ fra
 }
 
 // ---------------------------------------------------------------- launchers
-cudaError_t launch_colsum(const uint8_t* frames, const PlanDev& plan, int g_frames, uint32_t* colbuf, cudaStream_t st) {
-    dim3 grid(plan.bands_per_frame, g_frames);
-    k_colsum<<<grid, K1_THREADS, 0, st>>>(frames, plan, colbuf);
+cudaError_t launch_k1_marg(const uint8_t* frames, const PlanDev& plan, int g_frames, const K1Scratch& s, cudaStream_t st) {
+    dim3 grid(plan.k1tiles_per_frame, g_frames);
+    k_marg<<<grid, K1_THREADS, 0, st>>>(frames, plan, s);
     return cudaGetLastError();
 }
 
-cudaError_t launch_carry(const PlanDev& plan, int g_frames, uint32_t* colbuf, cudaStream_t st) {
-    dim3 grid((plan.maxW + K1_THREADS - 1) / K1_THREADS, plan.n_levels, g_frames);
-    k_carry<<<grid, K1_THREADS, 0, st>>>(plan, colbuf);
+cudaError_t launch_k1_carry(const PlanDev& plan, int g_frames, const K1Scratch& s, cudaStream_t st) {
+    int maxb = 0;
+    for (int k = 0; k < plan.n_levels; ++k) maxb = plan.lv[k].nbands > maxb ? plan.lv[k].nbands : maxb;
+    const int span = plan.maxW > maxb * BAND ? plan.maxW : maxb * BAND;
+    dim3 grid((span + K1_THREADS - 1) / K1_THREADS, 2 * plan.n_levels, g_frames);
+    k_carry<<<grid, K1_THREADS, 0, st>>>(plan, s);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return e;
+    dim3 g2((plan.bands_per_frame + K1_THREADS / 32 - 1) / (K1_THREADS / 32), g_frames);
+    k_corner<<<g2, K1_THREADS, 0, st>>>(plan, s);
     return cudaGetLastError();
 }
 
-cudaError_t launch_band(const uint8_t* frames, const PlanDev& plan, int g_frames, const uint32_t* colbuf, uint32_t* ws,
-                        cudaStream_t st) {
-    dim3 grid(plan.bands_per_frame, g_frames);
-    k_band<false><<<grid, K1_THREADS, 0, st>>>(frames, plan, colbuf, ws, nullptr, nullptr, 0);
+cudaError_t launch_k1_tiles(const uint8_t* frames, const PlanDev& plan, int g_frames, const K1Scratch& s, uint32_t* ws,
+                            cudaStream_t st) {
+    dim3 grid(plan.k1tiles_per_frame, g_frames);
+    k_tile<false><<<grid, K1_THREADS, 0, st>>>(frames, plan, s, ws, nullptr, nullptr, 0);
     return cudaGetLastError();
 }
 
-cudaError_t launch_integral_canonical(const uint8_t* img, const PlanDev& plan, int n, const uint32_t* colbuf,
-                                      uint32_t* ii, uint64_t* sqii, int out_pitch, cudaStream_t st) {
-    dim3 grid(plan.bands_per_frame, n);
-    k_band<true><<<grid, K1_THREADS, 0, st>>>(img, plan, colbuf, nullptr, ii,
-                                               reinterpret_cast<unsigned long long*>(sqii), out_pitch);
+cudaError_t launch_k1_tiles_canonical(const uint8_t* img, const PlanDev& plan, int n, const K1Scratch& s, uint32_t* ii,
+                                      uint64_t* sqii, int out_pitch, cudaStream_t st) {
+    dim3 grid(plan.k1tiles_per_frame, n);
+    k_tile<true><<<grid, K1_THREADS, 0, st>>>(img, plan, s, nullptr, ii, reinterpret_cast<unsigned long long*>(sqii),
+                                              out_pitch);
     return cudaGetLastError();
 }
 
