@@ -28,8 +28,10 @@
 #ifndef FD_H
 #define FD_H
 
+#ifndef __CUDACC_RTC__ /* the K2 kernel source is also compiled at run time by NVRTC (fd_jit.cpp) */
 #include <stddef.h>
 #include <stdint.h>
+#endif
 
 #ifdef __cplusplus
 extern "C" {

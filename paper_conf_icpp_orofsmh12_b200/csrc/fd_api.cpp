@@ -6,6 +6,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cerrno>
 #include <cmath>
 #include <cstdarg>
@@ -20,6 +21,7 @@
 #include <vector>
 
 #include "fd_internal.h"
+#include "fd_jit.h"
 
 using namespace fdk;
 
@@ -170,7 +172,10 @@ struct fd_cascade_s {
         std::vector<StageDev> h_st;         // host copy (first PSTAGE_MAX go to the parameter bank)
     };
     std::map<int, Packed> packed;           // tile width -> packed records
+    fdk::JitK2* jit = nullptr;              // step-1 K2 specialised for this cascade (fd_jit.cpp)
+    bool jit_tried = false;
     ~fd_cascade_s() {
+        fdk::jit_k2_free(jit);
         for (auto& kv : packed) {
             cudaFree(kv.second.d_rec);
             cudaFree(kv.second.d_st);
@@ -267,7 +272,7 @@ fd_status parse_cascade(const char* text, size_t len, fd_cascade_s* c) {
 
 // Pack stumps for a tile width TW: each Haar feature is compiled into its distinct
 // integral-image corners with integer coefficients (sum_r wt_r * R_r, R = A + D - B - C).
-fd_status pack_cascade(fd_cascade_s* c, int TW, Packed* out) {
+fd_status pack_cascade(fd_cascade_s* c, int TW, Packed* out, bool upload = true) {
     std::vector<uint32_t> rec(c->stumps.size() * REC_WORDS, 0u);
     for (size_t j = 0; j < c->stumps.size(); ++j) {
         const HStump& s = c->stumps[j];
@@ -305,6 +310,11 @@ fd_status pack_cascade(fd_cascade_s* c, int TW, Packed* out) {
         for (int j = st[s].first; j < st[s].first + st[s].n; ++j)
             mc = (int)rec[(size_t)j * REC_WORDS] > mc ? (int)rec[(size_t)j * REC_WORDS] : mc;
         st[s].mc = mc;
+    }
+    if (!upload) {
+        out->h_rec = std::move(rec);
+        out->h_st = std::move(st);
+        return FD_OK;
     }
     uint4* d_rec = nullptr;
     StageDev* d_st = nullptr;
@@ -355,7 +365,7 @@ EncodeTiledFn encode_fn() {
     return fn;
 }
 
-// box_planes: 2 = one TMA brings ii and sqii (k_cascade), 1 = one TMA per plane (k_cascade_ws)
+// box_planes: 2 = one TMA brings ii and sqii of a tile (k_cascade), 1 = one plane per TMA
 fd_status encode_maps(const PlanDev& p, uint32_t* ws, int step, int box_planes, CUtensorMap* maps) {
     EncodeTiledFn enc = encode_fn();
     if (!enc) return fail(FD_ECUDA, "cuTensorMapEncodeTiled unavailable");
@@ -538,10 +548,8 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         CK(w->scores.ensure(cap * 4));
     }
     // tensor maps + level table for K2 (global memory, copied in stream order)
-    // K2 variant: warp-specialised pipeline for step 1 (FD_K2_WS=1; experimental, off by default)
-    const bool use_ws = step == 1 && env_int("FD_K2_WS", 0) != 0;
     std::vector<CUtensorMap> maps((size_t)PD.n_levels);
-    s = encode_maps(PD, w->ws.as<uint32_t>(), step, use_ws ? 1 : 2, maps.data());
+    s = encode_maps(PD, w->ws.as<uint32_t>(), step, 2, maps.data());
     if (s != FD_OK) return s;
     CK(w->tmaps.ensure(sizeof(CUtensorMap) * FD_MAX_LEVELS));
     CK(w->lvbuf.ensure(sizeof(LevelDev) * FD_MAX_LEVELS));
@@ -571,7 +579,22 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     P.depth = d_depth;
     P.score = d_score;
     P.stage_counts = d_stage_counts;
-    P.lane_min = env_int("FD_LANE_MIN", 32);
+    // deep stages with fewer than lane_min windows share lanes among a window's stumps; the
+    // group mode covers every window in one pass only while n <= threads / 2
+    const int half = k2_threads(step) / 2;
+    P.lane_min = std::max(1, std::min(env_int("FD_LANE_MIN", half + 1), half + 1));
+    // step 1: the K2 specialised for this cascade (compiled once, FD_JIT=0 selects the generic kernel)
+    JitK2* jit = nullptr;
+    if (step == 1 && env_int("FD_JIT", 1) != 0 && env_int("FD_K2_STAGES", 1) != 2) {
+        std::lock_guard<std::mutex> lk(c->mu);
+        if (!c->jit_tried) {
+            c->jit_tried = true;
+            std::string err;
+            c->jit = jit_k2_build(pk->h_rec.data(), pk->h_st.data(), (int)pk->h_st.size(), &err);
+            if (!c->jit) return fail(FD_ECUDA, "K2 specialisation: %s", err.c_str());
+        }
+        jit = c->jit;
+    }
     const int grid = cascade_grid(depth, step);
     for (int gi = 0; gi < ngroups; ++gi) {
         const int f0 = gi * G, gf = (n - f0) < G ? (n - f0) : G;
@@ -587,8 +610,13 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         P.total_tiles = gf * PD.tiles_per_frame;
         P.tile_counter = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + gi;
         const int gr = grid < P.total_tiles ? grid : P.total_tiles;
-        if (use_ws)
-            LAUNCH(FD_K_CASCADE, st, launch_cascade_ws(P, depth, st));
+        if (jit) {
+            std::string err;
+            ProfScope ps(FD_K_CASCADE, st);
+            const cudaError_t e = jit_k2_launch(jit, P, depth, st, &err);
+            if (e != cudaSuccess)
+                return fail(FD_ECUDA, "specialised K2: %s", err.empty() ? cudaGetErrorString(e) : err.c_str());
+        }
         else
             LAUNCH(FD_K_CASCADE, st, launch_cascade(P, depth, step, gr, st));
     }
@@ -663,6 +691,24 @@ fd_status fd_load_cascade(const char* text, size_t len, fd_cascade* out) {
     s = get_packed(c.get(), 1, &pk);         // upload the step-1 packing now
     if (s != FD_OK) return s;
     *out = c.release();
+    return FD_OK;
+}
+
+// Diagnostic (not in fd.h's stable set): generate and NVRTC-compile the step-1 K2 specialised
+// for a cascade text without touching a device.  FD_OK, or FD_ECUDA with the compiler log.
+fd_status fd_debug_jit_compile(const char* text, size_t len, size_t* cubin_bytes) {
+    if (!text) return fail(FD_EINVAL, "NULL argument");
+    std::unique_ptr<fd_cascade_s> c(new fd_cascade_s());
+    fd_status s = parse_cascade(text, len, c.get());
+    if (s != FD_OK) return s;
+    Packed pk;
+    s = pack_cascade(c.get(), tile_w(1), &pk, false);
+    if (s != FD_OK) return s;
+    std::vector<char> cubin;
+    std::string lowered, err;
+    if (!jit_k2_compile(jit_program(pk.h_rec.data(), pk.h_st.data(), (int)pk.h_st.size()), false, &cubin, &lowered, &err))
+        return fail(FD_ECUDA, "%s", err.c_str());
+    if (cubin_bytes) *cubin_bytes = cubin.size();
     return FD_OK;
 }
 

@@ -9,11 +9,25 @@
 //   K1 column-sum scratch (u32), per frame: colbuf + g*col_frame + lv.col_off +
 //     (band * 2 + plane) * W_k + x
 #pragma once
+#ifdef __CUDACC_RTC__
+// NVRTC build of the K2 kernel (fd_jit.cpp): no host headers; fixed-width types and an opaque
+// tensor-map type of the driver's size and alignment
+typedef unsigned char uint8_t;
+typedef unsigned short uint16_t;
+typedef unsigned int uint32_t;
+typedef unsigned long long uint64_t;
+typedef int int32_t;
+typedef long long int64_t;
+typedef struct alignas(64) { unsigned long long opaque[16]; } CUtensorMap;
+typedef struct CUstream_st* cudaStream_t;
+#include "fd.h"
+#else
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
 #include "../../include/fd.h"
+#endif
 
 namespace fdk {
 
@@ -21,16 +35,18 @@ constexpr int WIN = FD_WINDOW;       // 24
 constexpr int BAND = 32;             // K1 band height (rows)
 constexpr int CHUNK = 128;           // K1 chunk width (ii columns): 32 lanes x 4
 constexpr int K1_THREADS = 256;
-constexpr int K2_THREADS = 256;      // 8 warps
 constexpr int REC_WORDS = 16;        // packed stump record: 16 u32 (64 B)
 constexpr int MAX_CORNERS = 12;
 constexpr int MAX_STEP = 4;
 
 // K2 tile geometry per window step (windows per tile TX x TY; a thread owns WPT windows of a
-// column; warps tile the x extent in 32-lane columns).  step 1: 64 x 32 windows, 88 x 56 ii.
+// column; warps tile the x extent in 32-lane columns).  step 1: 8 warps, 64 x 32 windows,
+// 88 x 56 ii values per plane.  (32 x 32-window tiles with 4-warp CTAs, 5 resident per SM, were
+// measured 30% slower: the per-tile cost of the deep-stage sequence doubles with the tile count.)
+__host__ __device__ constexpr int k2_threads(int) { return 256; }
 __host__ __device__ constexpr int k2_tx(int step) { return step <= 3 ? 64 : 32; }
 __host__ __device__ constexpr int k2_wpt(int step) { return step == 1 ? 8 : (step == 2 ? 4 : (step == 3 ? 2 : 1)); }
-__host__ __device__ constexpr int k2_ty(int step) { return (8 / (k2_tx(step) / 32)) * k2_wpt(step); }
+__host__ __device__ constexpr int k2_ty(int step) { return (k2_threads(step) / 32 / (k2_tx(step) / 32)) * k2_wpt(step); }
 __host__ __device__ constexpr int tile_w(int step) { return (((k2_tx(step) - 1) * step + WIN + 1) + 3) & ~3; }
 __host__ __device__ constexpr int tile_h(int step) { return (k2_ty(step) - 1) * step + WIN + 1; }
 
@@ -137,9 +153,6 @@ cudaError_t launch_pyramid(const uint8_t* frames, const PlanDev& plan, int n, ui
 cudaError_t launch_cascade(const CascadeParams& p, bool depth_mode, int step, int grid, cudaStream_t st);
 int cascade_grid(bool depth_mode, int step);       // persistent grid size (SMs x resident CTAs)
 size_t cascade_smem(int step);
-// warp-specialised K2 (step 1 only; one CTA per SM; tensor maps with a one-plane box)
-cudaError_t launch_cascade_ws(const CascadeParams& p, bool depth_mode, cudaStream_t st);
-size_t cascade_ws_smem();
 cudaError_t launch_keys_to_dets(const unsigned long long* keys, const float* scores, long long n,
                                 const double* f_levels_dev, int n_stages, fd_detection* out, cudaStream_t st);
 cudaError_t sort_pairs(void* tmp, size_t& tmp_bytes, const unsigned long long* kin, unsigned long long* kout,

@@ -1,0 +1,268 @@
+// fd_jit.cpp -- run-time specialisation of K2 for one cascade (window step 1).
+//
+// The first stage runs on every window of every level (94.5% of windows stop there),
+// so its code is generated from the cascade and compiled with NVRTC for sm_100a:
+//   * every Haar corner becomes an immediate shared-memory offset and an immediate integer
+//     coefficient (no record loads, no corner decoding);
+//   * a thread owns WPT windows of one column (rows i = 0..WPT-1), so corner (dx, dy) of window i
+//     reads tile row dy + i: the stage's corners are grouped by column dx and each distinct
+//     (dx, row) value is loaded ONCE per thread and added into every (stump, window)
+//     accumulator that uses it (c3's first stage: 536 -> 236 shared loads per thread);
+//   * leaf decisions are kept as bits and the leaves are added in stump order at the end, so the
+//     fp32 stage sum is the exact sequence of the definition (oracle c7/c8).
+// The rest of the kernel is k_cascade.cu itself (embedded at build time, jit_sources.h) compiled
+// with -DFD_JIT_STAGE1.  Compiled once per cascade and cached on it.
+#include <nvrtc.h>
+
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <sstream>
+#include <string>
+#include <vector>
+
+#include "fd_internal.h"
+#include "fd_jit.h"
+#include "jit_sources.h"
+
+namespace fdk {
+
+struct JitK2 {
+    std::string key;                              // generated program (NVRTC source)
+    cudaKernel_t kern[2] = {nullptr, nullptr};    // [depth], compiled on first use
+    int grid[2] = {0, 0};
+    size_t smem = 0;
+};
+
+namespace {
+
+constexpr int JIT_STEP = 1;
+
+std::string hexf(uint32_t bits) {
+    char b[40];
+    std::snprintf(b, sizeof b, "__int_as_float(0x%08x)", bits);
+    return b;
+}
+
+}  // namespace
+
+std::string jit_stage1_source(const uint32_t* rec_words, int first, int n) {
+    constexpr int TW = tile_w(JIT_STEP), WPT = k2_wpt(JIT_STEP);
+    struct Use {
+        int s, i;
+        uint32_t coef;
+    };
+    std::map<int, std::map<int, std::vector<Use>>> cols;     // dx -> row -> uses
+    std::vector<int> last_dx(n, -1);
+    for (int s = 0; s < n; ++s) {
+        const uint32_t* r = rec_words + (size_t)(first + s) * REC_WORDS;
+        const int nc = (int)r[0];
+        for (int c = 0; c < nc; ++c) {
+            const uint32_t w = r[4 + c];
+            const int off = (int)(w & 0xffffu) / 4;
+            const uint32_t coef = (uint32_t)((int32_t)w >> 16);
+            const int dy = off / TW, dx = off % TW;
+            for (int i = 0; i < WPT; ++i) cols[dx][dy + i].push_back({s, i, coef});
+            if (dx > last_dx[s]) last_dx[s] = dx;
+        }
+    }
+    std::ostringstream o;
+    o << "namespace fdk {\n"
+      << "__device__ __forceinline__ void jit_stage1(const uint32_t* __restrict__ T, const float* nf, float* sm) {\n";
+    const int nm = (n + 31) / 32;
+    for (int s = 0; s < n; ++s)
+        for (int i = 0; i < WPT; ++i) o << "  uint32_t a" << s << "_" << i << " = 0u;\n";
+    for (int w = 0; w < nm; ++w)
+        for (int i = 0; i < WPT; ++i) o << "  uint32_t m" << w << "_" << i << " = 0u;\n";
+    for (const auto& col : cols) {
+        const int dx = col.first;
+        for (const auto& row : col.second) {
+            o << "  { const uint32_t v = T[" << row.first * TW + dx << "];";
+            for (const Use& u : row.second) {
+                o << " a" << u.s << "_" << u.i;
+                if (u.coef == 1u)
+                    o << " += v;";
+                else if (u.coef == 0xffffffffu)
+                    o << " -= v;";
+                else
+                    o << " += v * " << u.coef << "u;";
+            }
+            o << " }\n";
+        }
+        for (int s = 0; s < n; ++s) {
+            if (last_dx[s] != dx) continue;
+            const uint32_t* r = rec_words + (size_t)(first + s) * REC_WORDS;
+            for (int i = 0; i < WPT; ++i)
+                o << "  if (__int2float_rn((int)a" << s << "_" << i << ") < __fmul_rn(" << hexf(r[1]) << ", nf[" << i
+                  << "])) m" << s / 32 << "_" << i << " |= " << (1u << (s % 32)) << "u;\n";
+        }
+    }
+    for (int s = 0; s < n; ++s) {
+        const uint32_t* r = rec_words + (size_t)(first + s) * REC_WORDS;
+        if (last_dx[s] < 0) {       // a stump without corners: f = 0
+            for (int i = 0; i < WPT; ++i)
+                o << "  if (0.0f < __fmul_rn(" << hexf(r[1]) << ", nf[" << i << "])) m" << s / 32 << "_" << i
+                  << " |= " << (1u << (s % 32)) << "u;\n";
+        }
+    }
+    for (int s = 0; s < n; ++s) {
+        const uint32_t* r = rec_words + (size_t)(first + s) * REC_WORDS;
+        for (int i = 0; i < WPT; ++i)
+            o << "  sm[" << i << "] = __fadd_rn(sm[" << i << "], (m" << s / 32 << "_" << i << " & " << (1u << (s % 32))
+              << "u) ? " << hexf(r[2]) << " : " << hexf(r[3]) << ");\n";
+    }
+    o << "}\n}  // namespace fdk\n";
+    return o.str();
+}
+
+std::string jit_deep_source(const uint32_t* rec_words, const StageDev* st, int k_end) {
+    constexpr int TW = tile_w(JIT_STEP);
+    std::ostringstream o;
+    o << "namespace fdk {\n"
+      << "__device__ __forceinline__ float jit_deep(int s, const uint32_t* __restrict__ T, float nf) {\n"
+      << "  float sum = 0.0f;\n  switch (s) {\n";
+    for (int s = 1; s < k_end; ++s) {
+        o << "  case " << s << ":\n";
+        for (int j = st[s].first; j < st[s].first + st[s].n; ++j) {
+            const uint32_t* r = rec_words + (size_t)j * REC_WORDS;
+            const int nc = (int)r[0];
+            o << "    { const uint32_t f = 0u";
+            for (int c = 0; c < nc; ++c) {
+                const uint32_t w = r[4 + c];
+                const int off = (int)(w & 0xffffu) / 4;
+                const uint32_t coef = (uint32_t)((int32_t)w >> 16);
+                (void)TW;
+                if (coef == 1u)
+                    o << " + T[" << off << "]";
+                else if (coef == 0xffffffffu)
+                    o << " - T[" << off << "]";
+                else
+                    o << " + " << coef << "u * T[" << off << "]";
+            }
+            o << ";\n      sum = __fadd_rn(sum, (__int2float_rn((int)f) < __fmul_rn(" << hexf(r[1]) << ", nf)) ? "
+              << hexf(r[2]) << " : " << hexf(r[3]) << "); }\n";
+        }
+        o << "    break;\n";
+    }
+    o << "  }\n  return sum;\n}\n}  // namespace fdk\n";
+    return o.str();
+}
+
+int jit_deep_end(const StageDev* st, int n_stages) {
+    int budget = 60;                                   // generated deep stumps (code size bound)
+    if (const char* e = std::getenv("FD_JIT_DEEP_STUMPS")) budget = std::atoi(e);
+    int k = 1;
+    while (k < n_stages && st[k].n <= budget) budget -= st[k++].n;
+    return k;
+}
+
+std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages) {
+    const int k_end = jit_deep_end(st, n_stages);
+    std::string src = "#include \"fd_internal.h\"\n" + jit_stage1_source(rec_words, st[0].first, st[0].n) +
+                      "#define FD_JIT_STAGE1 1\n";
+    if (k_end > 1) src += jit_deep_source(rec_words, st, k_end) + "#define FD_JIT_DEEP " + std::to_string(k_end) + "\n";
+    return src + "#include \"k_cascade.cu\"\n";
+}
+
+bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cubin, std::string* lowered,
+                    std::string* err) {
+    const char* hdr_src[] = {jit_src_fd_h, jit_src_fd_internal_h, jit_src_k_common_cuh, jit_src_k_cascade_cu};
+    const char* hdr_names[] = {"fd.h", "fd_internal.h", "k_common.cuh", "k_cascade.cu"};
+    nvrtcProgram prog = nullptr;
+    if (nvrtcCreateProgram(&prog, source.c_str(), "k_cascade_jit.cu", 4, hdr_src, hdr_names) != NVRTC_SUCCESS) {
+        *err = "nvrtcCreateProgram failed";
+        return false;
+    }
+    const char* name = depth ? "fdk::k_cascade<1, true, 1>" : "fdk::k_cascade<1, false, 1>";
+    nvrtcAddNameExpression(prog, name);
+    const bool verbose = std::getenv("FD_JIT_VERBOSE") && std::getenv("FD_JIT_VERBOSE")[0] == '1';
+    const char* opts[] = {"-arch=sm_100a", "-std=c++17", "--fmad=false", "-lineinfo", "-default-device",
+                          "--ptxas-options=-v"};
+    const nvrtcResult rc = nvrtcCompileProgram(prog, verbose ? 6 : 5, opts);
+    size_t ln = 0;
+    nvrtcGetProgramLogSize(prog, &ln);
+    std::string log(ln, '\0');
+    if (ln) nvrtcGetProgramLog(prog, &log[0]);
+    if (verbose) std::fprintf(stderr, "fd: NVRTC K2 (depth=%d): %s\n", (int)depth, log.c_str());
+    if (rc != NVRTC_SUCCESS) {
+        *err = std::string("NVRTC: ") + nvrtcGetErrorString(rc) + "\n" + log.substr(0, 4000);
+        nvrtcDestroyProgram(&prog);
+        return false;
+    }
+    size_t cb = 0;
+    nvrtcGetCUBINSize(prog, &cb);
+    cubin->resize(cb);
+    nvrtcGetCUBIN(prog, cubin->data());
+    const char* lw = nullptr;
+    nvrtcGetLoweredName(prog, name, &lw);
+    *lowered = lw ? lw : "";
+    nvrtcDestroyProgram(&prog);
+    return true;
+}
+
+JitK2* jit_k2_build(const uint32_t* rec_words, const StageDev* st, int n_stages, std::string* err) {
+    (void)err;
+    std::unique_ptr<JitK2> J(new JitK2());
+    J->key = jit_program(rec_words, st, n_stages);
+    return J.release();
+}
+
+namespace {
+// process-wide cache: generated stage source + depth -> loaded kernel (cascades loaded again
+// with the same first stage reuse the compiled code)
+struct Loaded {
+    cudaLibrary_t lib = nullptr;
+    cudaKernel_t kern = nullptr;
+    int grid = 0;
+};
+std::mutex g_jit_mu;
+std::map<std::pair<std::string, int>, Loaded> g_jit_cache;
+}  // namespace
+
+cudaError_t jit_k2_launch(JitK2* J, const CascadeParams& p, bool depth, cudaStream_t st, std::string* err) {
+    const int d = depth ? 1 : 0;
+    if (!J->kern[d]) {
+        std::lock_guard<std::mutex> lk(g_jit_mu);
+        Loaded& L = g_jit_cache[{J->key, d}];
+        if (!L.kern) {
+            std::vector<char> cubin;
+            std::string lowered;
+            if (!jit_k2_compile(J->key, depth, &cubin, &lowered, err)) {
+                g_jit_cache.erase({J->key, d});
+                return cudaErrorInvalidSource;
+            }
+            cudaError_t e = cudaLibraryLoadData(&L.lib, cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0);
+            int dev = 0, sms = 0, per = 0;
+            const size_t smem = cascade_smem(JIT_STEP);
+            if (e == cudaSuccess) e = cudaLibraryGetKernel(&L.kern, L.lib, lowered.c_str());
+            if (e == cudaSuccess) e = cudaGetDevice(&dev);
+            if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+            if (e == cudaSuccess)
+                e = cudaKernelSetAttributeForDevice(L.kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem, dev);
+            if (e == cudaSuccess)
+                e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, reinterpret_cast<const void*>(L.kern), k2_threads(JIT_STEP),
+                                                                  smem);
+            if (e != cudaSuccess) {
+                *err = std::string("JIT kernel load: ") + cudaGetErrorString(e);
+                g_jit_cache.erase({J->key, d});
+                return e;
+            }
+            const char* cap = std::getenv("FD_K2_CTAS");      // diagnostic: resident CTAs per SM cap
+            if (cap && std::atoi(cap) > 0 && std::atoi(cap) < per) per = std::atoi(cap);
+            L.grid = sms * (per > 0 ? per : 1);
+        }
+        J->kern[d] = L.kern;
+        J->grid[d] = L.grid;
+        J->smem = cascade_smem(JIT_STEP);
+    }
+    const int grid = J->grid[d] < p.total_tiles ? J->grid[d] : p.total_tiles;
+    void* args[] = {const_cast<CascadeParams*>(&p)};
+    return cudaLaunchKernel(reinterpret_cast<const void*>(J->kern[d]), dim3(grid), dim3(k2_threads(JIT_STEP)), args, J->smem, st);
+}
+
+void jit_k2_free(JitK2* J) { delete J; }    // loaded code stays in the process-wide cache
+
+}  // namespace fdk

@@ -1,0 +1,27 @@
+// fd_jit.h -- run-time specialised K2 (fd_jit.cpp); host-only, not part of the C ABI.
+#pragma once
+#include <string>
+#include <vector>
+
+#include "fd_internal.h"
+
+namespace fdk {
+
+struct JitK2;
+// CUDA source of the generated first stage (stage index `first`..first+n of the packed step-1
+// records, REC_WORDS u32 per stump)
+std::string jit_stage1_source(const uint32_t* rec_words, int first, int n);
+// generated deep stages [1, k_end) (lane-per-window code with immediate corner offsets)
+std::string jit_deep_source(const uint32_t* rec_words, const StageDev* st, int k_end);
+// the whole NVRTC program for a cascade (generated stages + k_cascade.cu)
+std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages);
+// NVRTC compile only (no device needed): cubin + lowered name of k_cascade<1, depth, 1>
+bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cubin, std::string* lowered,
+                    std::string* err);
+// specialisation handle for one cascade (code generated now, compiled and loaded on first launch)
+JitK2* jit_k2_build(const uint32_t* rec_words, const StageDev* st, int n_stages, std::string* err);
+// launch (compiling on first use; cudaErrorInvalidSource + *err when NVRTC fails)
+cudaError_t jit_k2_launch(JitK2* j, const CascadeParams& p, bool depth, cudaStream_t st, std::string* err);
+void jit_k2_free(JitK2* j);
+
+}  // namespace fdk

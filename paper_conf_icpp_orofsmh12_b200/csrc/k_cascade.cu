@@ -24,23 +24,27 @@
 
 namespace fdk {
 
-#ifdef FD_K2_TIMING
+#if defined(FD_K2_TIMING) && !defined(__CUDACC_RTC__)
 // [0] tiles, [1] TMA-wait cycles, [2] stage-1 cycles, [3] deep-stage cycles, [4+s] tiles whose
-// deepest stage loop ended at s (diagnostic build only: -DFD_K2_TIMING)
-__device__ unsigned long long g_k2_timing[16];
+// deepest stage loop ended at s, [16+s] cycles of deep stage s (block-wide loop iteration),
+// [48+s] tiles that ran deep stage s, [80] tail cycles, [81] tails, [82] mode-M cycles,
+// [83] mode-L cycles (diagnostic build only: -DFD_K2_TIMING)
+__device__ unsigned long long g_k2_timing[128];
 extern "C" int fd_debug_k2_timing(unsigned long long* out, int reset) {
     if (cudaMemcpyFromSymbol(out, g_k2_timing, sizeof(g_k2_timing)) != cudaSuccess) return -1;
     if (reset) {
-        unsigned long long z[16] = {};
+        unsigned long long z[128] = {};
         cudaMemcpyToSymbol(g_k2_timing, z, sizeof(z));
     }
     return 0;
 }
 #endif
 
-constexpr int GL = 8;                        // lanes per window in the sparse deep mode
-constexpr int WPW = 32 / GL;                 // windows per warp in the sparse deep mode
-constexpr int LEAF_CHUNK = 64;               // leaves parked per window before the ordered sum
+#ifndef FD_JIT_DEEP
+#define FD_JIT_DEEP 0        // run-time specialised kernel: deep stages [1, FD_JIT_DEEP) are generated code
+#endif
+
+constexpr int LC = 8;                        // leaves parked per lane before the ordered sum (group mode)
 
 template <int STEP>
 struct TileGeo {
@@ -54,7 +58,8 @@ struct TileGeo {
     static constexpr int BOX = 2 * PLANE;          // ii + sqii (one TMA box)
     static constexpr int BUF = (BOX + 255) & ~255; // buffer stride: keeps every TMA destination 1 KB aligned
     static constexpr int NW = TX * TY;             // windows per tile
-    static constexpr size_t LEAVES = (size_t)(K2_THREADS / 32) * WPW * LEAF_CHUNK;   // floats
+    static constexpr int THREADS = k2_threads(STEP);
+    static constexpr size_t LEAVES = (size_t)THREADS * LC;   // floats
     static constexpr size_t smem(int nst) {
         return (size_t)nst * BUF * 4 + (size_t)NW * 4 * 2 + LEAVES * 4 + (size_t)NW * 2 * 2;
     }
@@ -63,14 +68,14 @@ struct TileGeo {
 // NST = TMA stages: 2 = double-buffered tiles (prefetch the next tile during evaluation),
 // 1 = single buffer with one more resident CTA per SM.
 template <int STEP, bool DEPTH, int NST>
-__global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const __grid_constant__ CascadeParams p) {
+__global__ void __launch_bounds__(k2_threads(STEP), k2_threads(STEP) == 128 ? 5 : (NST == 1 ? 3 : 2)) k_cascade(const __grid_constant__ CascadeParams p) {
     using G = TileGeo<STEP>;
     constexpr int TW = G::TW, TX = G::TX, TY = G::TY, WPT = G::WPT;
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint32_t* tiles = reinterpret_cast<uint32_t*>(smem_raw);               // [NST][2][TH][TW]
     float* nfs = reinterpret_cast<float*>(tiles + NST * G::BUF);            // [NW] per-window nf
     float* sums = nfs + G::NW;                                              // [NW] last stage sum
-    float* leaves = sums + G::NW;                                           // [8 warps][WPW][LEAF_CHUNK]
+    float* leaves = sums + G::NW;                                           // [8 warps][LC][32]
     uint16_t* lists = reinterpret_cast<uint16_t*>(leaves + G::LEAVES);      // [2][NW]
     __shared__ __align__(8) uint64_t mbar[2];
     __shared__ int s_tile[2], s_lvl[2], s_tl[2];
@@ -156,10 +161,16 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
             nfs[(ly0 + i) * TX + lx] = nf[i];
             sm[i] = 0.0f;
         }
+#ifdef FD_JIT_STAGE1
+        // run-time specialised first stage (fd_jit.cpp): corner offsets, coefficients and
+        // thresholds are immediates and each (column, row) value is loaded once per thread
+        jit_stage1(T + base, nf, sm);
+#else
         if (st0.first + st0.n <= p.n_pstumps)
             dense_stage<WPT, STEP * TW>(T, base, nf, sm, prec, st0.first, st0.n);
         else
             dense_stage<WPT, STEP * TW>(T, base, nf, sm, grec, st0.first, st0.n);
+#endif
 
         // compaction of stage-1 survivors into lists[1] (count s_cnt[1])
 #pragma unroll
@@ -201,55 +212,39 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
         auto deep_stage = [&](const StageDev& sd, int n) {
             const uint16_t* lin = lists + (s & 1) * G::NW;
             uint16_t* lout = lists + ((s + 1) & 1) * G::NW;
-            if (n < p.lane_min) {
-                // few survivors: GL lanes per window (WPW windows per warp), the group's lanes
-                // evaluate different stumps in parallel and park the leaves in shared memory;
-                // the group leader then adds them in stump order (the exact fp32 sequence of
-                // the definition).
-                const int grp = lane / GL, q = lane % GL;
-                float* lv = leaves + (warp * WPW + grp) * LEAF_CHUNK;
-                for (int e0 = warp * WPW; e0 < n; e0 += (K2_THREADS / 32) * WPW) {
-                    const int e = e0 + grp;
-                    const bool act = e < n;
-                    const int idx = act ? lin[e] : 0;
-                    const int wlx = idx % TX, wly = idx / TX;
-                    const int b = wly * STEP * TW + wlx * STEP;
-                    const float nfw = nfs[idx];
-                    float sum = 0.0f;
-                    for (int c0 = 0; c0 < sd.n; c0 += LEAF_CHUNK) {
-                        const int cn = min(LEAF_CHUNK, sd.n - c0);
-                        if (act)
-                            for (int j = q; j < cn; j += GL)
-                                lv[j] = eval_stage(T, b, nfw, grec, sd.first + c0 + j, 1, sd.mc);
-                        __syncwarp();
-                        if (act && q == 0) {
-                            int t2 = 0;
-                            for (; t2 + 8 <= cn; t2 += 8) {         // loads batched, additions in order
-                                const float4 a = *reinterpret_cast<const float4*>(lv + t2);
-                                const float4 c = *reinterpret_cast<const float4*>(lv + t2 + 4);
-                                sum = __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(sum, a.x), a.y), a.z), a.w);
-                                sum = __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(sum, c.x), c.y), c.z), c.w);
-                            }
-                            for (; t2 < cn; ++t2) sum = __fadd_rn(sum, lv[t2]);
-                        }
-                        __syncwarp();
-                    }
-                    if (act && q == 0) {
-                        if (sum >= sd.T) {
-                            lout[atomicAdd(&s_cnt[(s + 1) % 3], 1)] = (uint16_t)idx;
-                            sums[idx] = sum;
-                        } else if (DEPTH) {
-                            const long long o = (long long)frame * p.win_per_frame + L.win0 +
-                                                (long long)(wy0 + wly) * L.nx + (wx0 + wlx);
-                            p.depth[o] = (uint8_t)(s < 255 ? s : 255);
-                            p.score[o] = sum;
-                        }
+            // stages [1, FD_JIT_DEEP) of the run-time specialised kernel: immediate-offset code,
+            // always one lane per window
+            const bool jit_s = FD_JIT_DEEP > 0 && s < FD_JIT_DEEP;
+            if (!jit_s && n < p.lane_min) {
+                // fewer windows than half the block: GL = 2^lg lanes per window (the largest
+                // power of two with n*GL <= THREADS, so one pass covers every window and
+                // all warps work); the group's lanes evaluate different stumps, the leader adds
+                // the leaves in stump order (the exact fp32 sequence of the definition).
+                int lg = 1;
+                while (lg < 5 && (n << (lg + 1)) <= G::THREADS) ++lg;
+                const int e = tid >> lg;
+                const bool act = e < n;
+                const int idx = act ? lin[e] : 0;
+                const int wlx = idx % TX, wly = idx / TX;
+                const int b = wly * STEP * TW + wlx * STEP;
+                const float nfw = act ? nfs[idx] : 1.0f;
+                const float sum = group_stage<LC>(T, b, nfw, grec, sd.first, sd.n, sd.mc, lg, act,
+                                                  leaves + warp * 32 * LC, lane);
+                if (act && (lane & ((1 << lg) - 1)) == 0) {
+                    if (sum >= sd.T) {
+                        lout[atomicAdd(&s_cnt[(s + 1) % 3], 1)] = (uint16_t)idx;
+                        sums[idx] = sum;
+                    } else if (DEPTH) {
+                        const long long o = (long long)frame * p.win_per_frame + L.win0 +
+                                            (long long)(wy0 + wly) * L.nx + (wx0 + wlx);
+                        p.depth[o] = (uint8_t)(s < 255 ? s : 255);
+                        p.score[o] = sum;
                     }
                 }
                 return;
             }
             const bool in_param = sd.first + sd.n <= p.n_pstumps;
-            for (int e0 = warp * 32; e0 < n; e0 += K2_THREADS) {
+            for (int e0 = warp * 32; e0 < n; e0 += G::THREADS) {
                 const int e = e0 + lane;
                 const bool act = e < n;
                 int idx = 0;
@@ -258,8 +253,13 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
                     idx = lin[e];
                     const int wlx = idx % TX, wly = idx / TX;
                     const int b = wly * STEP * TW + wlx * STEP;
-                    sum = in_param ? eval_stage(T, b, nfs[idx], prec, sd.first, sd.n, sd.mc)
-                                   : eval_stage(T, b, nfs[idx], grec, sd.first, sd.n, sd.mc);
+#if FD_JIT_DEEP > 0
+                    if (jit_s)
+                        sum = jit_deep(s, T + b, nfs[idx]);
+                    else
+#endif
+                        sum = in_param ? eval_stage(T, b, nfs[idx], prec, sd.first, sd.n, sd.mc)
+                                       : eval_stage(T, b, nfs[idx], grec, sd.first, sd.n, sd.mc);
                 }
                 const bool pass = act && (sum >= sd.T);
                 if (DEPTH && act && !pass) {
@@ -283,10 +283,13 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
         };
         bool tail_done = false;
         for (; s < N; ++s) {
+#ifdef FD_K2_TIMING
+            const long long ts0 = clock64();
+#endif
             const int n = s_cnt[s % 3];
             if (tid == 0 && p.stage_counts && n) atomicAdd(p.stage_counts + s, (unsigned long long)n);
             if (n == 0) break;
-            if (n <= K2_THREADS / 32) {
+            if (n <= G::THREADS / 32 && !(FD_JIT_DEEP > 0 && s < FD_JIT_DEEP)) {
                 // tail: at most one window per warp left -- each warp walks its window through
                 // all remaining stages on its own (one stump per lane, leaves added in stump
                 // order via shuffles), so no block barrier is paid per stage.
@@ -347,6 +350,12 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
                     }
                 }
                 tail_done = true;
+#ifdef FD_K2_TIMING
+                if (lane == 0 && warp < n) {
+                    atomicAdd(&g_k2_timing[80], (unsigned long long)(clock64() - ts0));
+                    atomicAdd(&g_k2_timing[81], 1ull);
+                }
+#endif
                 break;
             }
             if (tid == 0) s_cnt[(s + 2) % 3] = 0;
@@ -363,6 +372,15 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
                 deep_stage(sd, n);
             }
             __syncthreads();
+#ifdef FD_K2_TIMING
+            if (tid == 0) {
+                const unsigned long long dt = (unsigned long long)(clock64() - ts0);
+                const int si = s < 32 ? s : 31;
+                atomicAdd(&g_k2_timing[16 + si], dt);
+                atomicAdd(&g_k2_timing[48 + si], 1ull);
+                atomicAdd(&g_k2_timing[n < p.lane_min ? 82 : 83], dt);
+            }
+#endif
         }
 #ifdef FD_K2_TIMING
         if (tid == 0) {
@@ -378,7 +396,7 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
             const int nacc = s_cnt[N % 3];
             if (tid == 0 && p.stage_counts && nacc) atomicAdd(p.stage_counts + N, (unsigned long long)nacc);
             const uint16_t* lacc = lists + (N & 1) * G::NW;
-            for (int e0 = warp * 32; e0 < nacc; e0 += K2_THREADS) {
+            for (int e0 = warp * 32; e0 < nacc; e0 += G::THREADS) {
                 const int e = e0 + lane;
                 const bool act = e < nacc;
                 int idx = act ? lacc[e] : 0;
@@ -408,6 +426,7 @@ __global__ void __launch_bounds__(K2_THREADS, NST == 1 ? 3 : 2) k_cascade(const 
     }
 }
 
+#ifndef __CUDACC_RTC__
 // TMA stages (FD_K2_STAGES=1|2, default 1: measured faster, 3 CTAs/SM hide more latency)
 static int k2_stages() {
     static int v = [] {
@@ -422,7 +441,7 @@ static cudaError_t launch_one(const CascadeParams& p, int grid, cudaStream_t st)
     const size_t smem = TileGeo<STEP>::smem(NST);
     cudaError_t e = cudaFuncSetAttribute(k_cascade<STEP, DEPTH, NST>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    k_cascade<STEP, DEPTH, NST><<<grid, K2_THREADS, smem, st>>>(p);
+    k_cascade<STEP, DEPTH, NST><<<grid, k2_threads(STEP), smem, st>>>(p);
     return cudaGetLastError();
 }
 
@@ -433,7 +452,7 @@ static int grid_one() {
     int dev = 0, sms = 0, per = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_cascade<STEP, DEPTH, NST>, K2_THREADS, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_cascade<STEP, DEPTH, NST>, k2_threads(STEP), smem);
     return sms * (per > 0 ? per : 1);
 }
 
@@ -475,5 +494,7 @@ cudaError_t launch_cascade(const CascadeParams& p, bool depth, int step, int gri
         default: return cudaErrorInvalidValue;
     }
 }
+
+#endif  // !__CUDACC_RTC__
 
 }  // namespace fdk

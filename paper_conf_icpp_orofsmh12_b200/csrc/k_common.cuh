@@ -101,6 +101,47 @@ __device__ __forceinline__ float eval_stage(const uint32_t* __restrict__ T, int 
     return eval_stage_mc<MAX_CORNERS>(T, b, nf, rec, first, n);
 }
 
+// One stage for one window evaluated by a group of GL = 2^lg lanes (lane-aligned within a warp).
+// Per chunk of GL*LC stumps, lane q of the group evaluates stumps c0 + q + GL*r (r < LC,
+// independent, so LC loads are in flight) and parks the leaves at lv[r*32 + lane]
+// (conflict-free); the group leader (q == 0) then adds them in stump order, which keeps the
+// exact fp32 sequence of the definition (oracle c8).  The returned sum is valid in the leader.
+template <int MC, int LC>
+__device__ __forceinline__ float group_stage_mc(const uint32_t* __restrict__ T, int b, float nf, const GlobalRec& rec,
+                                                int first, int n, int lg, bool act, float* lv, int lane) {
+    const int gl = 1 << lg, q = lane & (gl - 1), g0 = lane & ~(gl - 1);
+    float sum = 0.0f;
+    for (int c0 = 0; c0 < n; c0 += gl * LC) {
+        if (act) {
+            float l[LC];
+#pragma unroll
+            for (int r = 0; r < LC; ++r) {
+                const int j = c0 + q + (r << lg);
+                l[r] = j < n ? eval_stump_mc<MC>(T, b, nf, rec, first + j) : 0.0f;
+            }
+#pragma unroll
+            for (int r = 0; r < LC; ++r) lv[r * 32 + lane] = l[r];
+        }
+        __syncwarp();
+        if (act && q == 0) {
+            const int cn = min(gl * LC, n - c0);
+#pragma unroll 8
+            for (int j = 0; j < cn; ++j) sum = __fadd_rn(sum, lv[(j >> lg) * 32 + g0 + (j & (gl - 1))]);
+        }
+        __syncwarp();
+    }
+    return sum;
+}
+
+template <int LC>
+__device__ __forceinline__ float group_stage(const uint32_t* __restrict__ T, int b, float nf, const GlobalRec& rec,
+                                             int first, int n, int mc, int lg, bool act, float* lv, int lane) {
+    if (mc <= 6) return group_stage_mc<6, LC>(T, b, nf, rec, first, n, lg, act, lv, lane);
+    if (mc <= 8) return group_stage_mc<8, LC>(T, b, nf, rec, first, n, lg, act, lv, lane);
+    if (mc <= 9) return group_stage_mc<9, LC>(T, b, nf, rec, first, n, lg, act, lv, lane);
+    return group_stage_mc<MAX_CORNERS, LC>(T, b, nf, rec, first, n, lg, act, lv, lane);
+}
+
 // Dense first stage: each thread owns WPT windows of one column (stride STEP*TW words in
 // shared memory).  The corner count nc is warp-uniform; common counts get a fully unrolled,
 // branch-free body.

@@ -74,3 +74,16 @@ def test_detect_rejects_null_cascade():
     st = L.fd_detect(None, buf.ctypes.data_as(C.c_void_p), 1, 24, 24, 24, 24, 1.1, 1, None, 0, C.byref(cnt), None)
     assert st == fd.FD_EINVAL
     assert b"cascade" in L.fd_last_error()
+
+
+@pytest.mark.parametrize("name", ["c1.fdc", "c3.fdc"])
+def test_specialised_k2_compiles_without_gpu(name):
+    """The step-1 K2 specialised for a cascade (fd_jit.cpp) is generated and NVRTC-compiled for
+    sm_100a; no device is touched."""
+    L = fd.lib()
+    L.fd_debug_jit_compile.argtypes = [C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]
+    text = open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "cascades", name), "rb").read()
+    n = C.c_size_t(0)
+    rc = L.fd_debug_jit_compile(text, len(text), C.byref(n))
+    assert rc == 0, fd.last_error() if hasattr(fd, "last_error") else rc
+    assert n.value > 100000

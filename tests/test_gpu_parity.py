@@ -115,6 +115,16 @@ def test_depth_maps_bit_exact_1080p():
     compare_depth(cascades(3), fr, 1.1)
 
 
+def test_depth_maps_generic_k2(monkeypatch):
+    """Step 1 runs the K2 specialised per cascade by default (fd_jit.cpp); the generic kernel
+    (FD_JIT=0) must agree too."""
+    monkeypatch.setenv("FD_JIT", "0")
+    fr, _ = gen(2, 3, 2)
+    compare_depth(cascades(2), fr, 1.2)
+    fr, _ = gen(3, 0, 1)
+    compare_depth(cascades(3), fr, 1.1)
+
+
 @pytest.mark.parametrize("step", [2, 3, 4])
 def test_depth_maps_step(step):
     fr, _ = gen(2, 7, 2)
