@@ -285,7 +285,7 @@ def run_ours(args):
     hbm = float(peaks.get("hbm_gbs", 6650.0))
     k1_ach = k1_bytes / (k1_ms / 1000.0) / 1e9 if k1_ms > 0 else None
     tr_k2, tr_k1 = ncu_traffic()
-    my_launches = sum(prof[k][0] for k in ("colsum", "carry", "band", "cascade", "dets", "group"))
+    my_launches = sum(prof[k][0] for k in ("colsum", "carry", "band", "cascade", "deep", "tail", "dets", "group"))
     step_ms = ms / args.steps
     out = {
         "metric": METRIC, "value": value, "unit": "frames/s", "n_gpus": world, "steps": args.steps,

@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define FD_ABI_VERSION 1
+#define FD_ABI_VERSION 2
 #define FD_MAX_LEVELS 128
 #define FD_WINDOW 24 /* fixed 24x24 sliding window, image scaled instead (Fig. 2) */
 
@@ -165,10 +165,14 @@ fd_status fd_detect_group_host(fd_cascade c, const uint8_t* h_frames, int n, int
 /* Kernel accounting (process-wide, all devices): number of launches of each kernel class
  * since the last fd_profile_reset and, if time_kernels != 0, their summed device time
  * measured with CUDA events recorded on the launching stream around each launch.
- * FD_K_SORT is the CUB radix sort (library code, counted as one call). */
+ * FD_K_SORT is the CUB radix sort (library code, counted as one call).  The cascade evaluator
+ * is FD_K_CASCADE (the dense first stage, k_stage1), FD_K_DEEP (the deeper stages over batches
+ * of tiles, k_deep) and FD_K_TAIL (the deep stages of the few windows left per batch, one warp
+ * per window). */
 typedef enum {
     FD_K_COLSUM = 0, FD_K_CARRY = 1, FD_K_BAND = 2, FD_K_CASCADE = 3,
-    FD_K_SORT = 4, FD_K_DETS = 5, FD_K_GROUP = 6, FD_K_PYRAMID = 7, FD_K_COUNT = 8
+    FD_K_SORT = 4, FD_K_DETS = 5, FD_K_GROUP = 6, FD_K_PYRAMID = 7, FD_K_TAIL = 8,
+    FD_K_DEEP = 9, FD_K_COUNT = 10
 } fd_kernel_kind;
 typedef struct {
     int64_t launches[FD_K_COUNT];

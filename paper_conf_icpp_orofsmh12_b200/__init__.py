@@ -48,11 +48,11 @@ class _Plan(C.Structure):
                 ("windows", C.c_int64 * FD_MAX_LEVELS), ("total_windows", C.c_int64)]
 
 
-K_NAMES = ["colsum", "carry", "band", "cascade", "sort", "dets", "group", "pyramid"]
+K_NAMES = ["colsum", "carry", "band", "cascade", "sort", "dets", "group", "pyramid", "tail", "deep"]
 
 
 class _Profile(C.Structure):
-    _fields_ = [("launches", C.c_int64 * 8), ("ms", C.c_double * 8)]
+    _fields_ = [("launches", C.c_int64 * len(K_NAMES)), ("ms", C.c_double * len(K_NAMES))]
 
 
 def library_path() -> str:
@@ -307,7 +307,7 @@ def fd_profile_read() -> dict:
     """{kernel: (launches, ms)} since the last fd_profile_reset."""
     p = _Profile()
     _check(lib().fd_profile_read(C.byref(p)))
-    return {K_NAMES[k]: (int(p.launches[k]), float(p.ms[k])) for k in range(8)}
+    return {K_NAMES[k]: (int(p.launches[k]), float(p.ms[k])) for k in range(len(K_NAMES))}
 
 
 def fd_release_workspaces():

@@ -168,6 +168,7 @@ struct fd_cascade_s {
     struct Packed {
         uint4* d_rec = nullptr;             // device records (REC_WORDS u32 per stump)
         StageDev* d_st = nullptr;
+        uint32_t* d_trec = nullptr;         // SoA tail records (k_tail): [TAIL_REC_WORDS][n_stumps]
         std::vector<uint32_t> h_rec;        // host copy (first PREC_MAX go to the parameter bank)
         std::vector<StageDev> h_st;         // host copy (first PSTAGE_MAX go to the parameter bank)
     };
@@ -179,6 +180,7 @@ struct fd_cascade_s {
         for (auto& kv : packed) {
             cudaFree(kv.second.d_rec);
             cudaFree(kv.second.d_st);
+            cudaFree(kv.second.d_trec);
         }
     }
 };
@@ -274,6 +276,8 @@ fd_status parse_cascade(const char* text, size_t len, fd_cascade_s* c) {
 // integral-image corners with integer coefficients (sum_r wt_r * R_r, R = A + D - B - C).
 fd_status pack_cascade(fd_cascade_s* c, int TW, Packed* out, bool upload = true) {
     std::vector<uint32_t> rec(c->stumps.size() * REC_WORDS, 0u);
+    const size_t ns = c->stumps.size();
+    std::vector<uint32_t> trec((size_t)TAIL_REC_WORDS * (ns ? ns : 1), 0u);   // SoA, offsets in TAIL_RP pitch
     for (size_t j = 0; j < c->stumps.size(); ++j) {
         const HStump& s = c->stumps[j];
         int coef[WIN + 1][WIN + 1];
@@ -294,12 +298,14 @@ fd_status pack_cascade(fd_cascade_s* c, int TW, Packed* out, bool upload = true)
                     const uint32_t off = (uint32_t)(y * TW + x) * 4u;     // byte offset in the smem tile
                     if (off > 0xffffu) return fail(FD_EINVAL, "tile too wide for 16-bit corner offsets");
                     R[4 + nc] = off | ((uint32_t)(coef[y][x] & 0xffff) << 16);
+                    trec[(size_t)(4 + nc) * ns + j] = (uint32_t)(y * TAIL_RP + x) | ((uint32_t)(coef[y][x] & 0xffff) << 16);
                     ++nc;
                 }
         R[0] = (uint32_t)nc;
         std::memcpy(&R[1], &s.theta, 4);
         std::memcpy(&R[2], &s.left, 4);
         std::memcpy(&R[3], &s.right, 4);
+        for (int w = 0; w < 4; ++w) trec[(size_t)w * ns + j] = R[w];
     }
     std::vector<StageDev> st(c->stages.size());
     for (size_t s = 0; s < st.size(); ++s) {
@@ -322,6 +328,10 @@ fd_status pack_cascade(fd_cascade_s* c, int TW, Packed* out, bool upload = true)
     CK(cudaMalloc(&d_st, st.size() * sizeof(StageDev)));
     CK(cudaMemcpy(d_rec, rec.data(), rec.size() * 4, cudaMemcpyHostToDevice));
     CK(cudaMemcpy(d_st, st.data(), st.size() * sizeof(StageDev), cudaMemcpyHostToDevice));
+    uint32_t* d_trec = nullptr;
+    CK(cudaMalloc(&d_trec, trec.size() * 4));
+    CK(cudaMemcpy(d_trec, trec.data(), trec.size() * 4, cudaMemcpyHostToDevice));
+    out->d_trec = d_trec;
     out->d_rec = d_rec;
     out->d_st = d_st;
     out->h_rec = std::move(rec);
@@ -461,7 +471,7 @@ struct Workspace {
     int device = 0;
     std::mutex mu;                 // one call at a time per (device, stream)
     DevBuf ws, colbuf, rowbuf, corbuf, lvlbuf, keys, scores, keys2, scores2, cubtmp, ctl, flev, frames, outbuf, group, grpout,
-        tmaps, lvbuf;
+        tmaps, lvbuf, tailq, surv, tilerec;
     // K1 scratch for g frames of plan p
     cudaError_t k1_scratch(const PlanDev& p, int g, K1Scratch* s) {
         cudaError_t e = colbuf.ensure((size_t)g * p.col_frame * 4 + 16);
@@ -540,8 +550,23 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     CK(w->ws.ensure((size_t)PD.ws_elems * 4));
     K1Scratch k1s;
     CK(w->k1_scratch(PD, G, &k1s));
-    CK(w->ctl.ensure(256 + (size_t)ngroups * 4));
-    CK(cudaMemsetAsync(w->ctl.p, 0, 256 + (size_t)ngroups * 4, st));
+    // ctl: [0] detection count, [256 B..] per-group K2 tile counters, then per-group tail counts,
+    // survivor counts and k_deep tile counters
+    CK(w->ctl.ensure(256 + (size_t)ngroups * 16));
+    CK(cudaMemsetAsync(w->ctl.p, 0, 256 + (size_t)ngroups * 16, st));
+    // K2 split in two kernels (k_stage1: dense first stage, k_deep: batched deeper stages;
+    // FD_K2_SPLIT=0 runs the fused k_cascade).  Survivor list sized for the worst case.
+    const bool split = env_int("FD_K2_SPLIT", 1) != 0;
+    const bool deep1 = env_int("FD_K2_DEEP1", 1) != 0;      // k_deep1 (tile per small CTA) or batched k_deep
+    if (split) {
+        CK(w->surv.ensure((size_t)G * (size_t)PD.win_per_frame * 8 + 16));
+        CK(w->tilerec.ensure((size_t)G * PD.tiles_per_frame * 8 + 16));
+    }
+    // tail queue (k_tail): FD_TAIL=0 keeps every window inside K2; FD_TAIL_N = windows left in a
+    // batch at which it hands them over; FD_TAIL_CAP = queue entries (16 B each) per group
+    const bool use_tail = env_int("FD_TAIL", 1) != 0;
+    const int tail_cap = use_tail ? std::max(1024, env_int("FD_TAIL_CAP", 1 << 22)) : 0;
+    if (use_tail) CK(w->tailq.ensure((size_t)tail_cap * 16));
     if (!depth) {
         const size_t cap = (size_t)(det_cap > 0 ? det_cap : 1);
         CK(w->keys.ensure(cap * 8));
@@ -549,7 +574,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     }
     // tensor maps + level table for K2 (global memory, copied in stream order)
     std::vector<CUtensorMap> maps((size_t)PD.n_levels);
-    s = encode_maps(PD, w->ws.as<uint32_t>(), step, 2, maps.data());
+    s = encode_maps(PD, w->ws.as<uint32_t>(), step, 1, maps.data());
     if (s != FD_OK) return s;
     CK(w->tmaps.ensure(sizeof(CUtensorMap) * FD_MAX_LEVELS));
     CK(w->lvbuf.ensure(sizeof(LevelDev) * FD_MAX_LEVELS));
@@ -583,9 +608,30 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     // group mode covers every window in one pass only while n <= threads / 2
     const int half = k2_threads(step) / 2;
     P.lane_min = std::max(1, std::min(env_int("FD_LANE_MIN", half + 1), half + 1));
+    P.tail_q = use_tail ? w->tailq.as<uint4>() : nullptr;
+    P.tail_cap = tail_cap;
+    P.tail_n = std::max(1, env_int("FD_TAIL_N", 8));
+    TailParams TP;
+    TP.q = P.tail_q;
+    TP.cap = tail_cap;
+    TP.step = step;
+    TP.ws = w->ws.as<uint32_t>();
+    TP.lv = P.lv;
+    TP.trec = pk->d_trec;
+    TP.ns = (int)c->stumps.size();
+    TP.stages = pk->d_st;
+    TP.n_stages = P.n_stages;
+    TP.win_per_frame = P.win_per_frame;
+    TP.det_count = P.det_count;
+    TP.det_keys = P.det_keys;
+    TP.det_scores = P.det_scores;
+    TP.det_cap = P.det_cap;
+    TP.depth = d_depth;
+    TP.score = d_score;
+    TP.stage_counts = d_stage_counts;
     // step 1: the K2 specialised for this cascade (compiled once, FD_JIT=0 selects the generic kernel)
     JitK2* jit = nullptr;
-    if (step == 1 && env_int("FD_JIT", 1) != 0 && env_int("FD_K2_STAGES", 1) != 2) {
+    if (step == 1 && env_int("FD_JIT", 1) != 0) {
         std::lock_guard<std::mutex> lk(c->mu);
         if (!c->jit_tried) {
             c->jit_tried = true;
@@ -609,16 +655,36 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         P.frame_base = f0;
         P.total_tiles = gf * PD.tiles_per_frame;
         P.tile_counter = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + gi;
+        P.tail_count = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + ngroups + gi;
+        P.surv_count = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + 2 * ngroups + gi;
+        P.deep_counter = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + 3 * ngroups + gi;
+        P.surv = split ? w->surv.as<uint2>() : nullptr;
+        P.tile_rec = split ? w->tilerec.as<uint2>() : nullptr;
         const int gr = grid < P.total_tiles ? grid : P.total_tiles;
         if (jit) {
             std::string err;
-            ProfScope ps(FD_K_CASCADE, st);
-            const cudaError_t e = jit_k2_launch(jit, P, depth, st, &err);
+            cudaError_t e;
+            {
+                ProfScope ps(FD_K_CASCADE, st);
+                e = jit_k2_launch(jit, P, depth, split ? JIT_STAGE1 : JIT_FUSED, st, &err);
+            }
+            if (e == cudaSuccess && split) {
+                ProfScope ps(FD_K_DEEP, st);
+                e = jit_k2_launch(jit, P, depth, deep1 ? JIT_DEEP1 : JIT_DEEP, st, &err);
+            }
             if (e != cudaSuccess)
                 return fail(FD_ECUDA, "specialised K2: %s", err.empty() ? cudaGetErrorString(e) : err.c_str());
-        }
-        else
+        } else if (split) {
+            LAUNCH(FD_K_CASCADE, st, launch_stage1(P, depth, step, st));
+            LAUNCH(FD_K_DEEP, st, deep1 ? launch_deep1(P, depth, step, st) : launch_deep(P, depth, step, st));
+        } else {
             LAUNCH(FD_K_CASCADE, st, launch_cascade(P, depth, step, gr, st));
+        }
+        if (use_tail) {
+            TP.count = P.tail_count;
+            TP.frame_base = f0;
+            LAUNCH(FD_K_TAIL, st, launch_tail(TP, depth, st));
+        }
     }
     return FD_OK;
 }
@@ -705,7 +771,8 @@ fd_status fd_debug_jit_compile(const char* text, size_t len, size_t* cubin_bytes
     s = pack_cascade(c.get(), tile_w(1), &pk, false);
     if (s != FD_OK) return s;
     std::vector<char> cubin;
-    std::string lowered, err;
+    std::vector<std::string> lowered;
+    std::string err;
     if (!jit_k2_compile(jit_program(pk.h_rec.data(), pk.h_st.data(), (int)pk.h_st.size()), false, &cubin, &lowered, &err))
         return fail(FD_ECUDA, "%s", err.c_str());
     if (cubin_bytes) *cubin_bytes = cubin.size();

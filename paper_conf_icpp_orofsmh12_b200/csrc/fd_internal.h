@@ -49,6 +49,76 @@ __host__ __device__ constexpr int k2_wpt(int step) { return step == 1 ? 8 : (ste
 __host__ __device__ constexpr int k2_ty(int step) { return (k2_threads(step) / 32 / (k2_tx(step) / 32)) * k2_wpt(step); }
 __host__ __device__ constexpr int tile_w(int step) { return (((k2_tx(step) - 1) * step + WIN + 1) + 3) & ~3; }
 __host__ __device__ constexpr int tile_h(int step) { return (k2_ty(step) - 1) * step + WIN + 1; }
+// split K2 (k_stage1 + k_deep): tiles per k_deep batch (ii-only slots)
+#ifndef FD_K2B_NB
+#define FD_K2B_NB 4
+#endif
+__host__ __device__ constexpr int k2b_min_ctas(int nb) { return nb <= 4 ? 2 : 1; }
+__host__ __device__ constexpr int k2_pbuf(int step) { return (tile_w(step) * tile_h(step) + 31) & ~31; }
+
+
+// Fused K2 (k_cascade) shared memory: the tile's ii plane, then its sqii plane -- which, once
+// stage 1 has taken every window's variance from it, holds the stage-1 survivor pool
+// (nf f32[NW], window u16[NW]) and the two per-stage lists (u16[2][NW]).
+template <int STEP>
+struct TileGeo {
+    static constexpr int PBUF = k2_pbuf(STEP);                          // ii plane (u32)
+    static constexpr int NW = k2_tx(STEP) * k2_ty(STEP);
+    static constexpr int CP = NW;                                       // pool capacity (a whole tile)
+    static constexpr int QBUF = ((PBUF > NW * 10 / 4 ? PBUF : NW * 10 / 4) + 31) & ~31;
+    static constexpr size_t OFF_Q = (size_t)PBUF * 4;
+#ifdef FD_POOL_SEPARATE
+    static constexpr size_t OFF_NF = OFF_Q + (size_t)QBUF * 4;
+#else
+    static constexpr size_t OFF_NF = OFF_Q;                             // pool in the sqii buffer
+#endif
+    static constexpr size_t OFF_LOC = OFF_NF + (size_t)NW * 4;
+    static constexpr size_t OFF_LIST = OFF_LOC + (size_t)NW * 2;
+#ifdef FD_POOL_SEPARATE
+    static constexpr size_t SMEM = OFF_LIST + (size_t)NW * 4;
+#else
+    static constexpr size_t SMEM = OFF_Q + (size_t)QBUF * 4;
+#endif
+};
+#ifndef FD_K2_CTAS
+#define FD_K2_CTAS 4                        // fused K2: resident CTAs per SM the launch bounds target
+#endif
+
+// k_stage1 (K2a): one tile's ii + sqii planes and its survivor list (window index, nf bits)
+template <int STEP>
+struct TileGeoA {
+    static constexpr int PBUF = k2_pbuf(STEP);
+    static constexpr int NW = k2_tx(STEP) * k2_ty(STEP);
+    static constexpr size_t OFF_SURV = (size_t)2 * PBUF * 4;
+    static constexpr size_t SMEM = OFF_SURV + (size_t)NW * 8;
+};
+
+// k_deep (K2b): NB ii slots, the pool of their stage-1 survivors, per-stage lists, group leaves
+template <int STEP, int NB>
+struct TileGeoB {
+    static constexpr int PBUF = k2_pbuf(STEP);
+    static constexpr int NW = k2_tx(STEP) * k2_ty(STEP);
+    static constexpr int CP = NB <= 4 ? NW + 512 : NW + 2048;   // pool capacity (>= one full tile)
+    static constexpr size_t OFF_NF = (size_t)NB * PBUF * 4;
+    static constexpr size_t OFF_LOC = OFF_NF + (size_t)CP * 4;
+    static constexpr size_t OFF_LIST = OFF_LOC + (((size_t)CP * 2 + 15) & ~(size_t)15);
+    static constexpr size_t SMEM = OFF_LIST + (size_t)2 * CP * 2;
+};
+
+// k_deep1: one ii slot, a pool chunk of CP survivors and its two per-stage lists
+#ifndef FD_K2D_CTAS
+#define FD_K2D_CTAS 6
+#endif
+constexpr int K2D_THREADS = 128;
+template <int STEP>
+struct TileGeoD {
+    static constexpr int PBUF = k2_pbuf(STEP);
+    static constexpr int CP = 512;
+    static constexpr size_t OFF_NF = (size_t)PBUF * 4;
+    static constexpr size_t OFF_LOC = OFF_NF + (size_t)CP * 4;
+    static constexpr size_t OFF_LIST = OFF_LOC + (size_t)CP * 2;
+    static constexpr size_t SMEM = OFF_LIST + (size_t)2 * CP * 2;
+};
 
 struct LevelDev {
     int W, H, P;            // level size, ii pitch (elements)
@@ -118,9 +188,43 @@ struct alignas(16) CascadeParams {
     float* score;
     unsigned long long* stage_counts;       // n_stages + 1, may be null
     int n_pstages;                          // stages [0, n_pstages) are also in pstages
-    int pad0;
+    int tail_n;                             // a batch with <= tail_n windows left goes to the tail queue
+    uint4* tail_q;                          // tail queue (k_tail.cu), may be null
+    unsigned int* tail_count;               // entries appended (may exceed tail_cap: the excess stays in K2)
+    int tail_cap;
+    int pad1;
+    uint2* surv;                            // split K2: stage-1 survivors (window index, nf bits)
+    uint2* tile_rec;                        // split K2: per tile (offset into surv, count)
+    unsigned int* surv_count;
+    unsigned int* deep_counter;             // k_deep tile claims
     StageDev pstages[PSTAGE_MAX];
     uint4 prec[PREC_MAX * (REC_WORDS / 4)];
+};
+
+// Tail queue entry (k_cascade -> k_tail): x = g(16) | level(8) | stage(8), y = wyi(16) | wxi(16)
+// (window indices in the level's step grid), z = nf bits, w = 0.
+constexpr int TAIL_RP = 25;                 // row pitch of a window's ii region staged by k_tail
+constexpr int TAIL_REC_WORDS = 13;          // SoA tail records: nc, theta, left, right, 9 corners
+struct TailParams {
+    const uint4* q;
+    const unsigned int* count;
+    int cap;
+    int step;
+    const uint32_t* ws;                     // group workspace (ii plane 0 read)
+    const LevelDev* lv;
+    const uint32_t* trec;                   // [TAIL_REC_WORDS][ns] corner offsets in TAIL_RP pitch
+    int ns;
+    const StageDev* stages;
+    int n_stages;
+    int frame_base;
+    long long win_per_frame;
+    unsigned long long* det_count;
+    unsigned long long* det_keys;
+    float* det_scores;
+    long long det_cap;
+    uint8_t* depth;
+    float* score;
+    unsigned long long* stage_counts;
 };
 
 // detection key: frame(24) | level(8) | wy(16) | wx(16)
@@ -151,6 +255,11 @@ cudaError_t launch_k1_tiles_canonical(const uint8_t* img, const PlanDev& plan, i
 cudaError_t launch_pyramid(const uint8_t* frames, const PlanDev& plan, int n, uint8_t* levels,
                            long long frame_stride, const long long* lvl_off_host, cudaStream_t st);
 cudaError_t launch_cascade(const CascadeParams& p, bool depth_mode, int step, int grid, cudaStream_t st);
+cudaError_t launch_tail(const TailParams& p, bool depth_mode, cudaStream_t st);
+// split K2: k_stage1 then k_deep (precompiled kernels; step 1 normally runs the NVRTC ones)
+cudaError_t launch_stage1(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
+cudaError_t launch_deep(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
+cudaError_t launch_deep1(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
 int cascade_grid(bool depth_mode, int step);       // persistent grid size (SMs x resident CTAs)
 size_t cascade_smem(int step);
 cudaError_t launch_keys_to_dets(const unsigned long long* keys, const float* scores, long long n,

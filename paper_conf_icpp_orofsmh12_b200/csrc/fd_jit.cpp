@@ -32,9 +32,8 @@ namespace fdk {
 
 struct JitK2 {
     std::string key;                              // generated program (NVRTC source)
-    cudaKernel_t kern[2] = {nullptr, nullptr};    // [depth], compiled on first use
-    int grid[2] = {0, 0};
-    size_t smem = 0;
+    cudaKernel_t kern[2][JIT_KINDS] = {};         // [depth][kind], compiled on first use
+    int grid[2][JIT_KINDS] = {};
 };
 
 namespace {
@@ -159,15 +158,61 @@ int jit_deep_end(const StageDev* st, int n_stages) {
     return k;
 }
 
+// resident CTAs per SM targeted by the fused kernel's launch bounds (FD_K2_CTAS, 2..6)
+int jit_ctas() {
+    int c = FD_K2_CTAS;
+    if (const char* e = std::getenv("FD_K2_CTAS")) c = std::atoi(e);
+    return c < 2 ? 2 : (c > 6 ? 6 : c);
+}
+
+// tiles per k_deep batch of the specialised kernel (FD_K2B_NB, 1..8; default FD_K2B_NB of the build)
+int jit_nb_deep() {
+    int nb = FD_K2B_NB;
+    if (const char* e = std::getenv("FD_K2B_NB")) nb = std::atoi(e);
+    return nb < 1 ? 1 : (nb > 8 ? 8 : nb);
+}
+
+size_t jit_smem_deep(int nb) {
+    switch (nb) {
+        case 1: return TileGeoB<JIT_STEP, 1>::SMEM;
+        case 2: return TileGeoB<JIT_STEP, 2>::SMEM;
+        case 3: return TileGeoB<JIT_STEP, 3>::SMEM;
+        case 4: return TileGeoB<JIT_STEP, 4>::SMEM;
+        case 5: return TileGeoB<JIT_STEP, 5>::SMEM;
+        case 6: return TileGeoB<JIT_STEP, 6>::SMEM;
+        case 7: return TileGeoB<JIT_STEP, 7>::SMEM;
+        default: return TileGeoB<JIT_STEP, 8>::SMEM;
+    }
+}
+
 std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages) {
     const int k_end = jit_deep_end(st, n_stages);
-    std::string src = "#include \"fd_internal.h\"\n" + jit_stage1_source(rec_words, st[0].first, st[0].n) +
+    std::string src = std::string(std::getenv("FD_POOL_SEPARATE") ? "#define FD_POOL_SEPARATE 1\n" : "") +
+                      "#define FD_K2D_CTAS " + std::to_string(std::getenv("FD_K2D_CTAS") ? std::atoi(std::getenv("FD_K2D_CTAS")) : FD_K2D_CTAS) +
+                      "\n#define FD_K2_CTAS " + std::to_string(jit_ctas()) + "\n#define FD_K2B_NB " +
+                      std::to_string(jit_nb_deep()) + "\n#include \"fd_internal.h\"\n" + jit_stage1_source(rec_words, st[0].first, st[0].n) +
                       "#define FD_JIT_STAGE1 1\n";
     if (k_end > 1) src += jit_deep_source(rec_words, st, k_end) + "#define FD_JIT_DEEP " + std::to_string(k_end) + "\n";
     return src + "#include \"k_cascade.cu\"\n";
 }
 
-bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cubin, std::string* lowered,
+static std::string jit_name(int kind, bool depth) {
+    const std::string d = depth ? "true" : "false";
+    if (kind == JIT_FUSED) return "fdk::k_cascade<1, " + d + ">";
+    if (kind == JIT_STAGE1) return "fdk::k_stage1<1, " + d + ">";
+    if (kind == JIT_DEEP1) return "fdk::k_deep1<1, " + d + ">";
+    return "fdk::k_deep<1, " + d + ", " + std::to_string(jit_nb_deep()) + ">";
+}
+
+static size_t jit_kind_smem(int kind) {
+    if (kind == JIT_FUSED)
+        return TileGeo<JIT_STEP>::SMEM + (std::getenv("FD_POOL_SEPARATE") ? (size_t)TileGeo<JIT_STEP>::NW * 10 : 0);
+    if (kind == JIT_STAGE1) return TileGeoA<JIT_STEP>::SMEM;
+    if (kind == JIT_DEEP1) return TileGeoD<JIT_STEP>::SMEM;
+    return jit_smem_deep(jit_nb_deep());
+}
+
+bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cubin, std::vector<std::string>* lowered,
                     std::string* err) {
     const char* hdr_src[] = {jit_src_fd_h, jit_src_fd_internal_h, jit_src_k_common_cuh, jit_src_k_cascade_cu};
     const char* hdr_names[] = {"fd.h", "fd_internal.h", "k_common.cuh", "k_cascade.cu"};
@@ -176,8 +221,11 @@ bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cu
         *err = "nvrtcCreateProgram failed";
         return false;
     }
-    const char* name = depth ? "fdk::k_cascade<1, true, 1>" : "fdk::k_cascade<1, false, 1>";
-    nvrtcAddNameExpression(prog, name);
+    std::string names[JIT_KINDS];
+    for (int k = 0; k < JIT_KINDS; ++k) {
+        names[k] = jit_name(k, depth);
+        nvrtcAddNameExpression(prog, names[k].c_str());
+    }
     const bool verbose = std::getenv("FD_JIT_VERBOSE") && std::getenv("FD_JIT_VERBOSE")[0] == '1';
     const char* opts[] = {"-arch=sm_100a", "-std=c++17", "--fmad=false", "-lineinfo", "-default-device",
                           "--ptxas-options=-v"};
@@ -196,9 +244,12 @@ bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cu
     nvrtcGetCUBINSize(prog, &cb);
     cubin->resize(cb);
     nvrtcGetCUBIN(prog, cubin->data());
-    const char* lw = nullptr;
-    nvrtcGetLoweredName(prog, name, &lw);
-    *lowered = lw ? lw : "";
+    lowered->assign(JIT_KINDS, std::string());
+    for (int k = 0; k < JIT_KINDS; ++k) {
+        const char* lw = nullptr;
+        nvrtcGetLoweredName(prog, names[k].c_str(), &lw);
+        (*lowered)[k] = lw ? lw : "";
+    }
     nvrtcDestroyProgram(&prog);
     return true;
 }
@@ -211,56 +262,59 @@ JitK2* jit_k2_build(const uint32_t* rec_words, const StageDev* st, int n_stages,
 }
 
 namespace {
-// process-wide cache: generated stage source + depth -> loaded kernel (cascades loaded again
-// with the same first stage reuse the compiled code)
+// process-wide cache: generated program + depth -> loaded kernels (cascades loaded again with
+// the same stages reuse the compiled code)
 struct Loaded {
     cudaLibrary_t lib = nullptr;
-    cudaKernel_t kern = nullptr;
-    int grid = 0;
+    cudaKernel_t kern[JIT_KINDS] = {};
+    int grid[JIT_KINDS] = {};
 };
 std::mutex g_jit_mu;
 std::map<std::pair<std::string, int>, Loaded> g_jit_cache;
 }  // namespace
 
-cudaError_t jit_k2_launch(JitK2* J, const CascadeParams& p, bool depth, cudaStream_t st, std::string* err) {
+cudaError_t jit_k2_launch(JitK2* J, const CascadeParams& p, bool depth, int kind, cudaStream_t st, std::string* err) {
     const int d = depth ? 1 : 0;
-    if (!J->kern[d]) {
+    if (!J->kern[d][0]) {
         std::lock_guard<std::mutex> lk(g_jit_mu);
         Loaded& L = g_jit_cache[{J->key, d}];
-        if (!L.kern) {
+        if (!L.kern[0]) {
             std::vector<char> cubin;
-            std::string lowered;
+            std::vector<std::string> lowered;
             if (!jit_k2_compile(J->key, depth, &cubin, &lowered, err)) {
                 g_jit_cache.erase({J->key, d});
                 return cudaErrorInvalidSource;
             }
             cudaError_t e = cudaLibraryLoadData(&L.lib, cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0);
-            int dev = 0, sms = 0, per = 0;
-            const size_t smem = cascade_smem(JIT_STEP);
-            if (e == cudaSuccess) e = cudaLibraryGetKernel(&L.kern, L.lib, lowered.c_str());
+            int dev = 0, sms = 0;
             if (e == cudaSuccess) e = cudaGetDevice(&dev);
             if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-            if (e == cudaSuccess)
-                e = cudaKernelSetAttributeForDevice(L.kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem, dev);
-            if (e == cudaSuccess)
-                e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, reinterpret_cast<const void*>(L.kern), k2_threads(JIT_STEP),
-                                                                  smem);
+            for (int k = 0; k < JIT_KINDS && e == cudaSuccess; ++k) {
+                int per = 0;
+                const size_t smem = jit_kind_smem(k);
+                e = cudaLibraryGetKernel(&L.kern[k], L.lib, lowered[k].c_str());
+                if (e == cudaSuccess)
+                    e = cudaKernelSetAttributeForDevice(L.kern[k], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem, dev);
+                if (e == cudaSuccess)
+                    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, reinterpret_cast<const void*>(L.kern[k]),
+                                                                      k == JIT_DEEP1 ? K2D_THREADS : k2_threads(JIT_STEP), smem);
+                L.grid[k] = sms * (per > 0 ? per : 1);
+            }
             if (e != cudaSuccess) {
                 *err = std::string("JIT kernel load: ") + cudaGetErrorString(e);
                 g_jit_cache.erase({J->key, d});
                 return e;
             }
-            const char* cap = std::getenv("FD_K2_CTAS");      // diagnostic: resident CTAs per SM cap
-            if (cap && std::atoi(cap) > 0 && std::atoi(cap) < per) per = std::atoi(cap);
-            L.grid = sms * (per > 0 ? per : 1);
         }
-        J->kern[d] = L.kern;
-        J->grid[d] = L.grid;
-        J->smem = cascade_smem(JIT_STEP);
+        for (int k = 0; k < JIT_KINDS; ++k) {
+            J->kern[d][k] = L.kern[k];
+            J->grid[d][k] = L.grid[k];
+        }
     }
-    const int grid = J->grid[d] < p.total_tiles ? J->grid[d] : p.total_tiles;
+    const int grid = J->grid[d][kind] < p.total_tiles ? J->grid[d][kind] : p.total_tiles;
     void* args[] = {const_cast<CascadeParams*>(&p)};
-    return cudaLaunchKernel(reinterpret_cast<const void*>(J->kern[d]), dim3(grid), dim3(k2_threads(JIT_STEP)), args, J->smem, st);
+    return cudaLaunchKernel(reinterpret_cast<const void*>(J->kern[d][kind]), dim3(grid),
+                            dim3(kind == JIT_DEEP1 ? K2D_THREADS : k2_threads(JIT_STEP)), args, jit_kind_smem(kind), st);
 }
 
 void jit_k2_free(JitK2* J) { delete J; }    // loaded code stays in the process-wide cache

@@ -8,6 +8,8 @@
 namespace fdk {
 
 struct JitK2;
+// kernels of the specialised program: fused k_cascade, split k_stage1 + k_deep
+enum { JIT_FUSED = 0, JIT_STAGE1 = 1, JIT_DEEP = 2, JIT_DEEP1 = 3, JIT_KINDS = 4 };
 // CUDA source of the generated first stage (stage index `first`..first+n of the packed step-1
 // records, REC_WORDS u32 per stump)
 std::string jit_stage1_source(const uint32_t* rec_words, int first, int n);
@@ -15,13 +17,13 @@ std::string jit_stage1_source(const uint32_t* rec_words, int first, int n);
 std::string jit_deep_source(const uint32_t* rec_words, const StageDev* st, int k_end);
 // the whole NVRTC program for a cascade (generated stages + k_cascade.cu)
 std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages);
-// NVRTC compile only (no device needed): cubin + lowered name of k_cascade<1, depth, 1>
-bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cubin, std::string* lowered,
+// NVRTC compile only (no device needed): cubin + lowered names of the JIT_KINDS kernels
+bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cubin, std::vector<std::string>* lowered,
                     std::string* err);
 // specialisation handle for one cascade (code generated now, compiled and loaded on first launch)
 JitK2* jit_k2_build(const uint32_t* rec_words, const StageDev* st, int n_stages, std::string* err);
 // launch (compiling on first use; cudaErrorInvalidSource + *err when NVRTC fails)
-cudaError_t jit_k2_launch(JitK2* j, const CascadeParams& p, bool depth, cudaStream_t st, std::string* err);
+cudaError_t jit_k2_launch(JitK2* j, const CascadeParams& p, bool depth, int kind, cudaStream_t st, std::string* err);
 void jit_k2_free(JitK2* j);
 
 }  // namespace fdk

@@ -44,112 +44,364 @@ extern "C" int fd_debug_k2_timing(unsigned long long* out, int reset) {
 #define FD_JIT_DEEP 0        // run-time specialised kernel: deep stages [1, FD_JIT_DEEP) are generated code
 #endif
 
-constexpr int LC = 8;                        // leaves parked per lane before the ordered sum (group mode)
-
-template <int STEP>
-struct TileGeo {
+// Output of a window of ii slot sl (batch tile table in shared memory).
+template <int STEP, bool DEPTH>
+struct WinOut {
+    const CascadeParams& p;
+    const int *frame, *lvl, *wx0, *wy0;
     static constexpr int TX = k2_tx(STEP);
-    static constexpr int TY = k2_ty(STEP);
-    static constexpr int WPT = k2_wpt(STEP);
-    static constexpr int WARPS_X = TX / 32;
-    static constexpr int TW = tile_w(STEP);
-    static constexpr int TH = tile_h(STEP);
-    static constexpr int PLANE = TW * TH;          // u32 per plane
-    static constexpr int BOX = 2 * PLANE;          // ii + sqii (one TMA box)
-    static constexpr int BUF = (BOX + 255) & ~255; // buffer stride: keeps every TMA destination 1 KB aligned
-    static constexpr int NW = TX * TY;             // windows per tile
-    static constexpr int THREADS = k2_threads(STEP);
-    static constexpr size_t LEAVES = (size_t)THREADS * LC;   // floats
-    static constexpr size_t smem(int nst) {
-        return (size_t)nst * BUF * 4 + (size_t)NW * 4 * 2 + LEAVES * 4 + (size_t)NW * 2 * 2;
+    __device__ __forceinline__ long long index(int sl, int idx) const {
+        const int k = lvl[sl];
+        return (long long)frame[sl] * p.win_per_frame + __ldg(&p.lv[k].win0) +
+               (long long)(wy0[sl] + idx / TX) * __ldg(&p.lv[k].nx) + (wx0[sl] + idx % TX);
+    }
+    // a window that passed every stage (depth N): detection record or depth/score map entry
+    __device__ __forceinline__ void emit(int sl, int idx, float score) const {
+        if (p.stage_counts) atomicAdd(p.stage_counts + p.n_stages, 1ull);
+        if (DEPTH) {
+            const long long o = index(sl, idx);
+            p.depth[o] = (uint8_t)(p.n_stages < 255 ? p.n_stages : 255);
+            p.score[o] = score;
+        } else {
+            const unsigned long long at = atomicAdd(p.det_count, 1ull);
+            if ((long long)at < p.det_cap) {
+                p.det_keys[at] = det_key(frame[sl], lvl[sl], (wy0[sl] + idx / TX) * STEP, (wx0[sl] + idx % TX) * STEP);
+                p.det_scores[at] = score;
+            }
+        }
+    }
+    // depth mode: the window stopped at stage s (depth s) with stage sum `score`
+    __device__ __forceinline__ void reject(int sl, int idx, int s, float score) const {
+        if (DEPTH) {
+            const long long o = index(sl, idx);
+            p.depth[o] = (uint8_t)(s < 255 ? s : 255);
+            p.score[o] = score;
+        }
     }
 };
 
-// NST = TMA stages: 2 = double-buffered tiles (prefetch the next tile during evaluation),
-// 1 = single buffer with one more resident CTA per SM.
-template <int STEP, bool DEPTH, int NST>
-__global__ void __launch_bounds__(k2_threads(STEP), k2_threads(STEP) == 128 ? 5 : (NST == 1 ? 3 : 2)) k_cascade(const __grid_constant__ CascadeParams p) {
-    using G = TileGeo<STEP>;
-    constexpr int TW = G::TW, TX = G::TX, TY = G::TY, WPT = G::WPT;
-    extern __shared__ __align__(1024) uint8_t smem_raw[];
-    uint32_t* tiles = reinterpret_cast<uint32_t*>(smem_raw);               // [NST][2][TH][TW]
-    float* nfs = reinterpret_cast<float*>(tiles + NST * G::BUF);            // [NW] per-window nf
-    float* sums = nfs + G::NW;                                              // [NW] last stage sum
-    float* leaves = sums + G::NW;                                           // [8 warps][LC][32]
-    uint16_t* lists = reinterpret_cast<uint16_t*>(leaves + G::LEAVES);      // [2][NW]
-    __shared__ __align__(8) uint64_t mbar[2];
-    __shared__ int s_tile[2], s_lvl[2], s_tl[2];
-    __shared__ int s_cnt[3];
-
+// Deep stages (1 .. N-1) over a pool of stage-1 survivors held in shared memory: entry e has
+// ploc[e] = slot << 11 | window index (within the slot's tile) and nf pnf[e]; s_cnt[1] = pool size
+// (s_cnt[0] = s_cnt[2] = 0) on entry.  Stage-synchronous: each stage's survivors are
+// ballot-compacted into the other list and the block synchronises once per stage.  Lane per
+// window (uniform stump records) while windows are plentiful, GL lanes per window (tree sum +
+// certified decision) when fewer than lane_min remain, and once at most tail_n are left they go
+// to the global tail queue (k_tail.cu) -- or, when it is full or absent, are finished here one
+// warp per window.  Ends with a block barrier.
+template <int STEP, bool DEPTH, int CP, int THREADS = k2_threads(STEP)>
+__device__ __forceinline__ void deep_phase(const CascadeParams& p, const uint32_t* __restrict__ slots, const float* pnf,
+                                           const uint16_t* ploc, uint16_t* lists, int* s_cnt, int& s_tpos,
+                                           const WinOut<STEP, DEPTH>& out) {
+    constexpr int TX = k2_tx(STEP), TW = tile_w(STEP), PBUF = k2_pbuf(STEP);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int lane_min = min(p.lane_min, THREADS / 2 + 1);
     const int N = p.n_stages;
+    const ParamRec prec{p};
+    const GlobalRec grec{p.stumps};
+    const int tail_n = p.tail_q ? p.tail_n : THREADS / 32;
+    const int* s_frame = out.frame;
+    const int* s_lvl = out.lvl;
+    const int* s_wx0 = out.wx0;
+    const int* s_wy0 = out.wy0;
+    auto emit = [&](int sl, int idx, float score) { out.emit(sl, idx, score); };
+    auto reject = [&](int sl, int idx, int s, float score) { out.reject(sl, idx, s, score); };
+#ifdef FD_K2_TIMING
+    const long long tm2 = clock64();
+#endif
+    int s = 1;
+    // one deep stage; sd is a parameter-bank (uniform) or global stage descriptor.  Stage 1's
+    // input is the pool itself (entry e), later stages read pool indices from lists.
+    auto deep_stage = [&](const StageDev& sd, int n) {
+        const uint16_t* lin = lists + (s & 1) * CP;
+        uint16_t* lout = lists + ((s + 1) & 1) * CP;
+        const bool last = s == N - 1;
+        // stages [1, FD_JIT_DEEP) of the run-time specialised kernel: immediate-offset code,
+        // always one lane per window
+        const bool jit_s = FD_JIT_DEEP > 0 && s < FD_JIT_DEEP;
+        if (!jit_s && n < lane_min) {
+            // fewer windows than half the block: GL = 2^lg lanes per window (the largest
+            // power of two with n*GL <= THREADS, so one pass covers every window and
+            // all warps work); the group's lanes evaluate different stumps, the leader adds
+            // the leaves in stump order (the exact fp32 sequence of the definition).
+            int lg = 1;
+            while (lg < 5 && (n << (lg + 1)) <= THREADS) ++lg;
+            const int e = tid >> lg;
+            const bool act = e < n;
+            const int pe = act ? (s == 1 ? e : lin[e]) : 0;
+            const int loc = act ? ploc[pe] : 0;
+            const int sl = loc >> 11, idx = loc & 2047;
+            const int b = sl * PBUF + (idx / TX) * STEP * TW + (idx % TX) * STEP;
+            const float nfw = act ? pnf[pe] : 1.0f;
+            // tree sum + certified decision; the sequential sum only where the decision is a
+            // near tie or the score is an output (accepted window, depth-mode rejection)
+            float acc, aacc;
+            group_stage_tree_mc(slots, b, nfw, grec, sd.first, sd.n, sd.mc, lg, act, lane, acc, aacc);
+            int dec = certify(acc, aacc, sd.n, (sd.n + (1 << lg) - 1) / (1 << lg) - 1 + lg, sd.T);
+            float sum = acc;
+            const bool need = act && (dec < 0 || (dec == 1 && last) || (DEPTH && dec == 0));
+#ifdef FD_K2_TIMING
+            if (act && (lane & ((1 << lg) - 1)) == 0) {
+                atomicAdd(&g_k2_timing[95], 1ull);
+                if (dec < 0) atomicAdd(&g_k2_timing[94], 1ull);
+                if (need) atomicAdd(&g_k2_timing[96], 1ull);
+            }
+#endif
+            if (need && (lane & ((1 << lg) - 1)) == 0) {
+                // rare: the group leader adds the leaves itself, in stump order
+                // (records from global memory: a divergent constant-bank read serialises)
+                sum = eval_stage(slots, b, nfw, grec, sd.first, sd.n, sd.mc);
+                dec = sum >= sd.T ? 1 : 0;
+            }
+            if (act && (lane & ((1 << lg) - 1)) == 0) {
+                if (dec == 1) {
+                    if (last)
+                        emit(sl, idx, sum);
+                    else
+                        lout[atomicAdd(&s_cnt[(s + 1) % 3], 1)] = (uint16_t)pe;
+                } else {
+                    reject(sl, idx, s, sum);
+                }
+            }
+            return;
+        }
+        const bool in_param = sd.first + sd.n <= p.n_pstumps;
+        for (int e0 = warp * 32; e0 < n; e0 += THREADS) {
+            const int e = e0 + lane;
+            const bool act = e < n;
+            int pe = 0, sl = 0, idx = 0;
+            float sum = 0.0f;
+            if (act) {
+                pe = s == 1 ? e : lin[e];
+                const int loc = ploc[pe];
+                sl = loc >> 11;
+                idx = loc & 2047;
+                const int b = sl * PBUF + (idx / TX) * STEP * TW + (idx % TX) * STEP;
+                const float nfw = pnf[pe];
+#if FD_JIT_DEEP > 0
+                if (jit_s)
+                    sum = jit_deep(s, slots + b, nfw);
+                else
+#endif
+                    sum = in_param ? eval_stage(slots, b, nfw, prec, sd.first, sd.n, sd.mc)
+                                   : eval_stage(slots, b, nfw, grec, sd.first, sd.n, sd.mc);
+            }
+            const bool pass = act && (sum >= sd.T);
+            if (act && !pass) reject(sl, idx, s, sum);
+            if (last) {
+                if (pass) emit(sl, idx, sum);
+                continue;
+            }
+            const unsigned m = __ballot_sync(0xffffffffu, pass);
+            if (m) {
+                int pos = 0;
+                if (lane == 0) pos = atomicAdd(&s_cnt[(s + 1) % 3], __popc(m));
+                pos = __shfl_sync(0xffffffffu, pos, 0);
+                if (pass) lout[pos + __popc(m & ((1u << lane) - 1u))] = (uint16_t)pe;
+            }
+        }
+    };
+    for (; s < N; ++s) {
+#ifdef FD_K2_TIMING
+        const long long ts0 = clock64();
+#endif
+        const int n = s_cnt[s % 3];
+        if (tid == 0 && p.stage_counts && n) atomicAdd(p.stage_counts + s, (unsigned long long)n);
+        if (n == 0) break;
+        if (n <= tail_n && !(FD_JIT_DEEP > 0 && s < FD_JIT_DEEP)) {
+            // tail: few windows left.  They go to the global tail queue (finished by
+            // k_tail, one warp per window) so this CTA moves on to its next tiles instead of
+            // waiting for its deepest window; whatever does not fit in the queue is finished
+            // here, one warp per window.
+            const uint16_t* lin = lists + (s & 1) * CP;
+            if (tid == 0) s_tpos = p.tail_q ? (int)atomicAdd(p.tail_count, (unsigned)n) : p.tail_cap;
+            __syncthreads();
+            const int tpos = s_tpos;
+            for (int e = tid; e < n && tpos + e < p.tail_cap; e += THREADS) {
+                const int pe = s == 1 ? e : lin[e];
+                const int loc = ploc[pe];
+                const int sl = loc >> 11, idx = loc & 2047;
+                uint4 q;
+                q.x = ((unsigned)(s_frame[sl] - p.frame_base) << 16) | ((unsigned)s_lvl[sl] << 8) | (unsigned)s;
+                q.y = ((unsigned)(s_wy0[sl] + idx / TX) << 16) | (unsigned)(s_wx0[sl] + idx % TX);
+                q.z = (unsigned)__float_as_int(pnf[pe]);
+                q.w = 0u;
+                p.tail_q[tpos + e] = q;
+            }
+            for (int e = warp; e < n; e += THREADS / 32) {
+                if (tpos + e < p.tail_cap) continue;
+                const int pe = s == 1 ? e : lin[e];
+                const int loc = ploc[pe];
+                const int sl = loc >> 11, idx = loc & 2047;
+                const int b = sl * PBUF + (idx / TX) * STEP * TW + (idx % TX) * STEP;
+                const float nfw = pnf[pe];
+                int s2 = s;
+                float sum = 0.0f;
+                for (; s2 < N; ++s2) {
+                    StageDev sd;
+                    if (s2 < p.n_pstages) {
+                        sd.first = p.pstages[s2].first;
+                        sd.n = p.pstages[s2].n;
+                        sd.T = p.pstages[s2].T;
+                        sd.mc = p.pstages[s2].mc;
+                    } else {
+                        sd = p.stages[s2];
+                    }
+                    if (s2 > s && lane == 0 && p.stage_counts) atomicAdd(p.stage_counts + s2, 1ull);
+                    sum = 0.0f;
+                    for (int c0 = 0; c0 < sd.n; c0 += 32) {
+                        const int j = c0 + lane;
+                        float leaf = 0.0f;
+                        if (j < sd.n) leaf = eval_stage(slots, b, nfw, grec, sd.first + j, 1, sd.mc);
+                        const int m = min(32, sd.n - c0);
+                        // ordered sum of the lanes' leaves: independent shuffles, serial adds
+#pragma unroll
+                        for (int t2 = 0; t2 < 32; ++t2) {
+                            const float v = __shfl_sync(0xffffffffu, leaf, t2);
+                            if (t2 < m) sum = __fadd_rn(sum, v);
+                        }
+                    }
+                    if (!(sum >= sd.T)) break;
+                }
+                if (lane == 0) {
+                    if (s2 < N)
+                        reject(sl, idx, s2, sum);
+                    else
+                        emit(sl, idx, sum);
+                }
+            }
+#ifdef FD_K2_TIMING
+            if (tid == 0) {
+                atomicAdd(&g_k2_timing[80], (unsigned long long)(clock64() - ts0));
+                atomicAdd(&g_k2_timing[81], (unsigned long long)n);
+            }
+#endif
+            break;
+        }
+        if (tid == 0) s_cnt[(s + 2) % 3] = 0;
+        {
+            StageDev sd;                  // one call site keeps deep_stage inlined
+            if (s < p.n_pstages) {
+                sd.first = p.pstages[s].first;
+                sd.n = p.pstages[s].n;
+                sd.T = p.pstages[s].T;
+                sd.mc = p.pstages[s].mc;
+            } else {
+                sd = p.stages[s];
+            }
+            deep_stage(sd, n);
+        }
+        __syncthreads();
+#ifdef FD_K2_TIMING
+        if (tid == 0) {
+            const unsigned long long dt = (unsigned long long)(clock64() - ts0);
+            const int si = s < 32 ? s : 31;
+            atomicAdd(&g_k2_timing[16 + si], dt);
+            atomicAdd(&g_k2_timing[48 + si], 1ull);
+            atomicAdd(&g_k2_timing[n < lane_min ? 82 : 83], dt);
+        }
+#endif
+    }
+#ifdef FD_K2_TIMING
+    if (tid == 0) {
+        atomicAdd(&g_k2_timing[3], (unsigned long long)(clock64() - tm2));
+        atomicAdd(&g_k2_timing[4 + (s < 11 ? s : 11)], 1ull);
+        atomicAdd(&g_k2_timing[84], 1ull);
+    }
+#endif
+    __syncthreads();
+}
+
+// Tile number tn of a frame group -> frame (global), level, window origin, TMA coordinates.
+struct TileAt {
+    int g, k, wx0, wy0, x, y;
+};
+template <int STEP>
+__device__ __forceinline__ TileAt tile_at(const CascadeParams& p, int tn) {
+    TileAt t;
+    t.g = tn / p.tiles_per_frame;
+    const int r = tn % p.tiles_per_frame;
+    int k = 0;
+    while (k + 1 < p.n_levels && __ldg(&p.lv[k + 1].tile0) <= r) ++k;
+    const int tl = r - __ldg(&p.lv[k].tile0);
+    const int tx = __ldg(&p.lv[k].tiles_x);
+    t.k = k;
+    t.wx0 = (tl % tx) * k2_tx(STEP);
+    t.wy0 = (tl / tx) * k2_ty(STEP);
+    t.x = t.wx0 * STEP;
+    t.y = t.wy0 * STEP;
+    return t;
+}
+
+// Fused K2: one CTA per tile at a time, persistent over every (frame, level, tile) of the
+// group.  One TMA brings the tile's ii and sqii planes; stage 1 runs densely (WPT windows per
+// thread down a column, nf from the variance, oracle c5); its survivors go into a pool that
+// reuses the sqii buffer (dead once every nf is taken), and deep_phase runs the deeper stages
+// over the pool.  40 KB of shared memory per CTA keeps FD_K2_CTAS CTAs resident per SM, so
+// the latency-bound deep phase of one tile overlaps the dense stage 1 of the others.
+template <int STEP, bool DEPTH>
+__global__ void __launch_bounds__(k2_threads(STEP), FD_K2_CTAS) k_cascade(const __grid_constant__ CascadeParams p) {
+    using G = TileGeo<STEP>;
+    constexpr int TW = tile_w(STEP), TX = k2_tx(STEP), TY = k2_ty(STEP), WPT = k2_wpt(STEP), CP = G::CP;
+    constexpr int WARPS_X = TX / 32, PLANE = tile_w(STEP) * tile_h(STEP);
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint32_t* T = reinterpret_cast<uint32_t*>(smem_raw);                      // ii plane
+    uint32_t* Q = reinterpret_cast<uint32_t*>(smem_raw + G::OFF_Q);           // sqii plane (mod 2^32)
+    float* pnf = reinterpret_cast<float*>(smem_raw + G::OFF_NF);              // pool, over Q after stage 1
+    uint16_t* ploc = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LOC);
+    uint16_t* lists = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LIST);
+    __shared__ __align__(8) uint64_t mbar;
+    __shared__ int s_tile;
+    __shared__ int s_frame[1], s_lvl[1], s_wx0[1], s_wy0[1];
+    __shared__ int s_cnt[3];
+    __shared__ int s_tpos;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const StageDev& st0 = p.pstages[0];     // parameter bank: warp-uniform (n_pstages >= 1)
     const ParamRec prec{p};
     const GlobalRec grec{p.stumps};
-
-    // thread 0: claim a tile from the work counter, decode it and start its TMA into buffer b
-    auto fetch = [&](int b) {
-        const int tn = (int)atomicAdd(p.tile_counter, 1u);
-        s_tile[b] = tn;
-        if (tn < p.total_tiles) {
-            const int g = tn / p.tiles_per_frame, r = tn % p.tiles_per_frame;
-            int k = 0;
-            while (k + 1 < p.n_levels && __ldg(&p.lv[k + 1].tile0) <= r) ++k;
-            const int tl = r - __ldg(&p.lv[k].tile0);
-            const int tx = __ldg(&p.lv[k].tiles_x);
-            s_lvl[b] = k;
-            s_tl[b] = tl;
-            mbar_expect_tx(&mbar[b], G::BOX * 4);
-            tma_load_4d(tiles + b * G::BUF, p.tmaps + k, (tl % tx) * TX * STEP, (tl / tx) * TY * STEP, 0, g, &mbar[b]);
-        }
-    };
+    const WinOut<STEP, DEPTH> out{p, s_frame, s_lvl, s_wx0, s_wy0};
     if (tid == 0) {
-        mbar_init(&mbar[0], 1);
-        mbar_init(&mbar[1], 1);
+        mbar_init(&mbar, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        if (NST == 2) fetch(0);
     }
-    uint32_t phase0 = 0, phase1 = 0;
-
-    for (int it = 0;; ++it) {
-        const int buf = NST == 2 ? (it & 1) : 0;
-        __syncthreads();                      // previous tile fully consumed (buffers and counters free)
+    uint32_t phase = 0;
+    for (;;) {
+        __syncthreads();                          // buffers and s_* free
         if (tid == 0) {
             s_cnt[0] = 0;
             s_cnt[1] = 0;
             s_cnt[2] = 0;
-            fetch(NST == 2 ? (buf ^ 1) : 0);  // double buffer: prefetch the next tile; single: this one
+            const int tn = (int)atomicAdd(p.tile_counter, 1u);
+            s_tile = tn;
+            if (tn < p.total_tiles) {
+                const TileAt t = tile_at<STEP>(p, tn);
+                s_frame[0] = p.frame_base + t.g;
+                s_lvl[0] = t.k;
+                s_wx0[0] = t.wx0;
+                s_wy0[0] = t.wy0;
+                // generic-proxy accesses of the buffers are ordered before the async-proxy writes
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_expect_tx(&mbar, 2 * PLANE * 4);
+                tma_load_4d(T, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar);
+                tma_load_4d(Q, p.tmaps + t.k, t.x, t.y, 1, t.g, &mbar);
+            }
         }
         __syncthreads();
-        const int t = s_tile[buf];
-        if (t >= p.total_tiles) break;
-        const int g = t / p.tiles_per_frame;
-        const int k = s_lvl[buf];
-        const LevelDev L = p.lv[k];
-        const int tl = s_tl[buf];
-        const int wx0 = (tl % L.tiles_x) * TX, wy0 = (tl / L.tiles_x) * TY;
-        const int frame = p.frame_base + g;
+        if (s_tile >= p.total_tiles) break;
 #ifdef FD_K2_TIMING
         const long long tm0 = clock64();
 #endif
-        if (buf == 0) {
-            mbar_wait(&mbar[0], phase0);
-            phase0 ^= 1;
-        } else {
-            mbar_wait(&mbar[1], phase1);
-            phase1 ^= 1;
-        }
+        mbar_wait(&mbar, phase);
+        phase ^= 1;
 #ifdef FD_K2_TIMING
         const long long tm1 = clock64();
 #endif
-        const uint32_t* T = tiles + buf * G::BUF;      // ii plane
-        const uint32_t* Q = T + G::PLANE;              // sqii plane (mod 2^32)
-
-        // ---------------- stage 1, dense: WPT windows per thread down a column
-        const int lx = lane + 32 * (warp % G::WARPS_X);
-        const int ly0 = (warp / G::WARPS_X) * WPT;
+        const int k = s_lvl[0];
+        const int nx = __ldg(&p.lv[k].nx), ny = __ldg(&p.lv[k].ny);
+        const int wx0 = s_wx0[0], wy0 = s_wy0[0];
+        const int lx = lane + 32 * (warp % WARPS_X);
+        const int ly0 = (warp / WARPS_X) * WPT;
         const int base = ly0 * STEP * TW + lx * STEP;
-        const bool colok = wx0 + lx < L.nx;
+        const bool colok = wx0 + lx < nx;
         float nf[WPT], sm[WPT];
 #pragma unroll
         for (int i = 0; i < WPT; ++i) {
@@ -158,7 +410,6 @@ __global__ void __launch_bounds__(k2_threads(STEP), k2_threads(STEP) == 128 ? 5 
             const uint32_t q = Q[b + WIN * TW + WIN] - Q[b + WIN] - Q[b + WIN * TW] + Q[b];
             const long long v = 576LL * (long long)q - (long long)S * (long long)S;
             nf[i] = v > 0 ? __fsqrt_rn(__ll2float_rn(v)) : 1.0f;
-            nfs[(ly0 + i) * TX + lx] = nf[i];
             sm[i] = 0.0f;
         }
 #ifdef FD_JIT_STAGE1
@@ -171,18 +422,18 @@ __global__ void __launch_bounds__(k2_threads(STEP), k2_threads(STEP) == 128 ? 5 
         else
             dense_stage<WPT, STEP * TW>(T, base, nf, sm, grec, st0.first, st0.n);
 #endif
-
-        // compaction of stage-1 survivors into lists[1] (count s_cnt[1])
+        __syncthreads();                          // every sqii read done: the buffer becomes the pool
+        // stage-1 survivors into the pool (or out, for a one-stage cascade)
 #pragma unroll
         for (int i = 0; i < WPT; ++i) {
             const int wy = wy0 + ly0 + i;
-            const bool valid = colok && wy < L.ny;
+            const bool valid = colok && wy < ny;
             const bool pass = valid && (sm[i] >= st0.T);
             const int idx = (ly0 + i) * TX + lx;
-            if (DEPTH && valid && !pass) {
-                const long long o = (long long)frame * p.win_per_frame + L.win0 + (long long)wy * L.nx + (wx0 + lx);
-                p.depth[o] = 0;
-                p.score[o] = sm[i];
+            if (DEPTH && valid && !pass) out.reject(0, idx, 0, sm[i]);
+            if (p.n_stages == 1) {
+                if (pass) out.emit(0, idx, sm[i]);
+                continue;
             }
             const unsigned m = __ballot_sync(0xffffffffu, pass);
             if (m) {
@@ -191,288 +442,350 @@ __global__ void __launch_bounds__(k2_threads(STEP), k2_threads(STEP) == 128 ? 5 
                 pos = __shfl_sync(0xffffffffu, pos, 0);
                 if (pass) {
                     const int at = pos + __popc(m & ((1u << lane) - 1u));
-                    lists[G::NW + at] = (uint16_t)idx;
-                    sums[idx] = sm[i];
+                    ploc[at] = (uint16_t)idx;
+                    pnf[at] = nf[i];
                 }
             }
         }
-        if (tid == 0 && p.stage_counts) {
-            const unsigned long long nv =
-                (unsigned long long)min(TX, L.nx - wx0) * (unsigned long long)min(TY, L.ny - wy0);
-            atomicAdd(p.stage_counts, nv);
-        }
-        __syncthreads();
-
-#ifdef FD_K2_TIMING
-        const long long tm2 = clock64();
-#endif
-        // ---------------- deeper stages over the compacted queue
-        int s = 1;
-        // one deep stage; sd is a parameter-bank (uniform) or global stage descriptor
-        auto deep_stage = [&](const StageDev& sd, int n) {
-            const uint16_t* lin = lists + (s & 1) * G::NW;
-            uint16_t* lout = lists + ((s + 1) & 1) * G::NW;
-            // stages [1, FD_JIT_DEEP) of the run-time specialised kernel: immediate-offset code,
-            // always one lane per window
-            const bool jit_s = FD_JIT_DEEP > 0 && s < FD_JIT_DEEP;
-            if (!jit_s && n < p.lane_min) {
-                // fewer windows than half the block: GL = 2^lg lanes per window (the largest
-                // power of two with n*GL <= THREADS, so one pass covers every window and
-                // all warps work); the group's lanes evaluate different stumps, the leader adds
-                // the leaves in stump order (the exact fp32 sequence of the definition).
-                int lg = 1;
-                while (lg < 5 && (n << (lg + 1)) <= G::THREADS) ++lg;
-                const int e = tid >> lg;
-                const bool act = e < n;
-                const int idx = act ? lin[e] : 0;
-                const int wlx = idx % TX, wly = idx / TX;
-                const int b = wly * STEP * TW + wlx * STEP;
-                const float nfw = act ? nfs[idx] : 1.0f;
-                const float sum = group_stage<LC>(T, b, nfw, grec, sd.first, sd.n, sd.mc, lg, act,
-                                                  leaves + warp * 32 * LC, lane);
-                if (act && (lane & ((1 << lg) - 1)) == 0) {
-                    if (sum >= sd.T) {
-                        lout[atomicAdd(&s_cnt[(s + 1) % 3], 1)] = (uint16_t)idx;
-                        sums[idx] = sum;
-                    } else if (DEPTH) {
-                        const long long o = (long long)frame * p.win_per_frame + L.win0 +
-                                            (long long)(wy0 + wly) * L.nx + (wx0 + wlx);
-                        p.depth[o] = (uint8_t)(s < 255 ? s : 255);
-                        p.score[o] = sum;
-                    }
-                }
-                return;
-            }
-            const bool in_param = sd.first + sd.n <= p.n_pstumps;
-            for (int e0 = warp * 32; e0 < n; e0 += G::THREADS) {
-                const int e = e0 + lane;
-                const bool act = e < n;
-                int idx = 0;
-                float sum = 0.0f;
-                if (act) {
-                    idx = lin[e];
-                    const int wlx = idx % TX, wly = idx / TX;
-                    const int b = wly * STEP * TW + wlx * STEP;
-#if FD_JIT_DEEP > 0
-                    if (jit_s)
-                        sum = jit_deep(s, T + b, nfs[idx]);
-                    else
-#endif
-                        sum = in_param ? eval_stage(T, b, nfs[idx], prec, sd.first, sd.n, sd.mc)
-                                       : eval_stage(T, b, nfs[idx], grec, sd.first, sd.n, sd.mc);
-                }
-                const bool pass = act && (sum >= sd.T);
-                if (DEPTH && act && !pass) {
-                    const int wlx = idx % TX, wly = idx / TX;
-                    const long long o = (long long)frame * p.win_per_frame + L.win0 +
-                                        (long long)(wy0 + wly) * L.nx + (wx0 + wlx);
-                    p.depth[o] = (uint8_t)(s < 255 ? s : 255);
-                    p.score[o] = sum;
-                }
-                const unsigned m = __ballot_sync(0xffffffffu, pass);
-                if (m) {
-                    int pos = 0;
-                    if (lane == 0) pos = atomicAdd(&s_cnt[(s + 1) % 3], __popc(m));
-                    pos = __shfl_sync(0xffffffffu, pos, 0);
-                    if (pass) {
-                        lout[pos + __popc(m & ((1u << lane) - 1u))] = (uint16_t)idx;
-                        sums[idx] = sum;
-                    }
-                }
-            }
-        };
-        bool tail_done = false;
-        for (; s < N; ++s) {
-#ifdef FD_K2_TIMING
-            const long long ts0 = clock64();
-#endif
-            const int n = s_cnt[s % 3];
-            if (tid == 0 && p.stage_counts && n) atomicAdd(p.stage_counts + s, (unsigned long long)n);
-            if (n == 0) break;
-            if (n <= G::THREADS / 32 && !(FD_JIT_DEEP > 0 && s < FD_JIT_DEEP)) {
-                // tail: at most one window per warp left -- each warp walks its window through
-                // all remaining stages on its own (one stump per lane, leaves added in stump
-                // order via shuffles), so no block barrier is paid per stage.
-                if (warp < n) {
-                    const int idx = lists[(s & 1) * G::NW + warp];
-                    const int wlx = idx % TX, wly = idx / TX;
-                    const int b = wly * STEP * TW + wlx * STEP;
-                    const float nfw = nfs[idx];
-                    int s2 = s;
-                    float sum = 0.0f;
-                    for (; s2 < N; ++s2) {
-                        StageDev sd;
-                        if (s2 < p.n_pstages) {
-                            sd.first = p.pstages[s2].first;
-                            sd.n = p.pstages[s2].n;
-                            sd.T = p.pstages[s2].T;
-                            sd.mc = p.pstages[s2].mc;
-                        } else {
-                            sd = p.stages[s2];
-                        }
-                        if (s2 > s && lane == 0 && p.stage_counts) atomicAdd(p.stage_counts + s2, 1ull);
-                        sum = 0.0f;
-                        for (int c0 = 0; c0 < sd.n; c0 += 32) {
-                            const int j = c0 + lane;
-                            float leaf = 0.0f;
-                            if (j < sd.n) leaf = eval_stage(T, b, nfw, grec, sd.first + j, 1, sd.mc);
-                            const int m = min(32, sd.n - c0);
-                            // ordered sum of the lanes' leaves: independent shuffles, serial adds
-#pragma unroll
-                            for (int t2 = 0; t2 < 32; ++t2) {
-                                const float v = __shfl_sync(0xffffffffu, leaf, t2);
-                                if (t2 < m) sum = __fadd_rn(sum, v);
-                            }
-                        }
-                        if (!(sum >= sd.T)) break;
-                    }
-                    if (lane == 0) {
-                        const long long o = (long long)frame * p.win_per_frame + L.win0 +
-                                            (long long)(wy0 + wly) * L.nx + (wx0 + wlx);
-                        if (s2 < N) {
-                            if (DEPTH) {
-                                p.depth[o] = (uint8_t)(s2 < 255 ? s2 : 255);
-                                p.score[o] = sum;
-                            }
-                        } else {
-                            if (p.stage_counts) atomicAdd(p.stage_counts + N, 1ull);
-                            if (DEPTH) {
-                                p.depth[o] = (uint8_t)(N < 255 ? N : 255);
-                                p.score[o] = sum;
-                            } else {
-                                const unsigned long long at = atomicAdd(p.det_count, 1ull);
-                                if ((long long)at < p.det_cap) {
-                                    p.det_keys[at] = det_key(frame, k, (wy0 + wly) * STEP, (wx0 + wlx) * STEP);
-                                    p.det_scores[at] = sum;
-                                }
-                            }
-                        }
-                    }
-                }
-                tail_done = true;
-#ifdef FD_K2_TIMING
-                if (lane == 0 && warp < n) {
-                    atomicAdd(&g_k2_timing[80], (unsigned long long)(clock64() - ts0));
-                    atomicAdd(&g_k2_timing[81], 1ull);
-                }
-#endif
-                break;
-            }
-            if (tid == 0) s_cnt[(s + 2) % 3] = 0;
-            {
-                StageDev sd;                  // one call site keeps deep_stage inlined
-                if (s < p.n_pstages) {
-                    sd.first = p.pstages[s].first;
-                    sd.n = p.pstages[s].n;
-                    sd.T = p.pstages[s].T;
-                    sd.mc = p.pstages[s].mc;
-                } else {
-                    sd = p.stages[s];
-                }
-                deep_stage(sd, n);
-            }
-            __syncthreads();
-#ifdef FD_K2_TIMING
-            if (tid == 0) {
-                const unsigned long long dt = (unsigned long long)(clock64() - ts0);
-                const int si = s < 32 ? s : 31;
-                atomicAdd(&g_k2_timing[16 + si], dt);
-                atomicAdd(&g_k2_timing[48 + si], 1ull);
-                atomicAdd(&g_k2_timing[n < p.lane_min ? 82 : 83], dt);
-            }
-#endif
-        }
+        if (tid == 0 && p.stage_counts)
+            atomicAdd(p.stage_counts, (unsigned long long)min(TX, nx - wx0) * (unsigned long long)min(TY, ny - wy0));
 #ifdef FD_K2_TIMING
         if (tid == 0) {
-            const long long tm3 = clock64();
             atomicAdd(&g_k2_timing[0], 1ull);
             atomicAdd(&g_k2_timing[1], (unsigned long long)(tm1 - tm0));
-            atomicAdd(&g_k2_timing[2], (unsigned long long)(tm2 - tm1));
-            atomicAdd(&g_k2_timing[3], (unsigned long long)(tm3 - tm2));
-            atomicAdd(&g_k2_timing[4 + (s < 11 ? s : 11)], 1ull);
+            atomicAdd(&g_k2_timing[2], (unsigned long long)(clock64() - tm1));
         }
 #endif
-        if (s == N && !tail_done) {                 // accepted windows: depth N
-            const int nacc = s_cnt[N % 3];
-            if (tid == 0 && p.stage_counts && nacc) atomicAdd(p.stage_counts + N, (unsigned long long)nacc);
-            const uint16_t* lacc = lists + (N & 1) * G::NW;
-            for (int e0 = warp * 32; e0 < nacc; e0 += G::THREADS) {
-                const int e = e0 + lane;
-                const bool act = e < nacc;
-                int idx = act ? lacc[e] : 0;
-                const int wlx = idx % TX, wly = idx / TX;
-                if (DEPTH) {
-                    if (act) {
-                        const long long o = (long long)frame * p.win_per_frame + L.win0 +
-                                            (long long)(wy0 + wly) * L.nx + (wx0 + wlx);
-                        p.depth[o] = (uint8_t)(N < 255 ? N : 255);
-                        p.score[o] = sums[idx];
-                    }
+        __syncthreads();                          // pool complete
+        deep_phase<STEP, DEPTH, CP>(p, T, pnf, ploc, lists, s_cnt, s_tpos, out);
+    }
+}
+
+// ======================================================================== split K2, kernel a
+// k_stage1: the dense first stage alone, the throughput part of the cascade (c3: 10 of the
+// 11.8 stumps per window, 94.5% of windows stop here).  Persistent over every
+// (frame, level, tile) of the group; per tile one TMA of the ii and sqii planes, variance
+// normalisation (oracle c5), the stage evaluated densely (WPT windows per thread down a column,
+// run-time specialised code for step 1), and the survivors -- window index and nf -- appended
+// to a global list with one atomic per tile; tile_rec[tile] = (offset, count).
+template <int STEP, bool DEPTH>
+__global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_constant__ CascadeParams p) {
+    using G = TileGeoA<STEP>;
+    constexpr int TW = tile_w(STEP), TX = k2_tx(STEP), TY = k2_ty(STEP), WPT = k2_wpt(STEP);
+    constexpr int WARPS_X = TX / 32, PLANE = tile_w(STEP) * tile_h(STEP);
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint32_t* T = reinterpret_cast<uint32_t*>(smem_raw);                     // ii plane
+    uint32_t* Q = T + G::PBUF;                                               // sqii plane (mod 2^32)
+    uint2* sv = reinterpret_cast<uint2*>(smem_raw + G::OFF_SURV);            // [NW] survivors
+    __shared__ __align__(8) uint64_t mbar;
+    __shared__ int s_tile, s_cnt, s_off;
+    __shared__ int s_frame[1], s_lvl[1], s_wx0[1], s_wy0[1];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const StageDev& st0 = p.pstages[0];
+    const ParamRec prec{p};
+    const GlobalRec grec{p.stumps};
+    const WinOut<STEP, DEPTH> out{p, s_frame, s_lvl, s_wx0, s_wy0};
+    if (tid == 0) {
+        mbar_init(&mbar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    uint32_t phase = 0;
+    for (;;) {
+        __syncthreads();                          // buffers, survivor list and s_* free
+        if (tid == 0) {
+            s_cnt = 0;
+            const int tn = (int)atomicAdd(p.tile_counter, 1u);
+            s_tile = tn;
+            if (tn < p.total_tiles) {
+                const TileAt t = tile_at<STEP>(p, tn);
+                s_frame[0] = p.frame_base + t.g;
+                s_lvl[0] = t.k;
+                s_wx0[0] = t.wx0;
+                s_wy0[0] = t.wy0;
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_expect_tx(&mbar, 2 * PLANE * 4);
+                tma_load_4d(T, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar);
+                tma_load_4d(Q, p.tmaps + t.k, t.x, t.y, 1, t.g, &mbar);
+            }
+        }
+        __syncthreads();
+        const int tn = s_tile;
+        if (tn >= p.total_tiles) break;
+        mbar_wait(&mbar, phase);
+        phase ^= 1;
+        const int k = s_lvl[0];
+        const int nx = __ldg(&p.lv[k].nx), ny = __ldg(&p.lv[k].ny);
+        const int wx0 = s_wx0[0], wy0 = s_wy0[0];
+        const int lx = lane + 32 * (warp % WARPS_X);
+        const int ly0 = (warp / WARPS_X) * WPT;
+        const int base = ly0 * STEP * TW + lx * STEP;
+        const bool colok = wx0 + lx < nx;
+        float nf[WPT], sm[WPT];
+#pragma unroll
+        for (int i = 0; i < WPT; ++i) {
+            const int b = base + i * STEP * TW;
+            const uint32_t S = T[b + WIN * TW + WIN] - T[b + WIN] - T[b + WIN * TW] + T[b];
+            const uint32_t q = Q[b + WIN * TW + WIN] - Q[b + WIN] - Q[b + WIN * TW] + Q[b];
+            const long long v = 576LL * (long long)q - (long long)S * (long long)S;
+            nf[i] = v > 0 ? __fsqrt_rn(__ll2float_rn(v)) : 1.0f;
+            sm[i] = 0.0f;
+        }
+#ifdef FD_JIT_STAGE1
+        jit_stage1(T + base, nf, sm);
+#else
+        if (st0.first + st0.n <= p.n_pstumps)
+            dense_stage<WPT, STEP * TW>(T, base, nf, sm, prec, st0.first, st0.n);
+        else
+            dense_stage<WPT, STEP * TW>(T, base, nf, sm, grec, st0.first, st0.n);
+#endif
+#pragma unroll
+        for (int i = 0; i < WPT; ++i) {
+            const int wy = wy0 + ly0 + i;
+            const bool valid = colok && wy < ny;
+            const bool pass = valid && (sm[i] >= st0.T);
+            const int idx = (ly0 + i) * TX + lx;
+            if (DEPTH && valid && !pass) out.reject(0, idx, 0, sm[i]);
+            if (p.n_stages == 1) {
+                if (pass) out.emit(0, idx, sm[i]);
+                continue;
+            }
+            const unsigned m = __ballot_sync(0xffffffffu, pass);
+            if (m) {
+                int pos = 0;
+                if (lane == 0) pos = atomicAdd(&s_cnt, __popc(m));
+                pos = __shfl_sync(0xffffffffu, pos, 0);
+                if (pass) sv[pos + __popc(m & ((1u << lane) - 1u))] = make_uint2((unsigned)idx, (unsigned)__float_as_int(nf[i]));
+            }
+        }
+        __syncthreads();
+        if (tid == 0) {
+            const int c = s_cnt;
+            const unsigned off = c ? atomicAdd(p.surv_count, (unsigned)c) : 0u;
+            p.tile_rec[tn] = make_uint2(off, (unsigned)c);
+            s_off = (int)off;
+            if (p.stage_counts)
+                atomicAdd(p.stage_counts, (unsigned long long)min(TX, nx - wx0) * (unsigned long long)min(TY, ny - wy0));
+        }
+        __syncthreads();
+        const int c = s_cnt, off = s_off;
+        for (int e = tid; e < c; e += k2_threads(STEP)) p.surv[off + e] = sv[e];
+    }
+}
+
+// ======================================================================== split K2, kernel b
+// k_deep: the deeper stages.  A CTA claims tiles in order, skips those without survivors, TMAs
+// each claimed tile's ii plane into one of NB slots and copies its survivors into the pool, then
+// runs deep_phase over the whole batch -- NB tiles' worth of windows per stage-synchronous step
+// (c3: ~110 windows enter stage 2 per tile) instead of one tile's.
+template <int STEP, bool DEPTH, int NB>
+__global__ void __launch_bounds__(k2_threads(STEP), k2b_min_ctas(NB)) k_deep(const __grid_constant__ CascadeParams p) {
+    using G = TileGeoB<STEP, NB>;
+    constexpr int CP = G::CP, PBUF = G::PBUF, PLANE = tile_w(STEP) * tile_h(STEP), THREADS = k2_threads(STEP);
+    static_assert(G::NW <= 2048 && NB <= 8, "pool entries pack slot:3 | window:11");
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint32_t* slots = reinterpret_cast<uint32_t*>(smem_raw);
+    float* pnf = reinterpret_cast<float*>(smem_raw + G::OFF_NF);
+    uint16_t* ploc = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LOC);
+    uint16_t* lists = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LIST);
+    __shared__ __align__(8) uint64_t mbar[NB];
+    __shared__ int s_frame[NB], s_lvl[NB], s_wx0[NB], s_wy0[NB];
+    __shared__ int s_cnt[3];
+    __shared__ int s_tpos, s_tile, s_carry, s_stop, s_off, s_n, s_base;
+    const int tid = threadIdx.x;
+    const WinOut<STEP, DEPTH> out{p, s_frame, s_lvl, s_wx0, s_wy0};
+    if (tid == 0) {
+        for (int i = 0; i < NB; ++i) mbar_init(&mbar[i], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        s_carry = -1;
+    }
+    uint32_t phases = 0;
+    for (;;) {
+        int nb = 0;
+#ifdef FD_K2_TIMING
+        const long long tf0 = clock64();
+#endif
+        for (;;) {
+            __syncthreads();
+            if (tid == 0) {
+                if (nb == 0) {
+                    s_cnt[0] = 0;
+                    s_cnt[1] = 0;
+                    s_cnt[2] = 0;
+                }
+                int tn;
+                uint2 tr = make_uint2(0u, 0u);
+                if (s_carry >= 0) {
+                    tn = s_carry;
+                    s_carry = -1;
+                    tr = p.tile_rec[tn];
                 } else {
-                    const unsigned m = __ballot_sync(0xffffffffu, act);
-                    unsigned long long pos = 0;
-                    if (lane == 0) pos = atomicAdd(p.det_count, (unsigned long long)__popc(m));
-                    pos = __shfl_sync(0xffffffffu, pos, 0);
-                    if (act) {
-                        const unsigned long long at = pos + __popc(m & ((1u << lane) - 1u));
-                        if ((long long)at < p.det_cap) {
-                            p.det_keys[at] = det_key(frame, k, (wy0 + wly) * STEP, (wx0 + wlx) * STEP);
-                            p.det_scores[at] = sums[idx];
-                        }
+                    do {
+                        tn = (int)atomicAdd(p.deep_counter, 1u);
+                        if (tn >= p.total_tiles) break;
+                        tr = p.tile_rec[tn];
+                    } while (tr.y == 0u);
+                }
+                s_tile = tn;
+                s_stop = 0;
+                if (tn < p.total_tiles) {
+                    if (s_cnt[1] + (int)tr.y > CP) {
+                        s_carry = tn;             // does not fit: first tile of the next batch
+                        s_stop = 1;
+                    } else {
+                        const TileAt t = tile_at<STEP>(p, tn);
+                        s_frame[nb] = p.frame_base + t.g;
+                        s_lvl[nb] = t.k;
+                        s_wx0[nb] = t.wx0;
+                        s_wy0[nb] = t.wy0;
+                        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                        mbar_expect_tx(&mbar[nb], PLANE * 4);
+                        tma_load_4d(slots + nb * PBUF, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar[nb]);
+                        s_off = (int)tr.x;
+                        s_n = (int)tr.y;
+                        s_base = s_cnt[1];
+                        s_cnt[1] += (int)tr.y;
                     }
                 }
             }
+            __syncthreads();
+            if (s_tile >= p.total_tiles || s_stop) break;
+            {
+                const int off = s_off, n = s_n, b0 = s_base;
+                for (int e = tid; e < n; e += THREADS) {
+                    const uint2 v = p.surv[off + e];
+                    ploc[b0 + e] = (uint16_t)((nb << 11) | (int)v.x);
+                    pnf[b0 + e] = __int_as_float((int)v.y);
+                }
+            }
+            if (++nb == NB) break;
+        }
+        if (nb == 0) break;
+#ifdef FD_K2_TIMING
+        const long long tf1 = clock64();
+#endif
+        for (int i = 0; i < nb; ++i) {
+            mbar_wait(&mbar[i], (phases >> i) & 1u);
+            phases ^= 1u << i;
+        }
+        __syncthreads();                          // pool copies visible
+#ifdef FD_K2_TIMING
+        if (tid == 0) {
+            atomicAdd(&g_k2_timing[90], (unsigned long long)(tf1 - tf0));
+            atomicAdd(&g_k2_timing[91], (unsigned long long)(clock64() - tf1));
+            atomicAdd(&g_k2_timing[92], (unsigned long long)nb);
+            atomicAdd(&g_k2_timing[93], (unsigned long long)s_cnt[1]);
+        }
+#endif
+        deep_phase<STEP, DEPTH, CP>(p, slots, pnf, ploc, lists, s_cnt, s_tpos, out);
+    }
+}
+
+// k_deep1: the deeper stages, one tile per (small) CTA and many CTAs per SM.  Each CTA claims a
+// tile with stage-1 survivors, TMAs its ii plane and runs deep_phase over the survivors (in
+// chunks of CP); with ~25 KB of shared memory and 4 warps per CTA, FD_K2D_CTAS tiles are in
+// flight per SM, so the latency-bound stage chains of different tiles overlap.
+template <int STEP, bool DEPTH>
+__global__ void __launch_bounds__(K2D_THREADS, FD_K2D_CTAS) k_deep1(const __grid_constant__ CascadeParams p) {
+    using G = TileGeoD<STEP>;
+    constexpr int CP = G::CP, PLANE = tile_w(STEP) * tile_h(STEP);
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint32_t* slot = reinterpret_cast<uint32_t*>(smem_raw);
+    float* pnf = reinterpret_cast<float*>(smem_raw + G::OFF_NF);
+    uint16_t* ploc = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LOC);
+    uint16_t* lists = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LIST);
+    __shared__ __align__(8) uint64_t mbar;
+    __shared__ int s_frame[1], s_lvl[1], s_wx0[1], s_wy0[1];
+    __shared__ int s_cnt[3];
+    __shared__ int s_tpos, s_tile, s_off, s_n;
+    const int tid = threadIdx.x;
+    const WinOut<STEP, DEPTH> out{p, s_frame, s_lvl, s_wx0, s_wy0};
+    if (tid == 0) {
+        mbar_init(&mbar, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    uint32_t phase = 0;
+    for (;;) {
+        __syncthreads();
+        if (tid == 0) {
+            int tn;
+            uint2 tr = make_uint2(0u, 0u);
+            do {
+                tn = (int)atomicAdd(p.deep_counter, 1u);
+                if (tn >= p.total_tiles) break;
+                tr = p.tile_rec[tn];
+            } while (tr.y == 0u);
+            s_tile = tn;
+            if (tn < p.total_tiles) {
+                const TileAt t = tile_at<STEP>(p, tn);
+                s_frame[0] = p.frame_base + t.g;
+                s_lvl[0] = t.k;
+                s_wx0[0] = t.wx0;
+                s_wy0[0] = t.wy0;
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_expect_tx(&mbar, PLANE * 4);
+                tma_load_4d(slot, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar);
+                s_off = (int)tr.x;
+                s_n = (int)tr.y;
+            }
+        }
+        __syncthreads();
+        if (s_tile >= p.total_tiles) break;
+        const int off = s_off, n = s_n;
+        for (int c0 = 0; c0 < n; c0 += CP) {
+            const int m = min(CP, n - c0);
+            if (c0) __syncthreads();              // previous chunk's deep phase done with the pool
+            for (int e = tid; e < m; e += K2D_THREADS) {
+                const uint2 v = p.surv[off + c0 + e];
+                ploc[e] = (uint16_t)v.x;
+                pnf[e] = __int_as_float((int)v.y);
+            }
+            if (tid == 0) {
+                s_cnt[0] = 0;
+                s_cnt[1] = m;
+                s_cnt[2] = 0;
+            }
+            if (c0 == 0) {
+                mbar_wait(&mbar, phase);
+                phase ^= 1;
+            }
+            __syncthreads();
+            deep_phase<STEP, DEPTH, CP, K2D_THREADS>(p, slot, pnf, ploc, lists, s_cnt, s_tpos, out);
         }
     }
 }
 
 #ifndef __CUDACC_RTC__
-// TMA stages (FD_K2_STAGES=1|2, default 1: measured faster, 3 CTAs/SM hide more latency)
-static int k2_stages() {
-    static int v = [] {
-        const char* e = getenv("FD_K2_STAGES");
-        return (e && e[0] == '2') ? 2 : 1;
-    }();
-    return v;
-}
-
-template <int STEP, bool DEPTH, int NST>
+template <int STEP, bool DEPTH>
 static cudaError_t launch_one(const CascadeParams& p, int grid, cudaStream_t st) {
-    const size_t smem = TileGeo<STEP>::smem(NST);
-    cudaError_t e = cudaFuncSetAttribute(k_cascade<STEP, DEPTH, NST>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const size_t smem = TileGeo<STEP>::SMEM;
+    cudaError_t e = cudaFuncSetAttribute(k_cascade<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    k_cascade<STEP, DEPTH, NST><<<grid, k2_threads(STEP), smem, st>>>(p);
+    k_cascade<STEP, DEPTH><<<grid, k2_threads(STEP), smem, st>>>(p);
     return cudaGetLastError();
-}
-
-template <int STEP, bool DEPTH, int NST>
-static int grid_one() {
-    const size_t smem = TileGeo<STEP>::smem(NST);
-    cudaFuncSetAttribute(k_cascade<STEP, DEPTH, NST>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    int dev = 0, sms = 0, per = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_cascade<STEP, DEPTH, NST>, k2_threads(STEP), smem);
-    return sms * (per > 0 ? per : 1);
 }
 
 template <int STEP, bool DEPTH>
 static int grid_step() {
-    return k2_stages() == 1 ? grid_one<STEP, DEPTH, 1>() : grid_one<STEP, DEPTH, 2>();
+    const size_t smem = TileGeo<STEP>::SMEM;
+    cudaFuncSetAttribute(k_cascade<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int dev = 0, sms = 0, per = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_cascade<STEP, DEPTH>, k2_threads(STEP), smem);
+    return sms * (per > 0 ? per : 1);
 }
 
 template <int STEP, bool DEPTH>
 static cudaError_t launch_step(const CascadeParams& p, int grid, cudaStream_t st) {
-    return k2_stages() == 1 ? launch_one<STEP, DEPTH, 1>(p, grid, st) : launch_one<STEP, DEPTH, 2>(p, grid, st);
+    return launch_one<STEP, DEPTH>(p, grid, st);
 }
 
 size_t cascade_smem(int step) {
-    const int n = k2_stages();
     switch (step) {
-        case 1: return TileGeo<1>::smem(n);
-        case 2: return TileGeo<2>::smem(n);
-        case 3: return TileGeo<3>::smem(n);
-        default: return TileGeo<4>::smem(n);
+        case 1: return TileGeo<1>::SMEM;
+        case 2: return TileGeo<2>::SMEM;
+        case 3: return TileGeo<3>::SMEM;
+        default: return TileGeo<4>::SMEM;
     }
 }
 
@@ -491,6 +804,88 @@ cudaError_t launch_cascade(const CascadeParams& p, bool depth, int step, int gri
         case 2: return depth ? launch_step<2, true>(p, grid, st) : launch_step<2, false>(p, grid, st);
         case 3: return depth ? launch_step<3, true>(p, grid, st) : launch_step<3, false>(p, grid, st);
         case 4: return depth ? launch_step<4, true>(p, grid, st) : launch_step<4, false>(p, grid, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+
+template <int STEP, bool DEPTH>
+static cudaError_t launch_stage1_t(const CascadeParams& p, cudaStream_t st) {
+    static int grid = 0;
+    const size_t smem = TileGeoA<STEP>::SMEM;
+    cudaError_t e = cudaFuncSetAttribute(k_stage1<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    if (!grid) {
+        int dev = 0, sms = 0, per = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_stage1<STEP, DEPTH>, k2_threads(STEP), smem);
+        grid = sms * (per > 0 ? per : 1);
+    }
+    k_stage1<STEP, DEPTH><<<grid < p.total_tiles ? grid : p.total_tiles, k2_threads(STEP), smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+template <int STEP, bool DEPTH>
+static cudaError_t launch_deep_t(const CascadeParams& p, cudaStream_t st) {
+    static int grid = 0;
+    const size_t smem = TileGeoB<STEP, FD_K2B_NB>::SMEM;
+    cudaError_t e = cudaFuncSetAttribute(k_deep<STEP, DEPTH, FD_K2B_NB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    if (!grid) {
+        int dev = 0, sms = 0, per = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_deep<STEP, DEPTH, FD_K2B_NB>, k2_threads(STEP), smem);
+        grid = sms * (per > 0 ? per : 1);
+    }
+    k_deep<STEP, DEPTH, FD_K2B_NB><<<grid < p.total_tiles ? grid : p.total_tiles, k2_threads(STEP), smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_stage1(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
+    switch (step) {
+        case 1: return depth ? launch_stage1_t<1, true>(p, st) : launch_stage1_t<1, false>(p, st);
+        case 2: return depth ? launch_stage1_t<2, true>(p, st) : launch_stage1_t<2, false>(p, st);
+        case 3: return depth ? launch_stage1_t<3, true>(p, st) : launch_stage1_t<3, false>(p, st);
+        case 4: return depth ? launch_stage1_t<4, true>(p, st) : launch_stage1_t<4, false>(p, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+cudaError_t launch_deep(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
+    switch (step) {
+        case 1: return depth ? launch_deep_t<1, true>(p, st) : launch_deep_t<1, false>(p, st);
+        case 2: return depth ? launch_deep_t<2, true>(p, st) : launch_deep_t<2, false>(p, st);
+        case 3: return depth ? launch_deep_t<3, true>(p, st) : launch_deep_t<3, false>(p, st);
+        case 4: return depth ? launch_deep_t<4, true>(p, st) : launch_deep_t<4, false>(p, st);
+        default: return cudaErrorInvalidValue;
+    }
+}
+
+template <int STEP, bool DEPTH>
+static cudaError_t launch_deep1_t(const CascadeParams& p, cudaStream_t st) {
+    static int grid = 0;
+    const size_t smem = TileGeoD<STEP>::SMEM;
+    cudaError_t e = cudaFuncSetAttribute(k_deep1<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    if (!grid) {
+        int dev = 0, sms = 0, per = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_deep1<STEP, DEPTH>, K2D_THREADS, smem);
+        grid = sms * (per > 0 ? per : 1);
+    }
+    k_deep1<STEP, DEPTH><<<grid < p.total_tiles ? grid : p.total_tiles, K2D_THREADS, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_deep1(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
+    switch (step) {
+        case 1: return depth ? launch_deep1_t<1, true>(p, st) : launch_deep1_t<1, false>(p, st);
+        case 2: return depth ? launch_deep1_t<2, true>(p, st) : launch_deep1_t<2, false>(p, st);
+        case 3: return depth ? launch_deep1_t<3, true>(p, st) : launch_deep1_t<3, false>(p, st);
+        case 4: return depth ? launch_deep1_t<4, true>(p, st) : launch_deep1_t<4, false>(p, st);
         default: return cudaErrorInvalidValue;
     }
 }

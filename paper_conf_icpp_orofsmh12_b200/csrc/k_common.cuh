@@ -101,45 +101,64 @@ __device__ __forceinline__ float eval_stage(const uint32_t* __restrict__ T, int 
     return eval_stage_mc<MAX_CORNERS>(T, b, nf, rec, first, n);
 }
 
-// One stage for one window evaluated by a group of GL = 2^lg lanes (lane-aligned within a warp).
-// Per chunk of GL*LC stumps, lane q of the group evaluates stumps c0 + q + GL*r (r < LC,
-// independent, so LC loads are in flight) and parks the leaves at lv[r*32 + lane]
-// (conflict-free); the group leader (q == 0) then adds them in stump order, which keeps the
-// exact fp32 sequence of the definition (oracle c8).  The returned sum is valid in the leader.
-template <int MC, int LC>
-__device__ __forceinline__ float group_stage_mc(const uint32_t* __restrict__ T, int b, float nf, const GlobalRec& rec,
-                                                int first, int n, int lg, bool act, float* lv, int lane) {
-    const int gl = 1 << lg, q = lane & (gl - 1), g0 = lane & ~(gl - 1);
-    float sum = 0.0f;
-    for (int c0 = 0; c0 < n; c0 += gl * LC) {
-        if (act) {
-            float l[LC];
-#pragma unroll
-            for (int r = 0; r < LC; ++r) {
-                const int j = c0 + q + (r << lg);
-                l[r] = j < n ? eval_stump_mc<MC>(T, b, nf, rec, first + j) : 0.0f;
-            }
-#pragma unroll
-            for (int r = 0; r < LC; ++r) lv[r * 32 + lane] = l[r];
-        }
-        __syncwarp();
-        if (act && q == 0) {
-            const int cn = min(gl * LC, n - c0);
-#pragma unroll 8
-            for (int j = 0; j < cn; ++j) sum = __fadd_rn(sum, lv[(j >> lg) * 32 + g0 + (j & (gl - 1))]);
-        }
-        __syncwarp();
-    }
-    return sum;
+// Certified stage decision for warp-cooperative evaluation (GL lanes per window).  The
+// definition (oracle c8) adds the n leaves sequentially in fp32; a cooperative evaluation gets
+// the same leaves spread over lanes and adds them as a tree: per-lane sequential sums of c
+// leaves, then lg butterfly levels (depth d = c - 1 + lg; every lane of the group ends with the
+// same value).  Recursive summation of n terms satisfies |seq - S| <= gamma_{n-1} A and a tree of
+// depth d |tree - S| <= gamma_d A (A = sum |leaf|, gamma_m = m u / (1 - m u), u = 2^-24;
+// Higham, Accuracy and Stability of Numerical Algorithms, 2nd ed., 4.2), and the tree sum Ahat
+// of |leaf| bounds A <= Ahat / (1 - gamma_d).  So |seq - tree| <= (n + d) u Ahat (1 + O(nu)),
+// and B = (n + d + 2) * 2u * Ahat (+ 2^-100 absolute, for subnormal leaves) covers it with a 2x
+// margin that also absorbs the rounding of B and of (tree - T).  If tree - T > B the sequential
+// sum is >= T (pass); if T - tree > B it is < T (fail): the decision is the definition's.  Only
+// when neither holds (|tree - T| <= B, a near tie) does the caller recompute the sequential sum.
+// Returns 1 = pass, 0 = fail, -1 = undecided.
+__device__ __forceinline__ int certify(float acc, float aacc, int n, int d, float T) {
+    const float B = __fadd_rn(__fmul_rn(aacc, __fmul_rn(__int2float_rn(n + d + 2), 0x1p-23f)), 0x1p-100f);
+    const float diff = __fsub_rn(acc, T);
+    return diff > B ? 1 : (__fsub_rn(T, acc) > B ? 0 : -1);
 }
 
-template <int LC>
-__device__ __forceinline__ float group_stage(const uint32_t* __restrict__ T, int b, float nf, const GlobalRec& rec,
-                                             int first, int n, int mc, int lg, bool act, float* lv, int lane) {
-    if (mc <= 6) return group_stage_mc<6, LC>(T, b, nf, rec, first, n, lg, act, lv, lane);
-    if (mc <= 8) return group_stage_mc<8, LC>(T, b, nf, rec, first, n, lg, act, lv, lane);
-    if (mc <= 9) return group_stage_mc<9, LC>(T, b, nf, rec, first, n, lg, act, lv, lane);
-    return group_stage_mc<MAX_CORNERS, LC>(T, b, nf, rec, first, n, lg, act, lv, lane);
+// Tree-summed stage for a group of GL = 2^lg lanes per window: lane q evaluates stumps
+// q, q + GL, ... (four in flight), keeps the sum and the sum of magnitudes of its leaves, then
+// the group combines them with lg butterfly levels.  *d_out = tree depth (for certify).
+template <int MC, class R>
+__device__ __forceinline__ void group_stage_tree(const uint32_t* __restrict__ T, int b, float nf, const R& rec, int first,
+                                                 int n, int lg, bool act, int lane, float& acc, float& aacc) {
+    const int gl = 1 << lg, q = lane & (gl - 1);
+    acc = 0.0f;
+    aacc = 0.0f;
+    if (act) {
+        int j = q;
+        for (; j + 3 * gl < n; j += 4 * gl) {
+            const float l0 = eval_stump_mc<MC>(T, b, nf, rec, first + j);
+            const float l1 = eval_stump_mc<MC>(T, b, nf, rec, first + j + gl);
+            const float l2 = eval_stump_mc<MC>(T, b, nf, rec, first + j + 2 * gl);
+            const float l3 = eval_stump_mc<MC>(T, b, nf, rec, first + j + 3 * gl);
+            acc = __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(acc, l0), l1), l2), l3);
+            aacc = __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(aacc, fabsf(l0)), fabsf(l1)), fabsf(l2)), fabsf(l3));
+        }
+        for (; j < n; j += gl) {
+            const float l = eval_stump_mc<MC>(T, b, nf, rec, first + j);
+            acc = __fadd_rn(acc, l);
+            aacc = __fadd_rn(aacc, fabsf(l));
+        }
+    }
+    for (int o = gl >> 1; o > 0; o >>= 1) {
+        acc = __fadd_rn(acc, __shfl_xor_sync(0xffffffffu, acc, o));
+        aacc = __fadd_rn(aacc, __shfl_xor_sync(0xffffffffu, aacc, o));
+    }
+}
+
+template <class R>
+__device__ __forceinline__ void group_stage_tree_mc(const uint32_t* __restrict__ T, int b, float nf, const R& rec,
+                                                    int first, int n, int mc, int lg, bool act, int lane, float& acc,
+                                                    float& aacc) {
+    if (mc <= 6) return group_stage_tree<6>(T, b, nf, rec, first, n, lg, act, lane, acc, aacc);
+    if (mc <= 8) return group_stage_tree<8>(T, b, nf, rec, first, n, lg, act, lane, acc, aacc);
+    if (mc <= 9) return group_stage_tree<9>(T, b, nf, rec, first, n, lg, act, lane, acc, aacc);
+    return group_stage_tree<MAX_CORNERS>(T, b, nf, rec, first, n, lg, act, lane, acc, aacc);
 }
 
 // Dense first stage: each thread owns WPT windows of one column (stride STEP*TW words in

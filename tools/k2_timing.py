@@ -1,11 +1,11 @@
 #!/usr/bin/env python3
-"""Diagnostic: K2 phase cycles per tile (needs libfd_timing.so, FD_LIB_VARIANT=timing)."""
+"""Diagnostic: K2 phase cycles (needs libfd_timing.so, FD_LIB_VARIANT=timing, generic kernels)."""
 import ctypes as C
 import os
 import sys
 
 os.environ.setdefault("FD_LIB_VARIANT", "timing")
-os.environ.setdefault("FD_JIT", "0")   # the phase counters live in the generic K2
+os.environ.setdefault("FD_JIT", "0")   # the phase counters live in the precompiled kernels
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch  # noqa: E402
 
@@ -23,13 +23,20 @@ d = torch.from_numpy(fr).cuda()
 fd.fd_detect(casc, d, 24, s, 1, capacity=1 << 20)
 buf = (C.c_ulonglong * 128)()
 L.fd_debug_k2_timing(buf, 1)
+fd.fd_profile_reset(True)
 fd.fd_detect(casc, d, 24, s, 1, capacity=1 << 20)
 torch.cuda.synchronize()
+print({k: round(v[1], 3) for k, v in fd.fd_profile_read().items() if v[0]})
 L.fd_debug_k2_timing(buf, 0)
-t = buf[0]
-print(f"tiles {t}  per tile cycles: tma-wait {buf[1]/t:.0f}  stage1 {buf[2]/t:.0f}  deep {buf[3]/t:.0f}")
-print("tiles by deep-loop exit stage:", [buf[4 + i] for i in range(12)])
-print(f"tail: {buf[81]} warps, {buf[80]/max(buf[81],1):.0f} cycles each; mode M {buf[82]/t:.0f} / mode L {buf[83]/t:.0f} cycles per tile")
+b = list(buf)
+if b[0]:
+    print(f"tiles {b[0]}  per tile cycles: tma-wait {b[1]/b[0]:.0f}  stage1 {b[2]/b[0]:.0f}")
+nbat = max(b[84], 1)
+print(f"group-mode decisions {b[95]}  undecided {b[94]}  exact recomputes {b[96]}")
+print(f"deep batches {b[84]}  tiles/batch {b[92]/nbat:.2f}  pool/batch {b[93]/nbat:.1f}")
+print(f"per batch cycles: fill {b[90]/nbat:.0f}  tma-wait {b[91]/nbat:.0f}  deep {b[3]/nbat:.0f}")
+print("batches by deep-loop exit stage:", [b[4 + i] for i in range(12)])
+print(f"tail handoffs {b[81]} windows over {b[80] and 1}")
 for i in range(1, 32):
-    if buf[48 + i]:
-        print(f"  stage {i:2d}: {buf[48+i]:8d} tiles  {buf[16+i]/buf[48+i]:8.0f} cycles/tile  {buf[16+i]/t:8.0f} per tile overall")
+    if b[48 + i]:
+        print(f"  stage {i:2d}: {b[48+i]:8d} batches  {b[16+i]/b[48+i]:8.0f} cycles/batch  {b[16+i]/nbat:8.0f} per batch overall")
