@@ -10,7 +10,8 @@
 // K4: grouping: "two detection windows d_i and d_j overlap whenever
 // S_eyes(d_i,d_j) < 0.5 ... an iterative process reduces the initial set of windows by
 // progressively averaging those with the highest overlapping", S_eyes = eq. 6.
-// One CTA per frame; the greedy closest-pair order of the definition (reading R10) is kept
+// One CTA per frame, split into independent components (one warp each); the greedy
+// closest-pair order of the definition (reading R10) is kept
 // exactly by maintaining every cluster's nearest neighbour (ties -> lowest index) and
 // taking the lexicographically smallest (S, i, j) each round.  Double precision without FMA.
 #include <math_constants.h>
@@ -90,6 +91,9 @@ struct GroupScratch {        // per detection (structure of arrays, length n eac
     int* nn;
     double* nnd;
     Eyes* eyes;
+    int* parent;             // union-find over the frame's detections (frame-local indices)
+    int* list;               // members of each independent component, increasing index order
+    unsigned long long* box; // per component root: 9 bounds (doubles >= 0 as ordered bit patterns)
 };
 
 __device__ __forceinline__ Eyes cluster_eyes(const GroupScratch& g, int i) {
@@ -110,68 +114,74 @@ __device__ __forceinline__ bool key_less(const PairKey& x, const PairKey& y) {
     return x.b < y.b;
 }
 
-// nearest active neighbour of cluster i among [0, m) (ties -> lowest index); sequential
-__device__ void nn_full(const GroupScratch& g, int m, int i) {
-    const Eyes ei = g.eyes[i];
-    double best = CUDART_INF;
-    int bj = -1;
-    for (int j = 0; j < m; ++j) {
-        if (j == i || g.cnt[j] == 0) continue;
-        const double s = s_eyes(ei, g.eyes[j]);
-        if (s < best) {
-            best = s;
-            bj = j;
-        }
-    }
-    g.nn[i] = bj;
-    g.nnd[i] = best;
-}
-
 constexpr int GT = 256;
-constexpr int GLIST = 2048;     // clusters re-scanned warp-parallel per merge (overflow: per thread)
+// Segments = runs of equal frame in the sorted input. seg_start[s], n_seg on device.
+// One CTA per segment (frame).  The greedy loop is a chain of dependent merges, so the frame is
+// first split into INDEPENDENT components and each component runs its own greedy loop in one
+// warp (no block barriers per merge):
+//   * a cluster's eyes are the mean of its members' eyes and its d lies between its members'
+//     (means of the member rectangles), so every cluster of a component stays inside the
+//     bounding boxes of the component's left eyes, right eyes and d values;
+//   * for clusters A, B of components P, Q: S_eyes(A, B) >= (gap(LE_P, LE_Q) + gap(RE_P, RE_Q)) /
+//     min(dmax_P, dmax_Q) (Euclidean gaps between the boxes); components are merged (union-find)
+//     until that bound is >= thresh for every pair (with a margin over rounding), so no pair
+//     across components ever merges;
+//   * merges in different components commute, and inside a component the greedy order is the
+//     definition's: smallest (S, i, j) first (frame-local indices, members kept in increasing
+//     order), so the final clusters equal those of the frame-wide greedy loop (reading R10).
+// Nearest neighbours are kept over pairs with S_eyes < thresh only (the global minimum pair is
+// the same whenever it is below the threshold, and the loop stops otherwise); a pair whose
+// left- or right-eye coordinate gap alone forces S_eyes >= thresh skips the square roots.
+constexpr int GWARPS = GT / 32;
+constexpr int GROOTS = 1024;            // components tracked per frame (beyond: one component)
 
-__device__ PairKey block_min(PairKey v, PairKey* red) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        PairKey w;
-        w.s = __shfl_xor_sync(0xffffffffu, v.s, o);
-        w.a = __shfl_xor_sync(0xffffffffu, v.a, o);
-        w.b = __shfl_xor_sync(0xffffffffu, v.b, o);
-        if (key_less(w, v)) v = w;
+__device__ __forceinline__ int uf_find(int* parent, int x) {
+    for (;;) {
+        const int q = *reinterpret_cast<volatile int*>(parent + x);
+        if (q == x) return x;
+        x = q;
     }
-    __syncthreads();
-    if (lane == 0) red[warp] = v;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        PairKey r = red[0];
-        for (int w = 1; w < GT / 32; ++w)
-            if (key_less(red[w], r)) r = red[w];
-        red[0] = r;
+}
+__device__ __forceinline__ void uf_union(int* parent, int a, int b) {
+    for (;;) {
+        a = uf_find(parent, a);
+        b = uf_find(parent, b);
+        if (a == b) return;
+        if (a < b) {
+            const int t = a;
+            a = b;
+            b = t;
+        }
+        if (atomicCAS(parent + a, a, b) == a) return;     // root a under the smaller root b
     }
-    __syncthreads();
-    return red[0];
+}
+__device__ __forceinline__ unsigned long long dbits(double v) { return (unsigned long long)__double_as_longlong(v); }
+__device__ __forceinline__ double bitsd(unsigned long long v) { return __longlong_as_double((long long)v); }
+// Euclidean gap between intervals boxes [ax0,ax1]x[ay0,ay1] and [bx0,bx1]x[by0,by1]
+__device__ __forceinline__ double box_gap(double ax0, double ax1, double ay0, double ay1, double bx0, double bx1,
+                                          double by0, double by1) {
+    const double gx = fmax(0.0, fmax(__dsub_rn(bx0, ax1), __dsub_rn(ax0, bx1)));
+    const double gy = fmax(0.0, fmax(__dsub_rn(by0, ay1), __dsub_rn(ay0, by1)));
+    return __dsqrt_rn(__dadd_rn(__dmul_rn(gx, gx), __dmul_rn(gy, gy)));
+}
+// true when no cluster inside box a can ever reach S_eyes < thresh with one inside box b
+// (1e-6 absolute / relative margins over the rounding of cluster means, eyes and d)
+__device__ __forceinline__ bool independent(double gl, double gr, double da, double db, double thresh) {
+    return __dsub_rn(__dadd_rn(gl, gr), 4e-6) > __dmul_rn(__dmul_rn(thresh, fmin(da, db)), 1.000001);
 }
 
-// Segments = runs of equal frame in the sorted input. seg_start[s], n_seg on device.
-// Only pairs with S_eyes < thresh can ever be merged, so nearest neighbours are kept over those
-// pairs only (the greedy order of the definition is unchanged: the global minimum pair is the
-// same whenever it is below the threshold, and the loop stops otherwise).  A pair whose left-
-// or right-eye coordinate gap alone already forces S_eyes >= thresh is skipped without the
-// square roots and the division.
 __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ in, long long n,
                                               const long long* __restrict__ seg_start, const int* __restrict__ n_seg_p,
                                               double thresh, int min_neighbors, GroupScratch gs, int* seg_next,
                                               int* seg_count, fd_detection* __restrict__ tmp) {
-    __shared__ PairKey red[GT / 32];
-    __shared__ int s_seg;
-    __shared__ int s_nlist;
-    __shared__ int s_list[GLIST];
+    __shared__ int s_seg, s_changed, s_nroots, s_q;
+    __shared__ int s_roots[GROOTS], s_off[GROOTS], s_cnt[GROOTS];
     const int n_seg = *n_seg_p;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const double tguard = thresh * (1.0 + 0x1p-40);
     for (;;) {
         __syncthreads();
-        if (threadIdx.x == 0) s_seg = atomicAdd(seg_next, 1);
+        if (tid == 0) s_seg = atomicAdd(seg_next, 1);
         __syncthreads();
         const int sgi = s_seg;
         if (sgi >= n_seg) break;
@@ -180,122 +190,272 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
         const int m = (int)(a1 - a0);
         GroupScratch g = gs;
         g.sx += a0; g.sy += a0; g.sw += a0; g.sh += a0; g.cnt += a0; g.smax += a0;
-        g.nn += a0; g.nnd += a0; g.eyes += a0;
-        for (int i = threadIdx.x; i < m; i += GT) {
+        g.nn += a0; g.nnd += a0; g.eyes += a0; g.parent += a0; g.list += a0; g.box += 9 * a0;
+        for (int i = tid; i < m; i += GT) {
             const fd_detection d = in[a0 + i];
             g.sx[i] = d.x; g.sy[i] = d.y; g.sw[i] = d.w; g.sh[i] = d.h;
             g.cnt[i] = 1;
             g.smax[i] = d.score;
             g.eyes[i] = eyes_of((double)d.x, (double)d.y, (double)d.w, (double)d.h);
+            g.parent[i] = i;
         }
         __syncthreads();
-        // S_eyes of clusters kk, j, or +inf when a single coordinate gap proves S >= thresh:
-        // S = (d_le + d_re)/min(d) >= |gap|/min(d); the 2^-40 margin keeps every skipped pair's
-        // rounded S above thresh.
-        const double tguard = thresh * (1.0 + 0x1p-40);
-        auto dist = [&](int kk, int j) -> double {
-            const Eyes& a = g.eyes[kk];
-            const Eyes& b = g.eyes[j];
-            const double lim = tguard * (a.d < b.d ? a.d : b.d);
-            if (fabs(a.lex - b.lex) > lim || fabs(a.ley - b.ley) > lim || fabs(a.rex - b.rex) > lim) return CUDART_INF;
-            return s_eyes(a, b);
-        };
-        // warp-parallel nearest neighbour of cluster kk (lowest index on ties)
-        auto warp_nn = [&](int kk) {
-            double bs = CUDART_INF;
-            int bj = 0x7fffffff;
-            for (int j = lane; j < m; j += 32) {
-                if (j == kk || g.cnt[j] == 0) continue;
-                const double s = dist(kk, j);
-                if (s < bs) {        // j increases per lane: first minimum = lowest index
-                    bs = s;
-                    bj = j;
-                }
+        // ---- components: singleton pairs first
+        for (int i = tid; i < m; i += GT) {
+            const Eyes ei = g.eyes[i];
+            for (int j = i + 1; j < m; ++j) {
+                const Eyes ej = g.eyes[j];
+                const double lim = __dmul_rn(__dmul_rn(thresh, fmin(ei.d, ej.d)), 1.000001) + 4e-6;
+                if (fabs(ei.lex - ej.lex) > lim || fabs(ei.ley - ej.ley) > lim || fabs(ei.rex - ej.rex) > lim ||
+                    fabs(ei.rey - ej.rey) > lim)
+                    continue;
+                const double gl = box_gap(ei.lex, ei.lex, ei.ley, ei.ley, ej.lex, ej.lex, ej.ley, ej.ley);
+                const double gr = box_gap(ei.rex, ei.rex, ei.rey, ei.rey, ej.rex, ej.rex, ej.rey, ej.rey);
+                if (!independent(gl, gr, ei.d, ej.d, thresh)) uf_union(g.parent, i, j);
             }
-#pragma unroll
-            for (int o = 16; o > 0; o >>= 1) {
-                const double os = __shfl_xor_sync(0xffffffffu, bs, o);
-                const int oj = __shfl_xor_sync(0xffffffffu, bj, o);
-                if (os < bs || (os == bs && oj < bj)) {
-                    bs = os;
-                    bj = oj;
-                }
-            }
-            if (lane == 0) {
-                g.nn[kk] = bj == 0x7fffffff ? -1 : bj;
-                g.nnd[kk] = bs;
-            }
-        };
-        for (int i = warp; i < m; i += GT / 32) warp_nn(i);
-        __syncthreads();
+        }
+        // ---- then component boxes, until every pair of components is independent
+        bool whole = false;
         for (;;) {
-            PairKey best;
-            best.s = CUDART_INF;
-            best.a = 0x7fffffff;
-            best.b = 0x7fffffff;
-            for (int i = threadIdx.x; i < m; i += GT) {
-                if (g.cnt[i] == 0 || g.nn[i] < 0) continue;
-                PairKey c;
-                c.s = g.nnd[i];
-                c.a = min(i, g.nn[i]);
-                c.b = max(i, g.nn[i]);
-                if (key_less(c, best)) best = c;
+            __syncthreads();
+            if (tid == 0) {
+                s_changed = 0;
+                s_nroots = 0;
             }
-            best = block_min(best, red);
-            if (!(best.s < thresh) || best.a == 0x7fffffff) break;
-            const int a = best.a, b = best.b;
-            if (threadIdx.x == 0) {       // merge b into a (sums, count, max score)
-                g.sx[a] += g.sx[b]; g.sy[a] += g.sy[b]; g.sw[a] += g.sw[b]; g.sh[a] += g.sh[b];
-                g.cnt[a] += g.cnt[b];
-                if (g.smax[b] > g.smax[a]) g.smax[a] = g.smax[b];
-                g.cnt[b] = 0;
-                g.eyes[a] = cluster_eyes(g, a);
-                s_nlist = 0;
+            for (int i = tid; i < m; i += GT) g.parent[i] = uf_find(g.parent, i);
+            __syncthreads();
+            for (int i = tid; i < m; i += GT) {
+                if (g.parent[i] != i) continue;
+                const int r = atomicAdd(&s_nroots, 1);
+                if (r < GROOTS) s_roots[r] = i;
+                unsigned long long* bx = g.box + 9 * i;
+#pragma unroll
+                for (int c = 0; c < 4; ++c) {
+                    bx[2 * c] = dbits(CUDART_INF);
+                    bx[2 * c + 1] = 0ull;
+                }
+                bx[8] = 0ull;
             }
             __syncthreads();
-            // nearest-neighbour maintenance: clusters whose neighbour was a or b (and a itself)
-            // are re-scanned warp-parallel below; every other cluster only compares with the new a.
-            for (int kk = threadIdx.x; kk < m; kk += GT) {
-                if (g.cnt[kk] == 0) continue;
-                const int nk = g.nn[kk];
-                if (kk == a || nk == a || nk == b) {
-                    const int pos = atomicAdd(&s_nlist, 1);
-                    if (pos < GLIST) s_list[pos] = kk;
-                    else nn_full(g, m, kk);
-                } else {
-                    const double s = dist(kk, a);
-                    if (s < g.nnd[kk] || (s == g.nnd[kk] && a < nk)) {
-                        g.nnd[kk] = s;
-                        g.nn[kk] = a;
+            if (s_nroots > GROOTS) {               // too many components to track: one for the frame
+                whole = true;
+                break;
+            }
+            for (int i = tid; i < m; i += GT) {
+                const Eyes e = g.eyes[i];
+                unsigned long long* bx = g.box + 9 * g.parent[i];
+                atomicMin(bx + 0, dbits(e.lex)); atomicMax(bx + 1, dbits(e.lex));
+                atomicMin(bx + 2, dbits(e.ley)); atomicMax(bx + 3, dbits(e.ley));
+                atomicMin(bx + 4, dbits(e.rex)); atomicMax(bx + 5, dbits(e.rex));
+                atomicMin(bx + 6, dbits(e.rey)); atomicMax(bx + 7, dbits(e.rey));
+                atomicMax(bx + 8, dbits(e.d));
+            }
+            __syncthreads();
+            const int K = s_nroots;
+            const long long npairs = (long long)K * (K - 1) / 2;
+            for (long long t = tid; t < npairs; t += GT) {
+                // pair index t -> (u, v), u < v
+                int u = (int)((sqrt(8.0 * (double)t + 1.0) - 1.0) * 0.5);
+                while ((long long)(u + 1) * u / 2 > t) --u;
+                while ((long long)(u + 2) * (u + 1) / 2 <= t) ++u;
+                const int v = (int)(t - (long long)(u + 1) * u / 2);
+                const int ra = s_roots[u + 1], rb = s_roots[v];
+                const unsigned long long* A = g.box + 9 * ra;
+                const unsigned long long* B = g.box + 9 * rb;
+                const double gl = box_gap(bitsd(A[0]), bitsd(A[1]), bitsd(A[2]), bitsd(A[3]), bitsd(B[0]), bitsd(B[1]),
+                                          bitsd(B[2]), bitsd(B[3]));
+                const double gr = box_gap(bitsd(A[4]), bitsd(A[5]), bitsd(A[6]), bitsd(A[7]), bitsd(B[4]), bitsd(B[5]),
+                                          bitsd(B[6]), bitsd(B[7]));
+                if (!independent(gl, gr, bitsd(A[8]), bitsd(B[8]), thresh)) {
+                    uf_union(g.parent, ra, rb);
+                    s_changed = 1;
+                }
+            }
+            __syncthreads();
+            if (!s_changed) break;
+        }
+        // ---- member lists (increasing index order) per component
+        const int K = whole ? 1 : s_nroots;
+        if (whole) {
+            for (int i = tid; i < m; i += GT) g.list[i] = i;
+            if (tid == 0) {
+                s_off[0] = 0;
+                s_cnt[0] = m;
+            }
+        } else {
+            for (int r = warp; r < K; r += GWARPS) {
+                const int root = s_roots[r];
+                int c = 0;
+                for (int k0 = 0; k0 < m; k0 += 32) {
+                    const int i = k0 + lane;
+                    c += __popc(__ballot_sync(0xffffffffu, i < m && g.parent[i] == root));
+                }
+                if (lane == 0) s_cnt[r] = c;
+            }
+            __syncthreads();
+            if (tid == 0) {
+                int acc = 0;
+                for (int r = 0; r < K; ++r) {
+                    s_off[r] = acc;
+                    acc += s_cnt[r];
+                }
+            }
+            __syncthreads();
+            for (int r = warp; r < K; r += GWARPS) {
+                const int root = s_roots[r];
+                int c = s_off[r];
+                for (int k0 = 0; k0 < m; k0 += 32) {
+                    const int i = k0 + lane;
+                    const bool in_r = i < m && g.parent[i] == root;
+                    const unsigned bm = __ballot_sync(0xffffffffu, in_r);
+                    if (in_r) g.list[c + __popc(bm & ((1u << lane) - 1u))] = i;
+                    c += __popc(bm);
+                }
+            }
+        }
+        __syncthreads();
+        // ---- greedy loop per component, one warp each
+        for (int r = warp; r < K; r += GWARPS) {
+            const int* L = g.list + s_off[r];
+            const int mc = s_cnt[r];
+            if (mc < 2) continue;
+            auto dist = [&](const Eyes& a, int j) -> double {
+                const Eyes b = g.eyes[j];
+                const double lim = tguard * (a.d < b.d ? a.d : b.d);
+                if (fabs(a.lex - b.lex) > lim || fabs(a.ley - b.ley) > lim || fabs(a.rex - b.rex) > lim) return CUDART_INF;
+                return s_eyes(a, b);
+            };
+            // nearest neighbour of cluster kk over the component (lowest index on ties)
+            auto warp_nn = [&](int kk) {
+                const Eyes ek = g.eyes[kk];
+                double bs = CUDART_INF;
+                int bj = 0x7fffffff;
+                for (int q = lane; q < mc; q += 32) {
+                    const int j = L[q];
+                    if (j == kk || g.cnt[j] == 0) continue;
+                    const double s = dist(ek, j);
+                    if (s < bs) {
+                        bs = s;
+                        bj = j;
+                    }
+                }
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) {
+                    const double os = __shfl_xor_sync(0xffffffffu, bs, o);
+                    const int oj = __shfl_xor_sync(0xffffffffu, bj, o);
+                    if (os < bs || (os == bs && oj < bj)) {
+                        bs = os;
+                        bj = oj;
+                    }
+                }
+                if (lane == 0) {
+                    g.nn[kk] = bj == 0x7fffffff ? -1 : bj;
+                    g.nnd[kk] = bs;
+                }
+            };
+            for (int q = lane; q < mc; q += 32) {
+                const int i = L[q];
+                const Eyes ei = g.eyes[i];
+                double bs = CUDART_INF;
+                int bj = -1;
+                for (int q2 = 0; q2 < mc; ++q2) {
+                    const int j = L[q2];
+                    if (j == i) continue;
+                    const double s = dist(ei, j);
+                    if (s < bs) {
+                        bs = s;
+                        bj = j;
+                    }
+                }
+                g.nn[i] = bj;
+                g.nnd[i] = bs;
+            }
+            __syncwarp();
+            for (;;) {
+                PairKey best;
+                best.s = CUDART_INF;
+                best.a = 0x7fffffff;
+                best.b = 0x7fffffff;
+                for (int q = lane; q < mc; q += 32) {
+                    const int i = L[q];
+                    if (g.cnt[i] == 0 || g.nn[i] < 0) continue;
+                    PairKey c;
+                    c.s = g.nnd[i];
+                    c.a = min(i, g.nn[i]);
+                    c.b = max(i, g.nn[i]);
+                    if (key_less(c, best)) best = c;
+                }
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) {
+                    PairKey w;
+                    w.s = __shfl_xor_sync(0xffffffffu, best.s, o);
+                    w.a = __shfl_xor_sync(0xffffffffu, best.a, o);
+                    w.b = __shfl_xor_sync(0xffffffffu, best.b, o);
+                    if (key_less(w, best)) best = w;
+                }
+                if (!(best.s < thresh) || best.a == 0x7fffffff) break;
+                const int a = best.a, b = best.b;
+                if (lane == 0) {       // merge b into a (sums, count, max score)
+                    g.sx[a] += g.sx[b]; g.sy[a] += g.sy[b]; g.sw[a] += g.sw[b]; g.sh[a] += g.sh[b];
+                    g.cnt[a] += g.cnt[b];
+                    if (g.smax[b] > g.smax[a]) g.smax[a] = g.smax[b];
+                    g.cnt[b] = 0;
+                    g.eyes[a] = cluster_eyes(g, a);
+                }
+                __syncwarp();
+                // clusters whose neighbour was a or b (and a itself) are re-scanned; every other
+                // cluster only compares with the new a
+                const Eyes ea = g.eyes[a];
+                for (int q0 = 0; q0 < mc; q0 += 32) {
+                    const int kk = q0 + lane < mc ? L[q0 + lane] : -1;
+                    bool rescan = false;
+                    if (kk >= 0 && g.cnt[kk] != 0) {
+                        const int nk = g.nn[kk];
+                        if (kk == a || nk == a || nk == b) {
+                            rescan = true;
+                        } else {
+                            const double s = dist(ea, kk);
+                            if (s < g.nnd[kk] || (s == g.nnd[kk] && a < nk)) {
+                                g.nnd[kk] = s;
+                                g.nn[kk] = a;
+                            }
+                        }
+                    }
+                    unsigned rm = __ballot_sync(0xffffffffu, rescan);
+                    __syncwarp();
+                    while (rm) {
+                        const int t = __ffs(rm) - 1;
+                        rm &= rm - 1;
+                        warp_nn(L[q0 + t]);
+                        __syncwarp();
                     }
                 }
             }
-            __syncthreads();
-            {
-                const int nl = min(s_nlist, GLIST);
-                for (int e = warp; e < nl; e += GT / 32) warp_nn(s_list[e]);
-            }
-            __syncthreads();
         }
-        // emit clusters in first-member order (thread 0; clusters are few)
-        if (threadIdx.x == 0) {
+        __syncthreads();
+        // ---- emit clusters in first-member order (warp 0, ballot compaction over the frame)
+        if (warp == 0) {
             int q = 0;
-            for (int i = 0; i < m; ++i) {
-                if (g.cnt[i] == 0 || g.cnt[i] < min_neighbors) continue;
-                const fd_detection d0 = in[a0 + i];
-                const double nn = (double)g.cnt[i];
-                fd_detection o;
-                o.frame = d0.frame; o.level = d0.level; o.wx = d0.wx; o.wy = d0.wy;
-                o.x = (int)floor(__dadd_rn(__ddiv_rn((double)g.sx[i], nn), 0.5));
-                o.y = (int)floor(__dadd_rn(__ddiv_rn((double)g.sy[i], nn), 0.5));
-                o.w = (int)floor(__dadd_rn(__ddiv_rn((double)g.sw[i], nn), 0.5));
-                o.h = (int)floor(__dadd_rn(__ddiv_rn((double)g.sh[i], nn), 0.5));
-                o.score = g.smax[i];
-                o.aux = g.cnt[i];
-                tmp[a0 + q] = o;
-                ++q;
+            for (int k0 = 0; k0 < m; k0 += 32) {
+                const int i = k0 + lane;
+                const bool keep = i < m && g.cnt[i] != 0 && g.cnt[i] >= min_neighbors;
+                const unsigned km = __ballot_sync(0xffffffffu, keep);
+                if (keep) {
+                    const fd_detection d0 = in[a0 + i];
+                    const double nn = (double)g.cnt[i];
+                    fd_detection o;
+                    o.frame = d0.frame; o.level = d0.level; o.wx = d0.wx; o.wy = d0.wy;
+                    o.x = (int)floor(__dadd_rn(__ddiv_rn((double)g.sx[i], nn), 0.5));
+                    o.y = (int)floor(__dadd_rn(__ddiv_rn((double)g.sy[i], nn), 0.5));
+                    o.w = (int)floor(__dadd_rn(__ddiv_rn((double)g.sw[i], nn), 0.5));
+                    o.h = (int)floor(__dadd_rn(__ddiv_rn((double)g.sh[i], nn), 0.5));
+                    o.score = g.smax[i];
+                    o.aux = g.cnt[i];
+                    tmp[a0 + q + __popc(km & ((1u << lane) - 1u))] = o;
+                }
+                q += __popc(km);
             }
-            seg_count[sgi] = q;
+            if (lane == 0) seg_count[sgi] = q;
         }
     }
 }
@@ -376,6 +536,9 @@ struct GroupLayout {
         g.nn = reinterpret_cast<int*>(take(a * 4));
         g.nnd = reinterpret_cast<double*>(take(a * 8));
         g.eyes = reinterpret_cast<Eyes*>(take(a * sizeof(Eyes)));
+        g.parent = reinterpret_cast<int*>(take(a * 4));
+        g.list = reinterpret_cast<int*>(take(a * 4));
+        g.box = reinterpret_cast<unsigned long long*>(take(a * 72));
         seg_start = reinterpret_cast<long long*>(take(a * 8));
         seg_count = reinterpret_cast<int*>(take(a * 4));
         seg_off = reinterpret_cast<long long*>(take(a * 8));
@@ -386,7 +549,7 @@ struct GroupLayout {
 
 size_t group_scratch_bytes(long long n) {
     const size_t a = (size_t)(n > 0 ? n : 1);
-    return a * (4 * 8 + 4 + 4 + 4 + 8 + sizeof(Eyes) + 8 + 4 + 8 + sizeof(fd_detection)) + 20 * 256;
+    return a * (4 * 8 + 4 + 4 + 4 + 8 + sizeof(Eyes) + 4 + 4 + 72 + 8 + 4 + 8 + sizeof(fd_detection)) + 24 * 256;
 }
 
 // phase 1: frame segments (runs of equal frame index)
@@ -409,7 +572,7 @@ cudaError_t launch_group_run(const fd_detection* in, long long n, double thresh,
     const int grid = (int)(n < (long long)sms * 4 ? n : (long long)sms * 4);
     k_group<<<grid, GT, 0, st>>>(in, n, L.seg_start, L.misc, thresh, min_neighbors, L.g, L.misc + 1, L.seg_count, L.tmp);
     k_seg_offsets<<<1, 32, 0, st>>>(L.misc, L.seg_count, L.seg_off, d_total);
-    k_seg_copy<<<grid, 256, 0, st>>>(L.misc, L.seg_start, L.seg_count, L.seg_off, L.tmp, out, cap);
+    k_seg_copy<<<grid < sms * 4 ? grid : sms * 4, 256, 0, st>>>(L.misc, L.seg_start, L.seg_count, L.seg_off, L.tmp, out, cap);
     return cudaGetLastError();
 }
 
