@@ -467,11 +467,12 @@ struct DevBuf {
     }
 };
 
-struct Workspace {
-    int device = 0;
-    std::mutex mu;                 // one call at a time per (device, stream)
-    DevBuf ws, colbuf, rowbuf, corbuf, lvlbuf, keys, scores, keys2, scores2, cubtmp, ctl, flev, frames, outbuf, group, grpout,
-        tmaps, lvbuf, tailq, surv, tilerec;
+// Per-frame-group buffers of the K1 -> K2 pipeline: integral planes, K1 scratch, tensor maps,
+// stage-1 survivor list, tile records and tail queue.  run_groups alternates frame groups
+// between two such slots on two streams, so K1 of group g+1 overlaps the latency-bound deep
+// stages and tail of group g (different resources: HBM vs issue/latency).
+struct PipeSlot {
+    DevBuf ws, colbuf, rowbuf, corbuf, lvlbuf, tmaps, tailq, surv, tilerec;
     // K1 scratch for g frames of plan p
     cudaError_t k1_scratch(const PlanDev& p, int g, K1Scratch* s) {
         cudaError_t e = colbuf.ensure((size_t)g * p.col_frame * 4 + 16);
@@ -484,14 +485,34 @@ struct Workspace {
         s->cor = corbuf.as<unsigned long long>();
         return e;
     }
+};
+
+struct Workspace {
+    int device = 0;
+    std::mutex mu;                 // one call at a time per (device, stream)
+    DevBuf keys, scores, keys2, scores2, cubtmp, ctl, flev, frames, outbuf, group, grpout, lvbuf;
+    PipeSlot slot[2];              // pipeline slots (slot 0 also serves fd_integral / fd_build_pyramid)
+    cudaStream_t side = nullptr;   // stream of slot 1, forked from / joined to the caller's stream
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    cudaError_t ensure_side() {
+        if (side) return cudaSuccess;
+        cudaError_t e = cudaStreamCreateWithFlags(&side, cudaStreamNonBlocking);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_fork, cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_join, cudaEventDisableTiming);
+        return e;
+    }
+    cudaError_t k1_scratch(const PlanDev& p, int g, K1Scratch* s) { return slot[0].k1_scratch(p, g, s); }
     unsigned long long* h_pinned = nullptr;     // pinned host word(s) for count read-back
     std::unique_ptr<CascadeParams> params{new CascadeParams()};
     std::unique_ptr<PlanDev> plan{new PlanDev()};
     // host staging of tensor maps + level table (kept alive until the async copies run)
-    std::unique_ptr<CUtensorMap[]> h_geo{new CUtensorMap[FD_MAX_LEVELS + (sizeof(LevelDev) * FD_MAX_LEVELS +
-                                                                          sizeof(CUtensorMap) - 1) / sizeof(CUtensorMap)]};
+    std::unique_ptr<CUtensorMap[]> h_geo{new CUtensorMap[2 * FD_MAX_LEVELS + (sizeof(LevelDev) * FD_MAX_LEVELS +
+                                                                              sizeof(CUtensorMap) - 1) / sizeof(CUtensorMap)]};
     ~Workspace() {
         if (h_pinned) cudaFreeHost(h_pinned);
+        if (ev_fork) cudaEventDestroy(ev_fork);
+        if (ev_join) cudaEventDestroy(ev_join);
+        if (side) cudaStreamDestroy(side);
     }
 };
 
@@ -547,45 +568,49 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     const int ngroups = (n + G - 1) / G;
     PlanDev& PD = *w->plan;
     make_plan_dev(pl, W, H, pitch, step, G, &PD);
-    CK(w->ws.ensure((size_t)PD.ws_elems * 4));
-    K1Scratch k1s;
-    CK(w->k1_scratch(PD, G, &k1s));
-    // ctl: [0] detection count, [256 B..] per-group K2 tile counters, then per-group tail counts,
-    // survivor counts and k_deep tile counters
-    CK(w->ctl.ensure(256 + (size_t)ngroups * 16));
-    CK(cudaMemsetAsync(w->ctl.p, 0, 256 + (size_t)ngroups * 16, st));
+    // two pipeline slots on two streams when there is more than one group (FD_PIPE=0: one)
+    const int nslots = (ngroups > 1 && env_int("FD_PIPE", 1) != 0) ? 2 : 1;
     // K2 split in two kernels (k_stage1: dense first stage, k_deep: batched deeper stages;
     // FD_K2_SPLIT=0 runs the fused k_cascade).  Survivor list sized for the worst case.
     const bool split = env_int("FD_K2_SPLIT", 1) != 0;
     const bool deep1 = env_int("FD_K2_DEEP1", 1) != 0;      // k_deep1 (tile per small CTA) or batched k_deep
-    if (split) {
-        CK(w->surv.ensure((size_t)G * (size_t)PD.win_per_frame * 8 + 16));
-        CK(w->tilerec.ensure((size_t)G * PD.tiles_per_frame * 8 + 16));
-    }
     // tail queue (k_tail): FD_TAIL=0 keeps every window inside K2; FD_TAIL_N = windows left in a
     // batch at which it hands them over; FD_TAIL_CAP = queue entries (16 B each) per group
     const bool use_tail = env_int("FD_TAIL", 1) != 0;
     const int tail_cap = use_tail ? std::max(1024, env_int("FD_TAIL_CAP", 1 << 22)) : 0;
-    if (use_tail) CK(w->tailq.ensure((size_t)tail_cap * 16));
+    K1Scratch k1s[2];
+    std::vector<CUtensorMap> maps((size_t)PD.n_levels);
+    for (int b = 0; b < nslots; ++b) {
+        PipeSlot& sl = w->slot[b];
+        CK(sl.ws.ensure((size_t)PD.ws_elems * 4));
+        CK(sl.k1_scratch(PD, G, &k1s[b]));
+        if (split) {
+            CK(sl.surv.ensure((size_t)G * (size_t)PD.win_per_frame * 8 + 16));
+            CK(sl.tilerec.ensure((size_t)G * PD.tiles_per_frame * 8 + 16));
+        }
+        if (use_tail) CK(sl.tailq.ensure((size_t)tail_cap * 16));
+        // tensor maps of this slot's integral planes (global memory, copied in stream order)
+        s = encode_maps(PD, sl.ws.as<uint32_t>(), step, 1, maps.data());
+        if (s != FD_OK) return s;
+        CK(sl.tmaps.ensure(sizeof(CUtensorMap) * FD_MAX_LEVELS));
+        std::memcpy(w->h_geo.get() + b * FD_MAX_LEVELS, maps.data(), sizeof(CUtensorMap) * PD.n_levels);
+        CK(cudaMemcpyAsync(sl.tmaps.p, w->h_geo.get() + b * FD_MAX_LEVELS, sizeof(CUtensorMap) * PD.n_levels,
+                           cudaMemcpyHostToDevice, st));
+    }
+    // ctl: [0] detection count, [256 B..] per-group K2 tile counters, then per-group tail counts,
+    // survivor counts and k_deep tile counters
+    CK(w->ctl.ensure(256 + (size_t)ngroups * 16));
+    CK(cudaMemsetAsync(w->ctl.p, 0, 256 + (size_t)ngroups * 16, st));
     if (!depth) {
         const size_t cap = (size_t)(det_cap > 0 ? det_cap : 1);
         CK(w->keys.ensure(cap * 8));
         CK(w->scores.ensure(cap * 4));
     }
-    // tensor maps + level table for K2 (global memory, copied in stream order)
-    std::vector<CUtensorMap> maps((size_t)PD.n_levels);
-    s = encode_maps(PD, w->ws.as<uint32_t>(), step, 1, maps.data());
-    if (s != FD_OK) return s;
-    CK(w->tmaps.ensure(sizeof(CUtensorMap) * FD_MAX_LEVELS));
     CK(w->lvbuf.ensure(sizeof(LevelDev) * FD_MAX_LEVELS));
-    std::memcpy(w->h_geo.get(), maps.data(), sizeof(CUtensorMap) * PD.n_levels);
-    std::memcpy(reinterpret_cast<char*>(w->h_geo.get()) + sizeof(CUtensorMap) * FD_MAX_LEVELS, PD.lv,
-                sizeof(LevelDev) * PD.n_levels);
-    CK(cudaMemcpyAsync(w->tmaps.p, w->h_geo.get(), sizeof(CUtensorMap) * PD.n_levels, cudaMemcpyHostToDevice, st));
-    CK(cudaMemcpyAsync(w->lvbuf.p, reinterpret_cast<char*>(w->h_geo.get()) + sizeof(CUtensorMap) * FD_MAX_LEVELS,
-                       sizeof(LevelDev) * PD.n_levels, cudaMemcpyHostToDevice, st));
+    char* h_lv = reinterpret_cast<char*>(w->h_geo.get() + 2 * FD_MAX_LEVELS);
+    std::memcpy(h_lv, PD.lv, sizeof(LevelDev) * PD.n_levels);
+    CK(cudaMemcpyAsync(w->lvbuf.p, h_lv, sizeof(LevelDev) * PD.n_levels, cudaMemcpyHostToDevice, st));
     CascadeParams& P = *w->params;
-    P.tmaps = w->tmaps.as<CUtensorMap>();
     P.lv = w->lvbuf.as<LevelDev>();
     P.n_levels = PD.n_levels;
     P.tiles_per_frame = PD.tiles_per_frame;
@@ -608,14 +633,11 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     // group mode covers every window in one pass only while n <= threads / 2
     const int half = k2_threads(step) / 2;
     P.lane_min = std::max(1, std::min(env_int("FD_LANE_MIN", half + 1), half + 1));
-    P.tail_q = use_tail ? w->tailq.as<uint4>() : nullptr;
     P.tail_cap = tail_cap;
     P.tail_n = std::max(1, env_int("FD_TAIL_N", 8));
     TailParams TP;
-    TP.q = P.tail_q;
     TP.cap = tail_cap;
     TP.step = step;
-    TP.ws = w->ws.as<uint32_t>();
     TP.lv = P.lv;
     TP.trec = pk->d_trec;
     TP.ns = (int)c->stumps.size();
@@ -641,16 +663,31 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         }
         jit = c->jit;
     }
+    // slot 1's stream starts after everything the caller queued on st so far (and the copies above)
+    cudaStream_t sts[2] = {st, st};
+    if (nslots == 2) {
+        CK(w->ensure_side());
+        CK(cudaEventRecord(w->ev_fork, st));
+        CK(cudaStreamWaitEvent(w->side, w->ev_fork, 0));
+        sts[1] = w->side;
+    }
     const int grid = cascade_grid(depth, step);
     for (int gi = 0; gi < ngroups; ++gi) {
+        // group gi runs on slot gi % nslots; the slot's stream orders it after group gi - nslots,
+        // the previous user of the slot's buffers
+        const int b = gi % nslots;
+        PipeSlot& sl = w->slot[b];
+        const cudaStream_t gs = sts[b];
         const int f0 = gi * G, gf = (n - f0) < G ? (n - f0) : G;
         const uint8_t* fr = d_frames + (size_t)f0 * H * pitch;
-        LAUNCH(FD_K_COLSUM, st, launch_k1_marg(fr, PD, gf, k1s, st));
+        LAUNCH(FD_K_COLSUM, gs, launch_k1_marg(fr, PD, gf, k1s[b], gs));
         {
-            ProfScope ps(FD_K_CARRY, st, 2);
-            CK(launch_k1_carry(PD, gf, k1s, st));
+            ProfScope ps(FD_K_CARRY, gs, 2);
+            CK(launch_k1_carry(PD, gf, k1s[b], gs));
         }
-        LAUNCH(FD_K_BAND, st, launch_k1_tiles(fr, PD, gf, k1s, w->ws.as<uint32_t>(), st));
+        LAUNCH(FD_K_BAND, gs, launch_k1_tiles(fr, PD, gf, k1s[b], sl.ws.as<uint32_t>(), gs));
+        P.tmaps = sl.tmaps.as<CUtensorMap>();
+        P.tail_q = use_tail ? sl.tailq.as<uint4>() : nullptr;
         P.g_frames = gf;
         P.frame_base = f0;
         P.total_tiles = gf * PD.tiles_per_frame;
@@ -658,33 +695,39 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         P.tail_count = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + ngroups + gi;
         P.surv_count = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + 2 * ngroups + gi;
         P.deep_counter = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + 3 * ngroups + gi;
-        P.surv = split ? w->surv.as<uint2>() : nullptr;
-        P.tile_rec = split ? w->tilerec.as<uint2>() : nullptr;
+        P.surv = split ? sl.surv.as<uint2>() : nullptr;
+        P.tile_rec = split ? sl.tilerec.as<uint2>() : nullptr;
         const int gr = grid < P.total_tiles ? grid : P.total_tiles;
         if (jit) {
             std::string err;
             cudaError_t e;
             {
-                ProfScope ps(FD_K_CASCADE, st);
-                e = jit_k2_launch(jit, P, depth, split ? JIT_STAGE1 : JIT_FUSED, st, &err);
+                ProfScope ps(FD_K_CASCADE, gs);
+                e = jit_k2_launch(jit, P, depth, split ? JIT_STAGE1 : JIT_FUSED, gs, &err);
             }
             if (e == cudaSuccess && split) {
-                ProfScope ps(FD_K_DEEP, st);
-                e = jit_k2_launch(jit, P, depth, deep1 ? JIT_DEEP1 : JIT_DEEP, st, &err);
+                ProfScope ps(FD_K_DEEP, gs);
+                e = jit_k2_launch(jit, P, depth, deep1 ? JIT_DEEP1 : JIT_DEEP, gs, &err);
             }
             if (e != cudaSuccess)
                 return fail(FD_ECUDA, "specialised K2: %s", err.empty() ? cudaGetErrorString(e) : err.c_str());
         } else if (split) {
-            LAUNCH(FD_K_CASCADE, st, launch_stage1(P, depth, step, st));
-            LAUNCH(FD_K_DEEP, st, deep1 ? launch_deep1(P, depth, step, st) : launch_deep(P, depth, step, st));
+            LAUNCH(FD_K_CASCADE, gs, launch_stage1(P, depth, step, gs));
+            LAUNCH(FD_K_DEEP, gs, deep1 ? launch_deep1(P, depth, step, gs) : launch_deep(P, depth, step, gs));
         } else {
-            LAUNCH(FD_K_CASCADE, st, launch_cascade(P, depth, step, gr, st));
+            LAUNCH(FD_K_CASCADE, gs, launch_cascade(P, depth, step, gr, gs));
         }
         if (use_tail) {
+            TP.q = P.tail_q;
+            TP.ws = sl.ws.as<uint32_t>();
             TP.count = P.tail_count;
             TP.frame_base = f0;
-            LAUNCH(FD_K_TAIL, st, launch_tail(TP, depth, st));
+            LAUNCH(FD_K_TAIL, gs, launch_tail(TP, depth, gs));
         }
+    }
+    if (nslots == 2) {       // the caller's stream continues after both slots
+        CK(cudaEventRecord(w->ev_join, w->side));
+        CK(cudaStreamWaitEvent(st, w->ev_join, 0));
     }
     return FD_OK;
 }

@@ -82,6 +82,7 @@ def main():
              f"(one K2 launch = {a.frames_per_launch} 1080p frames). ncu flushes caches before each replayed "
              "kernel, so DRAM bytes are cold-cache upper bounds.", ""]
     traffic = {}
+    seen = set()
     for k in kernels:
         name = k.get("Kernel Name", "?").split("(")[0]
         lines.append(f"## {name}")
@@ -95,11 +96,14 @@ def main():
         dr = (num(k.get("dram__bytes_read.sum")) or 0) + (num(k.get("dram__bytes_write.sum")) or 0)
         ub = units.get("dram__bytes_read.sum", "byte")
         scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(ub, 1)
-        if "k_cascade" in name and "k_cascade_dram_bytes_per_launch" not in traffic:
-            traffic["k_cascade_dram_bytes_per_launch"] = dr * scale
+        # per-launch DRAM bytes of each K2 kernel family and of K1 (first capture of each kernel)
+        fam = ("k_stage1" if "k_stage1" in name else "k_deep" if ("k_deep" in name or "k_tail" in name)
+               else "k1" if any(t in name for t in ("k_marg", "k_carry", "k_corner", "k_tile")) else None)
+        if fam and name not in seen:
+            seen.add(name)
+            key = f"{fam}_dram_bytes_per_launch"
+            traffic[key] = traffic.get(key, 0.0) + dr * scale
             traffic["frames_per_launch"] = a.frames_per_launch
-        if "k_band" in name and "k_band_dram_bytes_per_launch" not in traffic:
-            traffic["k_band_dram_bytes_per_launch"] = dr * scale
     if a.launches:
         agg = launches(a.launches)
         tot = sum(v[1] for v in agg.values())
