@@ -334,7 +334,7 @@ def run_ours(args):
         "stage_entries_per_frame": [round(c / (F * args.steps), 1) for c in counts[:6]],
         "roofline": dominant,
         "roofline_k2_other": other,
-        "roofline_k1": {"kernel": "k_colsum+k_carry+k_band (K1)", "bound": "hbm", "achieved": k1_ach,
+        "roofline_k1": {"kernel": "k_marg+k_carry+k_corner+k_tile (K1)", "bound": "hbm", "achieved": k1_ach,
                         "peak": hbm, "unit": "GB/s", "frac": (k1_ach / hbm) if k1_ach else None,
                         "traffic": tr_k1, "peak_basis": "MEASURED_PEAKS.json hbm_gbs (burst copy)"},
         "kernel_ms_per_step": {k: v[1] / args.steps for k, v in prof.items() if v[0]},

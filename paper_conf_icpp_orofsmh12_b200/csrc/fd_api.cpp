@@ -572,7 +572,11 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     const int nslots = (ngroups > 1 && env_int("FD_PIPE", 1) != 0) ? 2 : 1;
     // K2 split in two kernels (k_stage1: dense first stage, k_deep: batched deeper stages;
     // FD_K2_SPLIT=0 runs the fused k_cascade).  Survivor list sized for the worst case.
-    const bool split = env_int("FD_K2_SPLIT", 1) != 0;
+    // default (FD_K2_SPLIT=1): k_stage1 + k_deep1 (+ k_tail).  FD_K2_WS=1: the warp-specialised
+    // k_ws (stage-1 and deep warp groups in one kernel; measured slower on B200, kept as an
+    // alternative schedule under the same parity tests); FD_K2_SPLIT=0: the fused k_cascade
+    const bool wsk = env_int("FD_K2_WS", 0) != 0;
+    const bool split = !wsk && env_int("FD_K2_SPLIT", 1) != 0;
     const bool deep1 = env_int("FD_K2_DEEP1", 1) != 0;      // k_deep1 (tile per small CTA) or batched k_deep
     // tail queue (k_tail): FD_TAIL=0 keeps every window inside K2; FD_TAIL_N = windows left in a
     // batch at which it hands them over; FD_TAIL_CAP = queue entries (16 B each) per group
@@ -635,6 +639,10 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     P.lane_min = std::max(1, std::min(env_int("FD_LANE_MIN", half + 1), half + 1));
     P.tail_cap = tail_cap;
     P.tail_n = std::max(1, env_int("FD_TAIL_N", 8));
+    // split path: k_stage1 runs stages [0, s0) (FD_S0, default 2); with FD_S1_TAIL=1 it hands the
+    // windows entering stage s0 straight to k_tail (no k_deep launch)
+    P.s0 = split ? std::max(1, env_int("FD_S0", 2)) : (wsk ? std::max(1, env_int("FD_WS_S0", 2)) : 1);
+    P.s1_tail = (split && use_tail && env_int("FD_S1_TAIL", 0) != 0) ? 1 : 0;
     TailParams TP;
     TP.cap = tail_cap;
     TP.step = step;
@@ -703,17 +711,20 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
             cudaError_t e;
             {
                 ProfScope ps(FD_K_CASCADE, gs);
-                e = jit_k2_launch(jit, P, depth, split ? JIT_STAGE1 : JIT_FUSED, gs, &err);
+                e = jit_k2_launch(jit, P, depth, wsk ? JIT_WS : (split ? JIT_STAGE1 : JIT_FUSED), gs, &err);
             }
-            if (e == cudaSuccess && split) {
+            if (e == cudaSuccess && split && !P.s1_tail) {
                 ProfScope ps(FD_K_DEEP, gs);
                 e = jit_k2_launch(jit, P, depth, deep1 ? JIT_DEEP1 : JIT_DEEP, gs, &err);
             }
             if (e != cudaSuccess)
                 return fail(FD_ECUDA, "specialised K2: %s", err.empty() ? cudaGetErrorString(e) : err.c_str());
+        } else if (wsk) {
+            LAUNCH(FD_K_CASCADE, gs, launch_ws(P, depth, step, gs));
         } else if (split) {
             LAUNCH(FD_K_CASCADE, gs, launch_stage1(P, depth, step, gs));
-            LAUNCH(FD_K_DEEP, gs, deep1 ? launch_deep1(P, depth, step, gs) : launch_deep(P, depth, step, gs));
+            if (!P.s1_tail)
+                LAUNCH(FD_K_DEEP, gs, deep1 ? launch_deep1(P, depth, step, gs) : launch_deep(P, depth, step, gs));
         } else {
             LAUNCH(FD_K_CASCADE, gs, launch_cascade(P, depth, step, gr, gs));
         }
@@ -966,7 +977,7 @@ fd_status fd_group(const fd_detection* d_in, int64_t n, double eyes_thresh, int 
     CK(w->group.ensure(group_scratch_bytes(n) + 128));
     long long* d_total = reinterpret_cast<long long*>(w->group.as<char>() + w->group.n - 64);
     {
-        ProfScope ps(FD_K_GROUP, st, 5);
+        ProfScope ps(FD_K_GROUP, st, 7);
         CK(launch_group_plan(d_in, n, w->group.p, st));
         CK(launch_group_run(d_in, n, eyes_thresh, min_neighbors < 1 ? 1 : min_neighbors, w->group.p, d_out, capacity,
                             d_total, st));

@@ -85,10 +85,12 @@ struct TileGeo {
 #endif
 
 // k_stage1 (K2a): one tile's ii + sqii planes and its survivor list (window index, nf bits)
+// (the sqii plane, dead once every nf is taken, holds the stage-2 survivor list)
 template <int STEP>
 struct TileGeoA {
     static constexpr int PBUF = k2_pbuf(STEP);
     static constexpr int NW = k2_tx(STEP) * k2_ty(STEP);
+    static_assert(PBUF * 4 >= NW * 8, "stage-2 survivor list fits in the sqii plane");
     static constexpr size_t OFF_SURV = (size_t)2 * PBUF * 4;
     static constexpr size_t SMEM = OFF_SURV + (size_t)NW * 8;
 };
@@ -106,6 +108,28 @@ struct TileGeoB {
 };
 
 // k_deep1: one ii slot, a pool chunk of CP survivors and its two per-stage lists
+// k_ws (warp-specialised K2): 256 stage-1 threads + WS_DEEP deep-stage threads per CTA.  The
+// stage-1 group streams tiles (ii + sqii planes by TMA, variance, dense stage 1); each tile's
+// ii plane and stage-1 survivors are handed to the deep group in a second buffer, which runs
+// stages 1.. while the stage-1 group moves on.
+#ifndef FD_WS_DEEP_WARPS
+#define FD_WS_DEEP_WARPS 2
+#endif
+constexpr int WS_S1 = 256;
+constexpr int WS_DEEP = 32 * FD_WS_DEEP_WARPS;
+constexpr int WS_THREADS = WS_S1 + WS_DEEP;
+template <int STEP>
+struct TileGeoW {
+    static constexpr int PBUF = k2_pbuf(STEP);
+    static constexpr int NW = k2_tx(STEP) * k2_ty(STEP);
+    static constexpr int CP = NW;                                        // pool: a whole tile
+    static constexpr size_t OFF_B = (size_t)2 * PBUF * 4;                // ii copy for the deep group
+    static constexpr size_t OFF_NF = OFF_B + (size_t)PBUF * 4;
+    static constexpr size_t OFF_LOC = OFF_NF + (size_t)NW * 4;
+    static constexpr size_t OFF_LIST = OFF_LOC + (size_t)NW * 2;
+    static constexpr size_t SMEM = OFF_LIST + (size_t)2 * NW * 2;
+};
+
 #ifndef FD_K2D_CTAS
 #define FD_K2D_CTAS 6
 #endif
@@ -189,6 +213,8 @@ struct alignas(16) CascadeParams {
     unsigned long long* stage_counts;       // n_stages + 1, may be null
     int n_pstages;                          // stages [0, n_pstages) are also in pstages
     int tail_n;                             // a batch with <= tail_n windows left goes to the tail queue
+    int s0;                                 // first stage of the deep kernels (k_stage1 runs [0, s0))
+    int s1_tail;                            // 1: k_stage1 hands its stage-s0 windows to the tail queue (no k_deep)
     uint4* tail_q;                          // tail queue (k_tail.cu), may be null
     unsigned int* tail_count;               // entries appended (may exceed tail_cap: the excess stays in K2)
     int tail_cap;
@@ -204,7 +230,7 @@ struct alignas(16) CascadeParams {
 // Tail queue entry (k_cascade -> k_tail): x = g(16) | level(8) | stage(8), y = wyi(16) | wxi(16)
 // (window indices in the level's step grid), z = nf bits, w = 0.
 constexpr int TAIL_RP = 25;                 // row pitch of a window's ii region staged by k_tail
-constexpr int TAIL_REC_WORDS = 13;          // SoA tail records: nc, theta, left, right, 9 corners
+constexpr int TAIL_REC_WORDS = 4 + MAX_CORNERS;   // SoA tail records: nc, theta, left, right, corners
 struct TailParams {
     const uint4* q;
     const unsigned int* count;
@@ -260,6 +286,7 @@ cudaError_t launch_tail(const TailParams& p, bool depth_mode, cudaStream_t st);
 cudaError_t launch_stage1(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
 cudaError_t launch_deep(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
 cudaError_t launch_deep1(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
+cudaError_t launch_ws(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
 int cascade_grid(bool depth_mode, int step);       // persistent grid size (SMs x resident CTAs)
 size_t cascade_smem(int step);
 cudaError_t launch_keys_to_dets(const unsigned long long* keys, const float* scores, long long n,

@@ -185,10 +185,16 @@ size_t jit_smem_deep(int nb) {
     }
 }
 
+static int jit_ws_deep_warps() {
+    const char* e = std::getenv("FD_WS_DEEP_WARPS");
+    return e ? std::atoi(e) : FD_WS_DEEP_WARPS;
+}
+
 std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages) {
     const int k_end = jit_deep_end(st, n_stages);
     std::string src = std::string(std::getenv("FD_POOL_SEPARATE") ? "#define FD_POOL_SEPARATE 1\n" : "") +
                       "#define FD_K2D_CTAS " + std::to_string(std::getenv("FD_K2D_CTAS") ? std::atoi(std::getenv("FD_K2D_CTAS")) : FD_K2D_CTAS) +
+                      "\n#define FD_WS_DEEP_WARPS " + std::to_string(jit_ws_deep_warps()) +
                       "\n#define FD_K2_CTAS " + std::to_string(jit_ctas()) + "\n#define FD_K2B_NB " +
                       std::to_string(jit_nb_deep()) + "\n#include \"fd_internal.h\"\n" + jit_stage1_source(rec_words, st[0].first, st[0].n) +
                       "#define FD_JIT_STAGE1 1\n";
@@ -201,7 +207,12 @@ static std::string jit_name(int kind, bool depth) {
     if (kind == JIT_FUSED) return "fdk::k_cascade<1, " + d + ">";
     if (kind == JIT_STAGE1) return "fdk::k_stage1<1, " + d + ">";
     if (kind == JIT_DEEP1) return "fdk::k_deep1<1, " + d + ">";
+    if (kind == JIT_WS) return "fdk::k_ws<1, " + d + ">";
     return "fdk::k_deep<1, " + d + ", " + std::to_string(jit_nb_deep()) + ">";
+}
+
+static int jit_kind_threads(int kind) {
+    return kind == JIT_DEEP1 ? K2D_THREADS : (kind == JIT_WS ? WS_S1 + 32 * jit_ws_deep_warps() : k2_threads(JIT_STEP));
 }
 
 static size_t jit_kind_smem(int kind) {
@@ -209,6 +220,7 @@ static size_t jit_kind_smem(int kind) {
         return TileGeo<JIT_STEP>::SMEM + (std::getenv("FD_POOL_SEPARATE") ? (size_t)TileGeo<JIT_STEP>::NW * 10 : 0);
     if (kind == JIT_STAGE1) return TileGeoA<JIT_STEP>::SMEM;
     if (kind == JIT_DEEP1) return TileGeoD<JIT_STEP>::SMEM;
+    if (kind == JIT_WS) return TileGeoW<JIT_STEP>::SMEM;
     return jit_smem_deep(jit_nb_deep());
 }
 
@@ -297,7 +309,7 @@ cudaError_t jit_k2_launch(JitK2* J, const CascadeParams& p, bool depth, int kind
                     e = cudaKernelSetAttributeForDevice(L.kern[k], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem, dev);
                 if (e == cudaSuccess)
                     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, reinterpret_cast<const void*>(L.kern[k]),
-                                                                      k == JIT_DEEP1 ? K2D_THREADS : k2_threads(JIT_STEP), smem);
+                                                                      jit_kind_threads(k), smem);
                 L.grid[k] = sms * (per > 0 ? per : 1);
             }
             if (e != cudaSuccess) {
@@ -314,7 +326,7 @@ cudaError_t jit_k2_launch(JitK2* J, const CascadeParams& p, bool depth, int kind
     const int grid = J->grid[d][kind] < p.total_tiles ? J->grid[d][kind] : p.total_tiles;
     void* args[] = {const_cast<CascadeParams*>(&p)};
     return cudaLaunchKernel(reinterpret_cast<const void*>(J->kern[d][kind]), dim3(grid),
-                            dim3(kind == JIT_DEEP1 ? K2D_THREADS : k2_threads(JIT_STEP)), args, jit_kind_smem(kind), st);
+                            dim3(jit_kind_threads(kind)), args, jit_kind_smem(kind), st);
 }
 
 void jit_k2_free(JitK2* J) { delete J; }    // loaded code stays in the process-wide cache

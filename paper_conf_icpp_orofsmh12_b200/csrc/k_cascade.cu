@@ -80,20 +80,73 @@ struct WinOut {
     }
 };
 
+// One window finished by one warp from stage s on (tail queue full or absent): lane j evaluates
+// stump c0 + j, the leaves are added in stump order (independent shuffles, serial adds -- the
+// definition's fp32 sequence), early exit on the first failed stage.
+template <int STEP, bool DEPTH>
+__device__ __noinline__ void finish_window_warp(const CascadeParams& p, const uint32_t* __restrict__ slots, int b,
+                                                float nfw, int s, int sl, int idx, const WinOut<STEP, DEPTH>& out) {
+    const int lane = threadIdx.x & 31, N = p.n_stages;
+    const GlobalRec grec{p.stumps};
+    int s2 = s;
+    float sum = 0.0f;
+    for (; s2 < N; ++s2) {
+        StageDev sd;
+        if (s2 < p.n_pstages) {
+            sd.first = p.pstages[s2].first;
+            sd.n = p.pstages[s2].n;
+            sd.T = p.pstages[s2].T;
+            sd.mc = p.pstages[s2].mc;
+        } else {
+            sd = p.stages[s2];
+        }
+        if (s2 > s && lane == 0 && p.stage_counts) atomicAdd(p.stage_counts + s2, 1ull);
+        sum = 0.0f;
+        for (int c0 = 0; c0 < sd.n; c0 += 32) {
+            const int j = c0 + lane;
+            float leaf = 0.0f;
+            if (j < sd.n) leaf = eval_stage(slots, b, nfw, grec, sd.first + j, 1, sd.mc);
+            const int m = min(32, sd.n - c0);
+#pragma unroll
+            for (int t2 = 0; t2 < 32; ++t2) {
+                const float v = __shfl_sync(0xffffffffu, leaf, t2);
+                if (t2 < m) sum = __fadd_rn(sum, v);
+            }
+        }
+        if (!(sum >= sd.T)) break;
+    }
+    if (lane == 0) {
+        if (s2 < N)
+            out.reject(sl, idx, s2, sum);
+        else
+            out.emit(sl, idx, sum);
+    }
+}
+
 // Deep stages (1 .. N-1) over a pool of stage-1 survivors held in shared memory: entry e has
-// ploc[e] = slot << 11 | window index (within the slot's tile) and nf pnf[e]; s_cnt[1] = pool size
-// (s_cnt[0] = s_cnt[2] = 0) on entry.  Stage-synchronous: each stage's survivors are
+// ploc[e] = slot << 11 | window index (within the slot's tile) and nf pnf[e]; s_cnt[s0 % 3] = pool
+// size (the other two 0) on entry; the pool enters stage s0.  Stage-synchronous: each stage's survivors are
 // ballot-compacted into the other list and the block synchronises once per stage.  Lane per
 // window (uniform stump records) while windows are plentiful, GL lanes per window (tree sum +
 // certified decision) when fewer than lane_min remain, and once at most tail_n are left they go
 // to the global tail queue (k_tail.cu) -- or, when it is full or absent, are finished here one
 // warp per window.  Ends with a block barrier.
-template <int STEP, bool DEPTH, int CP, int THREADS = k2_threads(STEP)>
-__device__ __forceinline__ void deep_phase(const CascadeParams& p, const uint32_t* __restrict__ slots, const float* pnf,
-                                           const uint16_t* ploc, uint16_t* lists, int* s_cnt, int& s_tpos,
-                                           const WinOut<STEP, DEPTH>& out) {
+// Barrier over the threads running a phase: the whole CTA (BAR = 0) or the named barrier BAR
+// over THREADS threads (a warp group of a warp-specialised kernel).
+template <int BAR, int THREADS>
+__device__ __forceinline__ void phase_sync() {
+    if constexpr (BAR == 0)
+        __syncthreads();
+    else
+        asm volatile("bar.sync %0, %1;" ::"n"(BAR), "n"(THREADS) : "memory");
+}
+
+template <int STEP, bool DEPTH, int CP, int THREADS = k2_threads(STEP), int TID0 = 0, int BAR = 0>
+__device__ __forceinline__ void deep_phase(const CascadeParams& p, int s0, const uint32_t* __restrict__ slots,
+                                           const float* pnf, const uint16_t* ploc, uint16_t* lists, int* s_cnt,
+                                           int& s_tpos, const WinOut<STEP, DEPTH>& out) {
     constexpr int TX = k2_tx(STEP), TW = tile_w(STEP), PBUF = k2_pbuf(STEP);
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int tid = (int)threadIdx.x - TID0, warp = tid >> 5, lane = tid & 31;
     const int lane_min = min(p.lane_min, THREADS / 2 + 1);
     const int N = p.n_stages;
     const ParamRec prec{p};
@@ -108,8 +161,8 @@ __device__ __forceinline__ void deep_phase(const CascadeParams& p, const uint32_
 #ifdef FD_K2_TIMING
     const long long tm2 = clock64();
 #endif
-    int s = 1;
-    // one deep stage; sd is a parameter-bank (uniform) or global stage descriptor.  Stage 1's
+    int s = s0;
+    // one deep stage; sd is a parameter-bank (uniform) or global stage descriptor.  Stage s0's
     // input is the pool itself (entry e), later stages read pool indices from lists.
     auto deep_stage = [&](const StageDev& sd, int n) {
         const uint16_t* lin = lists + (s & 1) * CP;
@@ -127,7 +180,7 @@ __device__ __forceinline__ void deep_phase(const CascadeParams& p, const uint32_
             while (lg < 5 && (n << (lg + 1)) <= THREADS) ++lg;
             const int e = tid >> lg;
             const bool act = e < n;
-            const int pe = act ? (s == 1 ? e : lin[e]) : 0;
+            const int pe = act ? (s == s0 ? e : lin[e]) : 0;
             const int loc = act ? ploc[pe] : 0;
             const int sl = loc >> 11, idx = loc & 2047;
             const int b = sl * PBUF + (idx / TX) * STEP * TW + (idx % TX) * STEP;
@@ -171,7 +224,7 @@ __device__ __forceinline__ void deep_phase(const CascadeParams& p, const uint32_
             int pe = 0, sl = 0, idx = 0;
             float sum = 0.0f;
             if (act) {
-                pe = s == 1 ? e : lin[e];
+                pe = s == s0 ? e : lin[e];
                 const int loc = ploc[pe];
                 sl = loc >> 11;
                 idx = loc & 2047;
@@ -214,10 +267,10 @@ __device__ __forceinline__ void deep_phase(const CascadeParams& p, const uint32_
             // here, one warp per window.
             const uint16_t* lin = lists + (s & 1) * CP;
             if (tid == 0) s_tpos = p.tail_q ? (int)atomicAdd(p.tail_count, (unsigned)n) : p.tail_cap;
-            __syncthreads();
+            phase_sync<BAR, THREADS>();
             const int tpos = s_tpos;
             for (int e = tid; e < n && tpos + e < p.tail_cap; e += THREADS) {
-                const int pe = s == 1 ? e : lin[e];
+                const int pe = s == s0 ? e : lin[e];
                 const int loc = ploc[pe];
                 const int sl = loc >> 11, idx = loc & 2047;
                 uint4 q;
@@ -229,45 +282,11 @@ __device__ __forceinline__ void deep_phase(const CascadeParams& p, const uint32_
             }
             for (int e = warp; e < n; e += THREADS / 32) {
                 if (tpos + e < p.tail_cap) continue;
-                const int pe = s == 1 ? e : lin[e];
+                const int pe = s == s0 ? e : lin[e];
                 const int loc = ploc[pe];
                 const int sl = loc >> 11, idx = loc & 2047;
                 const int b = sl * PBUF + (idx / TX) * STEP * TW + (idx % TX) * STEP;
-                const float nfw = pnf[pe];
-                int s2 = s;
-                float sum = 0.0f;
-                for (; s2 < N; ++s2) {
-                    StageDev sd;
-                    if (s2 < p.n_pstages) {
-                        sd.first = p.pstages[s2].first;
-                        sd.n = p.pstages[s2].n;
-                        sd.T = p.pstages[s2].T;
-                        sd.mc = p.pstages[s2].mc;
-                    } else {
-                        sd = p.stages[s2];
-                    }
-                    if (s2 > s && lane == 0 && p.stage_counts) atomicAdd(p.stage_counts + s2, 1ull);
-                    sum = 0.0f;
-                    for (int c0 = 0; c0 < sd.n; c0 += 32) {
-                        const int j = c0 + lane;
-                        float leaf = 0.0f;
-                        if (j < sd.n) leaf = eval_stage(slots, b, nfw, grec, sd.first + j, 1, sd.mc);
-                        const int m = min(32, sd.n - c0);
-                        // ordered sum of the lanes' leaves: independent shuffles, serial adds
-#pragma unroll
-                        for (int t2 = 0; t2 < 32; ++t2) {
-                            const float v = __shfl_sync(0xffffffffu, leaf, t2);
-                            if (t2 < m) sum = __fadd_rn(sum, v);
-                        }
-                    }
-                    if (!(sum >= sd.T)) break;
-                }
-                if (lane == 0) {
-                    if (s2 < N)
-                        reject(sl, idx, s2, sum);
-                    else
-                        emit(sl, idx, sum);
-                }
+                finish_window_warp<STEP, DEPTH>(p, slots, b, pnf[pe], s, sl, idx, out);
             }
 #ifdef FD_K2_TIMING
             if (tid == 0) {
@@ -290,7 +309,7 @@ __device__ __forceinline__ void deep_phase(const CascadeParams& p, const uint32_
             }
             deep_stage(sd, n);
         }
-        __syncthreads();
+        phase_sync<BAR, THREADS>();
 #ifdef FD_K2_TIMING
         if (tid == 0) {
             const unsigned long long dt = (unsigned long long)(clock64() - ts0);
@@ -308,7 +327,7 @@ __device__ __forceinline__ void deep_phase(const CascadeParams& p, const uint32_
         atomicAdd(&g_k2_timing[84], 1ull);
     }
 #endif
-    __syncthreads();
+    phase_sync<BAR, THREADS>();
 }
 
 // Tile number tn of a frame group -> frame (global), level, window origin, TMA coordinates.
@@ -457,28 +476,31 @@ __global__ void __launch_bounds__(k2_threads(STEP), FD_K2_CTAS) k_cascade(const 
         }
 #endif
         __syncthreads();                          // pool complete
-        deep_phase<STEP, DEPTH, CP>(p, T, pnf, ploc, lists, s_cnt, s_tpos, out);
+        deep_phase<STEP, DEPTH, CP>(p, 1, T, pnf, ploc, lists, s_cnt, s_tpos, out);
     }
 }
 
 // ======================================================================== split K2, kernel a
-// k_stage1: the dense first stage alone, the throughput part of the cascade (c3: 10 of the
-// 11.8 stumps per window, 94.5% of windows stop here).  Persistent over every
-// (frame, level, tile) of the group; per tile one TMA of the ii and sqii planes, variance
-// normalisation (oracle c5), the stage evaluated densely (WPT windows per thread down a column,
-// run-time specialised code for step 1), and the survivors -- window index and nf -- appended
+// k_stage1: the dense first stage and the second stage, the throughput part of the cascade
+// (c3: 10 of the 11.8 stumps per window, 94.5% of windows stop at stage 1, 71% of the rest at
+// stage 2).  Persistent over every (frame, level, tile) of the group; per tile one
+// TMA of the ii and sqii planes, variance normalisation (oracle c5), stage 1 evaluated densely
+// (WPT windows per thread down a column, run-time specialised code for step 1), its survivors
+// ballot-compacted into a shared list, stage 2 evaluated over that list one lane per window
+// (p.s0 == 2), and the survivors of the last stage run here -- window index and nf -- appended
 // to a global list with one atomic per tile; tile_rec[tile] = (offset, count).
 template <int STEP, bool DEPTH>
 __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_constant__ CascadeParams p) {
     using G = TileGeoA<STEP>;
     constexpr int TW = tile_w(STEP), TX = k2_tx(STEP), TY = k2_ty(STEP), WPT = k2_wpt(STEP);
-    constexpr int WARPS_X = TX / 32, PLANE = tile_w(STEP) * tile_h(STEP);
+    constexpr int WARPS_X = TX / 32, PLANE = tile_w(STEP) * tile_h(STEP), THREADS = k2_threads(STEP);
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint32_t* T = reinterpret_cast<uint32_t*>(smem_raw);                     // ii plane
     uint32_t* Q = T + G::PBUF;                                               // sqii plane (mod 2^32)
-    uint2* sv = reinterpret_cast<uint2*>(smem_raw + G::OFF_SURV);            // [NW] survivors
+    uint2* sv = reinterpret_cast<uint2*>(smem_raw + G::OFF_SURV);            // [NW] stage-1 survivors
+    uint2* sv2 = reinterpret_cast<uint2*>(Q);                                // [NW] stage-2 survivors (over sqii)
     __shared__ __align__(8) uint64_t mbar;
-    __shared__ int s_tile, s_cnt, s_off;
+    __shared__ int s_tile, s_c3[3], s_off;
     __shared__ int s_frame[1], s_lvl[1], s_wx0[1], s_wy0[1];
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const StageDev& st0 = p.pstages[0];
@@ -491,9 +513,11 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
     }
     uint32_t phase = 0;
     for (;;) {
-        __syncthreads();                          // buffers, survivor list and s_* free
+        __syncthreads();                          // buffers, survivor lists and s_* free
         if (tid == 0) {
-            s_cnt = 0;
+            s_c3[0] = 0;
+            s_c3[1] = 0;
+            s_c3[2] = 0;
             const int tn = (int)atomicAdd(p.tile_counter, 1u);
             s_tile = tn;
             if (tn < p.total_tiles) {
@@ -523,9 +547,9 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
         float nf[WPT], sm[WPT];
 #pragma unroll
         for (int i = 0; i < WPT; ++i) {
-            const int b = base + i * STEP * TW;
-            const uint32_t S = T[b + WIN * TW + WIN] - T[b + WIN] - T[b + WIN * TW] + T[b];
-            const uint32_t q = Q[b + WIN * TW + WIN] - Q[b + WIN] - Q[b + WIN * TW] + Q[b];
+            const int bo = base + i * STEP * TW;
+            const uint32_t S = T[bo + WIN * TW + WIN] - T[bo + WIN] - T[bo + WIN * TW] + T[bo];
+            const uint32_t q = Q[bo + WIN * TW + WIN] - Q[bo + WIN] - Q[bo + WIN * TW] + Q[bo];
             const long long v = 576LL * (long long)q - (long long)S * (long long)S;
             nf[i] = v > 0 ? __fsqrt_rn(__ll2float_rn(v)) : 1.0f;
             sm[i] = 0.0f;
@@ -552,14 +576,98 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
             const unsigned m = __ballot_sync(0xffffffffu, pass);
             if (m) {
                 int pos = 0;
-                if (lane == 0) pos = atomicAdd(&s_cnt, __popc(m));
+                if (lane == 0) pos = atomicAdd(&s_c3[1], __popc(m));
                 pos = __shfl_sync(0xffffffffu, pos, 0);
                 if (pass) sv[pos + __popc(m & ((1u << lane) - 1u))] = make_uint2((unsigned)idx, (unsigned)__float_as_int(nf[i]));
             }
         }
-        __syncthreads();
+        __syncthreads();                          // stage-1 survivors complete; sqii plane dead
+        // stages [1, s_end) over the survivor lists (sv -> sv2 -> sv ...), one lane per window;
+        // s_c3[s % 3] = windows entering stage s
+        int c = s_c3[1];
+        int s = 1;
+        const int s_end = min(p.s0, p.n_stages);
+        for (; s < s_end && c > 0; ++s) {
+            const uint2* lin = (s & 1) ? sv : sv2;
+            uint2* lout = (s & 1) ? sv2 : sv;
+            StageDev sd;
+            if (s < p.n_pstages) {
+                sd.first = p.pstages[s].first;
+                sd.n = p.pstages[s].n;
+                sd.T = p.pstages[s].T;
+                sd.mc = p.pstages[s].mc;
+            } else {
+                sd = p.stages[s];
+            }
+            const bool last = s == p.n_stages - 1;
+            if (tid == 0) {
+                s_c3[(s + 2) % 3] = 0;
+                if (p.stage_counts) atomicAdd(p.stage_counts + s, (unsigned long long)c);
+            }
+            for (int e0 = warp * 32; e0 < c; e0 += THREADS) {
+                const int e = e0 + lane;
+                const bool act = e < c;
+                uint2 v = make_uint2(0u, 0u);
+                float sum = 0.0f;
+                if (act) {
+                    v = lin[e];
+                    const int idx = (int)v.x;
+                    const int bo = (idx / TX) * STEP * TW + (idx % TX) * STEP;
+                    const float nfw = __int_as_float((int)v.y);
+#if FD_JIT_DEEP > 1
+                    if (s < FD_JIT_DEEP)
+                        sum = jit_deep(s, T + bo, nfw);
+                    else
+#endif
+                        sum = sd.first + sd.n <= p.n_pstumps ? eval_stage(T, bo, nfw, prec, sd.first, sd.n, sd.mc)
+                                                             : eval_stage(T, bo, nfw, grec, sd.first, sd.n, sd.mc);
+                }
+                const bool pass = act && (sum >= sd.T);
+                if (act && !pass) out.reject(0, (int)v.x, s, sum);
+                if (last) {
+                    if (pass) out.emit(0, (int)v.x, sum);
+                    continue;
+                }
+                const unsigned m = __ballot_sync(0xffffffffu, pass);
+                if (m) {
+                    int pos = 0;
+                    if (lane == 0) pos = atomicAdd(&s_c3[(s + 1) % 3], __popc(m));
+                    pos = __shfl_sync(0xffffffffu, pos, 0);
+                    if (pass) lout[pos + __popc(m & ((1u << lane) - 1u))] = v;
+                }
+            }
+            __syncthreads();
+            c = last ? 0 : s_c3[(s + 1) % 3];
+        }
+        const uint2* lst = (s & 1) ? sv : sv2;    // the c windows entering stage s
+        if (p.s1_tail && c > 0) {
+            // hand the windows entering stage s to the tail queue (k_tail finishes them, one warp
+            // per window); what does not fit is finished here, one warp per window
+            if (tid == 0) {
+                if (p.stage_counts) atomicAdd(p.stage_counts + s, (unsigned long long)c);
+                s_off = (int)atomicAdd(p.tail_count, (unsigned)c);
+                p.tile_rec[tn] = make_uint2(0u, 0u);
+                if (p.stage_counts)
+                    atomicAdd(p.stage_counts, (unsigned long long)min(TX, nx - wx0) * (unsigned long long)min(TY, ny - wy0));
+            }
+            __syncthreads();
+            const int tpos = s_off;
+            const unsigned fl = ((unsigned)(s_frame[0] - p.frame_base) << 16) | ((unsigned)k << 8) | (unsigned)s;
+            for (int e = tid; e < c && tpos + e < p.tail_cap; e += THREADS) {
+                const uint2 v = lst[e];
+                const int idx = (int)v.x;
+                p.tail_q[tpos + e] = make_uint4(fl, ((unsigned)(wy0 + idx / TX) << 16) | (unsigned)(wx0 + idx % TX), v.y, 0u);
+            }
+            for (int e = warp; e < c; e += THREADS / 32) {
+                if (tpos + e < p.tail_cap) continue;
+                const uint2 v = lst[e];
+                const int idx = (int)v.x;
+                finish_window_warp<STEP, DEPTH>(p, T, (idx / TX) * STEP * TW + (idx % TX) * STEP,
+                                                __int_as_float((int)v.y), s, 0, idx, out);
+            }
+            continue;
+        }
         if (tid == 0) {
-            const int c = s_cnt;
             const unsigned off = c ? atomicAdd(p.surv_count, (unsigned)c) : 0u;
             p.tile_rec[tn] = make_uint2(off, (unsigned)c);
             s_off = (int)off;
@@ -567,8 +675,8 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
                 atomicAdd(p.stage_counts, (unsigned long long)min(TX, nx - wx0) * (unsigned long long)min(TY, ny - wy0));
         }
         __syncthreads();
-        const int c = s_cnt, off = s_off;
-        for (int e = tid; e < c; e += k2_threads(STEP)) p.surv[off + e] = sv[e];
+        const int off = s_off;
+        for (int e = tid; e < c; e += THREADS) p.surv[off + e] = lst[e];
     }
 }
 
@@ -628,7 +736,7 @@ __global__ void __launch_bounds__(k2_threads(STEP), k2b_min_ctas(NB)) k_deep(con
                 s_tile = tn;
                 s_stop = 0;
                 if (tn < p.total_tiles) {
-                    if (s_cnt[1] + (int)tr.y > CP) {
+                    if (s_cnt[p.s0 % 3] + (int)tr.y > CP) {
                         s_carry = tn;             // does not fit: first tile of the next batch
                         s_stop = 1;
                     } else {
@@ -642,8 +750,8 @@ __global__ void __launch_bounds__(k2_threads(STEP), k2b_min_ctas(NB)) k_deep(con
                         tma_load_4d(slots + nb * PBUF, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar[nb]);
                         s_off = (int)tr.x;
                         s_n = (int)tr.y;
-                        s_base = s_cnt[1];
-                        s_cnt[1] += (int)tr.y;
+                        s_base = s_cnt[p.s0 % 3];
+                        s_cnt[p.s0 % 3] += (int)tr.y;
                     }
                 }
             }
@@ -673,10 +781,10 @@ __global__ void __launch_bounds__(k2_threads(STEP), k2b_min_ctas(NB)) k_deep(con
             atomicAdd(&g_k2_timing[90], (unsigned long long)(tf1 - tf0));
             atomicAdd(&g_k2_timing[91], (unsigned long long)(clock64() - tf1));
             atomicAdd(&g_k2_timing[92], (unsigned long long)nb);
-            atomicAdd(&g_k2_timing[93], (unsigned long long)s_cnt[1]);
+            atomicAdd(&g_k2_timing[93], (unsigned long long)s_cnt[p.s0 % 3]);
         }
 #endif
-        deep_phase<STEP, DEPTH, CP>(p, slots, pnf, ploc, lists, s_cnt, s_tpos, out);
+        deep_phase<STEP, DEPTH, CP>(p, p.s0, slots, pnf, ploc, lists, s_cnt, s_tpos, out);
     }
 }
 
@@ -741,15 +849,247 @@ __global__ void __launch_bounds__(K2D_THREADS, FD_K2D_CTAS) k_deep1(const __grid
             }
             if (tid == 0) {
                 s_cnt[0] = 0;
-                s_cnt[1] = m;
+                s_cnt[1] = 0;
                 s_cnt[2] = 0;
+                s_cnt[p.s0 % 3] = m;
             }
             if (c0 == 0) {
                 mbar_wait(&mbar, phase);
                 phase ^= 1;
             }
             __syncthreads();
-            deep_phase<STEP, DEPTH, CP, K2D_THREADS>(p, slot, pnf, ploc, lists, s_cnt, s_tpos, out);
+            deep_phase<STEP, DEPTH, CP, K2D_THREADS>(p, p.s0, slot, pnf, ploc, lists, s_cnt, s_tpos, out);
+        }
+    }
+}
+
+
+// ======================================================================== warp-specialised K2
+// k_ws: one persistent CTA = a stage-1 warp group (WS_S1 threads) + a deep warp group (WS_DEEP
+// threads), 2 CTAs per SM.  The stage-1 group claims tiles, TMAs their ii + sqii planes, computes
+// the variance normalisation and the dense first stage exactly as k_stage1, then (once the deep
+// group has released the hand-off buffer) ballot-compacts the survivors into the pool and copies
+// the ii plane into the hand-off buffer B; the deep group runs deep_phase (stages 1..N-1,
+// named barrier 2) over the pool while the stage-1 group already streams the next tile.  The
+// hand-off is a one-slot pipeline on two mbarriers: FULL (every stage-1 thread arrives after
+// its pool / B writes) and EMPTY (every deep thread arrives when done with B and the pool).
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+template <int STEP, bool DEPTH>
+__global__ void __launch_bounds__(WS_THREADS, 2) k_ws(const __grid_constant__ CascadeParams p) {
+    using G = TileGeoW<STEP>;
+    constexpr int TW = tile_w(STEP), TX = k2_tx(STEP), TY = k2_ty(STEP), WPT = k2_wpt(STEP), CP = G::CP;
+    constexpr int WARPS_X = TX / 32, PLANE = tile_w(STEP) * tile_h(STEP);
+    static_assert(k2_threads(STEP) == WS_S1, "stage-1 group = the k_stage1 thread layout");
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    uint32_t* T = reinterpret_cast<uint32_t*>(smem_raw);                     // ii plane (TMA)
+    uint32_t* Q = T + G::PBUF;                                               // sqii plane (TMA)
+    uint32_t* B = reinterpret_cast<uint32_t*>(smem_raw + G::OFF_B);          // ii plane of the deep group
+    float* pnf = reinterpret_cast<float*>(smem_raw + G::OFF_NF);
+    uint16_t* ploc = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LOC);
+    uint16_t* lists = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LIST);
+    __shared__ __align__(8) uint64_t mbar_tma, mbar_full, mbar_empty;
+    __shared__ int s_tile, s_pc, s_l1;
+    __shared__ int s_frame[1], s_lvl[1], s_wx0[1], s_wy0[1];                // stage-1 group's tile
+    __shared__ int d_frame[1], d_lvl[1], d_wx0[1], d_wy0[1];                // deep group's tile
+    __shared__ int d_n, d_s0, d_stop, d_cnt[3], d_tpos;
+    const int tid = threadIdx.x;
+    if (tid == 0) {
+        mbar_init(&mbar_tma, 1);
+        mbar_init(&mbar_full, WS_S1);
+        mbar_init(&mbar_empty, WS_DEEP);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (tid < WS_S1) {
+        // ------------------------------------------------------------ stage-1 group
+        const int warp = tid >> 5, lane = tid & 31;
+        const StageDev& st0 = p.pstages[0];
+        const ParamRec prec{p};
+        const GlobalRec grec{p.stumps};
+        const WinOut<STEP, DEPTH> out{p, s_frame, s_lvl, s_wx0, s_wy0};
+        uint32_t ph_tma = 0, ph_empty = 0;
+        bool first = true;
+        for (;;) {
+            phase_sync<1, WS_S1>();               // planes, s_* free
+            if (tid == 0) {
+                s_pc = 0;
+                const int tn = (int)atomicAdd(p.tile_counter, 1u);
+                s_tile = tn;
+                if (tn < p.total_tiles) {
+                    const TileAt t = tile_at<STEP>(p, tn);
+                    s_frame[0] = p.frame_base + t.g;
+                    s_lvl[0] = t.k;
+                    s_wx0[0] = t.wx0;
+                    s_wy0[0] = t.wy0;
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    mbar_expect_tx(&mbar_tma, 2 * PLANE * 4);
+                    tma_load_4d(T, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar_tma);
+                    tma_load_4d(Q, p.tmaps + t.k, t.x, t.y, 1, t.g, &mbar_tma);
+                }
+            }
+            phase_sync<1, WS_S1>();
+            if (s_tile >= p.total_tiles) break;
+            mbar_wait(&mbar_tma, ph_tma);
+            ph_tma ^= 1;
+            const int k = s_lvl[0];
+            const int nx = __ldg(&p.lv[k].nx), ny = __ldg(&p.lv[k].ny);
+            const int wx0 = s_wx0[0], wy0 = s_wy0[0];
+            const int lx = lane + 32 * (warp % WARPS_X);
+            const int ly0 = (warp / WARPS_X) * WPT;
+            const int base = ly0 * STEP * TW + lx * STEP;
+            const bool colok = wx0 + lx < nx;
+            float nf[WPT], sm[WPT];
+#pragma unroll
+            for (int i = 0; i < WPT; ++i) {
+                const int bo = base + i * STEP * TW;
+                const uint32_t S = T[bo + WIN * TW + WIN] - T[bo + WIN] - T[bo + WIN * TW] + T[bo];
+                const uint32_t q = Q[bo + WIN * TW + WIN] - Q[bo + WIN] - Q[bo + WIN * TW] + Q[bo];
+                const long long v = 576LL * (long long)q - (long long)S * (long long)S;
+                nf[i] = v > 0 ? __fsqrt_rn(__ll2float_rn(v)) : 1.0f;
+                sm[i] = 0.0f;
+            }
+#ifdef FD_JIT_STAGE1
+            jit_stage1(T + base, nf, sm);
+#else
+            if (st0.first + st0.n <= p.n_pstumps)
+                dense_stage<WPT, STEP * TW>(T, base, nf, sm, prec, st0.first, st0.n);
+            else
+                dense_stage<WPT, STEP * TW>(T, base, nf, sm, grec, st0.first, st0.n);
+#endif
+            // stage-1 survivors: straight into the pool (s0 == 1) or, when this group also runs
+            // stage 2 (s0 == 2), into a list over the sqii plane (dead once every nf is taken)
+            const bool s2here = p.s0 >= 2 && p.n_stages >= 2;
+            uint2* l1 = reinterpret_cast<uint2*>(Q);
+            if (s2here) {
+                if (tid == 0) s_l1 = 0;
+                phase_sync<1, WS_S1>();           // every sqii read done, s_l1 zeroed
+            }
+            // the hand-off buffer and the pool are free once the deep group has finished the
+            // previous tile
+            if (!first && !s2here) {
+                mbar_wait(&mbar_empty, ph_empty);
+                ph_empty ^= 1;
+            }
+#pragma unroll
+            for (int i = 0; i < WPT; ++i) {
+                const int wy = wy0 + ly0 + i;
+                const bool valid = colok && wy < ny;
+                const bool pass = valid && (sm[i] >= st0.T);
+                const int idx = (ly0 + i) * TX + lx;
+                if (DEPTH && valid && !pass) out.reject(0, idx, 0, sm[i]);
+                if (p.n_stages == 1) {
+                    if (pass) out.emit(0, idx, sm[i]);
+                    continue;
+                }
+                const unsigned m = __ballot_sync(0xffffffffu, pass);
+                if (m) {
+                    int pos = 0;
+                    if (lane == 0) pos = atomicAdd(s2here ? &s_l1 : &s_pc, __popc(m));
+                    pos = __shfl_sync(0xffffffffu, pos, 0);
+                    if (pass) {
+                        const int at = pos + __popc(m & ((1u << lane) - 1u));
+                        if (s2here) {
+                            l1[at] = make_uint2((unsigned)idx, (unsigned)__float_as_int(nf[i]));
+                        } else {
+                            ploc[at] = (uint16_t)idx;
+                            pnf[at] = nf[i];
+                        }
+                    }
+                }
+            }
+            if (s2here) {
+                phase_sync<1, WS_S1>();           // stage-1 survivor list complete
+                if (!first) {
+                    mbar_wait(&mbar_empty, ph_empty);
+                    ph_empty ^= 1;
+                }
+                // stage 2 over the list, one lane per window; survivors into the pool
+                const int c = s_l1;
+                const StageDev& sd = p.pstages[1];
+                const bool last = p.n_stages == 2;
+                if (tid == 0 && p.stage_counts && c) atomicAdd(p.stage_counts + 1, (unsigned long long)c);
+                for (int e0 = warp * 32; e0 < c; e0 += WS_S1) {
+                    const int e = e0 + lane;
+                    const bool act = e < c;
+                    uint2 v = make_uint2(0u, 0u);
+                    float sum = 0.0f;
+                    if (act) {
+                        v = l1[e];
+                        const int idx = (int)v.x;
+                        const int bo = (idx / TX) * STEP * TW + (idx % TX) * STEP;
+                        const float nfw = __int_as_float((int)v.y);
+#if FD_JIT_DEEP > 1
+                        sum = jit_deep(1, T + bo, nfw);
+#else
+                        sum = sd.first + sd.n <= p.n_pstumps ? eval_stage(T, bo, nfw, prec, sd.first, sd.n, sd.mc)
+                                                             : eval_stage(T, bo, nfw, grec, sd.first, sd.n, sd.mc);
+#endif
+                    }
+                    const bool pass = act && (sum >= sd.T);
+                    if (act && !pass) out.reject(0, (int)v.x, 1, sum);
+                    if (last) {
+                        if (pass) out.emit(0, (int)v.x, sum);
+                        continue;
+                    }
+                    const unsigned m = __ballot_sync(0xffffffffu, pass);
+                    if (m) {
+                        int pos = 0;
+                        if (lane == 0) pos = atomicAdd(&s_pc, __popc(m));
+                        pos = __shfl_sync(0xffffffffu, pos, 0);
+                        if (pass) {
+                            const int at = pos + __popc(m & ((1u << lane) - 1u));
+                            ploc[at] = (uint16_t)v.x;
+                            pnf[at] = __int_as_float((int)v.y);
+                        }
+                    }
+                }
+            }
+            first = false;
+            {   // ii plane -> hand-off buffer (uint4 copies)
+                const uint4* src = reinterpret_cast<const uint4*>(T);
+                uint4* dst = reinterpret_cast<uint4*>(B);
+                for (int i = tid; i < G::PBUF / 4; i += WS_S1) dst[i] = src[i];
+            }
+            phase_sync<1, WS_S1>();               // pool, B and s_pc complete
+            if (tid == 0) {
+                d_n = p.n_stages <= (p.s0 >= 2 ? 2 : 1) ? 0 : s_pc;
+                d_s0 = p.s0 >= 2 ? 2 : 1;
+                d_frame[0] = s_frame[0];
+                d_lvl[0] = k;
+                d_wx0[0] = wx0;
+                d_wy0[0] = wy0;
+                d_stop = 0;
+                if (p.stage_counts)
+                    atomicAdd(p.stage_counts, (unsigned long long)min(TX, nx - wx0) * (unsigned long long)min(TY, ny - wy0));
+            }
+            mbar_arrive(&mbar_full);
+        }
+        // no more tiles: stop the deep group once it is idle
+        if (!first) mbar_wait(&mbar_empty, ph_empty);
+        if (tid == 0) d_stop = 1;
+        mbar_arrive(&mbar_full);
+    } else {
+        // ------------------------------------------------------------ deep group
+        const int dt = tid - WS_S1;
+        const WinOut<STEP, DEPTH> out{p, d_frame, d_lvl, d_wx0, d_wy0};
+        uint32_t ph_full = 0;
+        for (;;) {
+            mbar_wait(&mbar_full, ph_full);
+            ph_full ^= 1;
+            if (d_stop) break;
+            const int s0 = d_s0;
+            if (dt == 0) {
+                d_cnt[0] = 0;
+                d_cnt[1] = 0;
+                d_cnt[2] = 0;
+                d_cnt[s0 % 3] = d_n;
+            }
+            phase_sync<2, WS_DEEP>();
+            deep_phase<STEP, DEPTH, CP, WS_DEEP, WS_S1, 2>(p, s0, B, pnf, ploc, lists, d_cnt, d_tpos, out);
+            mbar_arrive(&mbar_empty);
         }
     }
 }
@@ -878,6 +1218,33 @@ static cudaError_t launch_deep1_t(const CascadeParams& p, cudaStream_t st) {
     }
     k_deep1<STEP, DEPTH><<<grid < p.total_tiles ? grid : p.total_tiles, K2D_THREADS, smem, st>>>(p);
     return cudaGetLastError();
+}
+
+template <int STEP, bool DEPTH>
+static cudaError_t launch_ws_t(const CascadeParams& p, cudaStream_t st) {
+    static int grid = 0;
+    const size_t smem = TileGeoW<STEP>::SMEM;
+    cudaError_t e = cudaFuncSetAttribute(k_ws<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    if (!grid) {
+        int dev = 0, sms = 0, per = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_ws<STEP, DEPTH>, WS_THREADS, smem);
+        grid = sms * (per > 0 ? per : 1);
+    }
+    k_ws<STEP, DEPTH><<<grid < p.total_tiles ? grid : p.total_tiles, WS_THREADS, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_ws(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
+    switch (step) {
+        case 1: return depth ? launch_ws_t<1, true>(p, st) : launch_ws_t<1, false>(p, st);
+        case 2: return depth ? launch_ws_t<2, true>(p, st) : launch_ws_t<2, false>(p, st);
+        case 3: return depth ? launch_ws_t<3, true>(p, st) : launch_ws_t<3, false>(p, st);
+        case 4: return depth ? launch_ws_t<4, true>(p, st) : launch_ws_t<4, false>(p, st);
+        default: return cudaErrorInvalidValue;
+    }
 }
 
 cudaError_t launch_deep1(const CascadeParams& p, bool depth, int step, cudaStream_t st) {

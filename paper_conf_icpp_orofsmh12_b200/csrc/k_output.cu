@@ -133,13 +133,19 @@ constexpr int GT = 256;
 // the same whenever it is below the threshold, and the loop stops otherwise); a pair whose
 // left- or right-eye coordinate gap alone forces S_eyes >= thresh skips the square roots.
 constexpr int GWARPS = GT / 32;
-constexpr int GROOTS = 1024;            // components tracked per frame (beyond: one component)
+constexpr int GROOTS = 512;             // components tracked per frame (beyond: one component)
+constexpr int GPS = 2048;               // frames with <= GPS detections keep union-find in shared memory
+constexpr int GBOX = 256;               // ... and, with <= GBOX components, their eye boxes too
 
+// find with path halving: x's parent becomes its grandparent (an ancestor, so concurrent finds and
+// root links stay correct); links only ever change a root's parent (uf_union's CAS)
 __device__ __forceinline__ int uf_find(int* parent, int x) {
     for (;;) {
         const int q = *reinterpret_cast<volatile int*>(parent + x);
         if (q == x) return x;
-        x = q;
+        const int qq = *reinterpret_cast<volatile int*>(parent + q);
+        if (qq != q) *reinterpret_cast<volatile int*>(parent + x) = qq;
+        x = qq;
     }
 }
 __device__ __forceinline__ void uf_union(int* parent, int a, int b) {
@@ -170,15 +176,20 @@ __device__ __forceinline__ bool independent(double gl, double gr, double da, dou
     return __dsub_rn(__dadd_rn(gl, gr), 4e-6) > __dmul_rn(__dmul_rn(thresh, fmin(da, db)), 1.000001);
 }
 
-__global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ in, long long n,
-                                              const long long* __restrict__ seg_start, const int* __restrict__ n_seg_p,
-                                              double thresh, int min_neighbors, GroupScratch gs, int* seg_next,
-                                              int* seg_count, fd_detection* __restrict__ tmp) {
-    __shared__ int s_seg, s_changed, s_nroots, s_q;
+// K4a: one CTA per frame: cluster state, independent components (union-find over the eye-box
+// bound), member lists; every component with >= 2 members is appended to the global work list
+// comp[] = (frame start a0, list offset, member count).
+__global__ void __launch_bounds__(GT) k_group_comp(const fd_detection* __restrict__ in, long long n,
+                                                   const long long* __restrict__ seg_start,
+                                                   const int* __restrict__ n_seg_p, double thresh, GroupScratch gs,
+                                                   int* seg_next, longlong2* comp, int* n_comp) {
+    __shared__ int s_seg, s_changed, s_nroots, s_cbase;
     __shared__ int s_roots[GROOTS], s_off[GROOTS], s_cnt[GROOTS];
+    __shared__ int s_par[GPS], s_ord[GPS];
+    __shared__ unsigned long long s_box[GBOX * 9];
+    extern __shared__ float4 s_key[];       // [GPS] dynamic: coarse eye keys
     const int n_seg = *n_seg_p;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const double tguard = thresh * (1.0 + 0x1p-40);
     for (;;) {
         __syncthreads();
         if (tid == 0) s_seg = atomicAdd(seg_next, 1);
@@ -197,13 +208,31 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
             g.cnt[i] = 1;
             g.smax[i] = d.score;
             g.eyes[i] = eyes_of((double)d.x, (double)d.y, (double)d.w, (double)d.h);
-            g.parent[i] = i;
+        }
+        const bool fast = m <= GPS;
+        int* par = fast ? s_par : g.parent;
+        for (int i = tid; i < m; i += GT) {
+            par[i] = i;
+            if (fast) {
+                const Eyes e = g.eyes[i];
+                s_key[i] = make_float4((float)e.lex, (float)e.ley, (float)e.rex, (float)e.d);
+            }
         }
         __syncthreads();
-        // ---- components: singleton pairs first
+        __syncthreads();
+        // ---- components: singleton pairs first.  A conservative float pre-test on shared-memory
+        // keys (lex, ley, rex, d; 1e-2 px slack covers their rounding) skips far pairs; the exact
+        // double test follows for the rest
+        const float tf = (float)thresh * 1.0001f;
         for (int i = tid; i < m; i += GT) {
+            const float4 ki = fast ? s_key[i] : make_float4(0.f, 0.f, 0.f, 0.f);
             const Eyes ei = g.eyes[i];
             for (int j = i + 1; j < m; ++j) {
+                if (fast) {
+                    const float4 kj = s_key[j];
+                    const float lf = __fadd_ru(__fmul_ru(tf, fminf(ki.w, kj.w)), 1e-2f);
+                    if (fabsf(ki.x - kj.x) > lf || fabsf(ki.y - kj.y) > lf || fabsf(ki.z - kj.z) > lf) continue;
+                }
                 const Eyes ej = g.eyes[j];
                 const double lim = __dmul_rn(__dmul_rn(thresh, fmin(ei.d, ej.d)), 1.000001) + 4e-6;
                 if (fabs(ei.lex - ej.lex) > lim || fabs(ei.ley - ej.ley) > lim || fabs(ei.rex - ej.rex) > lim ||
@@ -211,7 +240,7 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
                     continue;
                 const double gl = box_gap(ei.lex, ei.lex, ei.ley, ei.ley, ej.lex, ej.lex, ej.ley, ej.ley);
                 const double gr = box_gap(ei.rex, ei.rex, ei.rey, ei.rey, ej.rex, ej.rex, ej.rey, ej.rey);
-                if (!independent(gl, gr, ei.d, ej.d, thresh)) uf_union(g.parent, i, j);
+                if (!independent(gl, gr, ei.d, ej.d, thresh)) uf_union(par, i, j);
             }
         }
         // ---- then component boxes, until every pair of components is independent
@@ -222,28 +251,39 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
                 s_changed = 0;
                 s_nroots = 0;
             }
-            for (int i = tid; i < m; i += GT) g.parent[i] = uf_find(g.parent, i);
+            for (int i = tid; i < m; i += GT) par[i] = uf_find(par, i);
             __syncthreads();
             for (int i = tid; i < m; i += GT) {
-                if (g.parent[i] != i) continue;
+                if (par[i] != i) continue;
                 const int r = atomicAdd(&s_nroots, 1);
                 if (r < GROOTS) s_roots[r] = i;
-                unsigned long long* bx = g.box + 9 * i;
+                if (fast) s_ord[i] = r;
+                // both candidate boxes (which one is used depends on the final component count)
+                unsigned long long* bxs[2] = {g.box + 9 * i, fast && r < GBOX ? s_box + 9 * r : g.box + 9 * i};
 #pragma unroll
-                for (int c = 0; c < 4; ++c) {
-                    bx[2 * c] = dbits(CUDART_INF);
-                    bx[2 * c + 1] = 0ull;
+                for (int t = 0; t < 2; ++t) {
+                    unsigned long long* bx = bxs[t];
+#pragma unroll
+                    for (int c = 0; c < 4; ++c) {
+                        bx[2 * c] = dbits(CUDART_INF);
+                        bx[2 * c + 1] = 0ull;
+                    }
+                    bx[8] = 0ull;
                 }
-                bx[8] = 0ull;
             }
             __syncthreads();
             if (s_nroots > GROOTS) {               // too many components to track: one for the frame
                 whole = true;
                 break;
             }
+            // eye boxes: shared-memory atomics when the frame and its component count are small
+            const bool sbox = fast && s_nroots <= GBOX;
+            auto box_of = [&](int root) -> unsigned long long* {
+                return sbox ? s_box + 9 * s_ord[root] : g.box + 9 * root;
+            };
             for (int i = tid; i < m; i += GT) {
                 const Eyes e = g.eyes[i];
-                unsigned long long* bx = g.box + 9 * g.parent[i];
+                unsigned long long* bx = box_of(par[i]);
                 atomicMin(bx + 0, dbits(e.lex)); atomicMax(bx + 1, dbits(e.lex));
                 atomicMin(bx + 2, dbits(e.ley)); atomicMax(bx + 3, dbits(e.ley));
                 atomicMin(bx + 4, dbits(e.rex)); atomicMax(bx + 5, dbits(e.rex));
@@ -260,14 +300,14 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
                 while ((long long)(u + 2) * (u + 1) / 2 <= t) ++u;
                 const int v = (int)(t - (long long)(u + 1) * u / 2);
                 const int ra = s_roots[u + 1], rb = s_roots[v];
-                const unsigned long long* A = g.box + 9 * ra;
-                const unsigned long long* B = g.box + 9 * rb;
+                const unsigned long long* A = box_of(ra);
+                const unsigned long long* B = box_of(rb);
                 const double gl = box_gap(bitsd(A[0]), bitsd(A[1]), bitsd(A[2]), bitsd(A[3]), bitsd(B[0]), bitsd(B[1]),
                                           bitsd(B[2]), bitsd(B[3]));
                 const double gr = box_gap(bitsd(A[4]), bitsd(A[5]), bitsd(A[6]), bitsd(A[7]), bitsd(B[4]), bitsd(B[5]),
                                           bitsd(B[6]), bitsd(B[7]));
                 if (!independent(gl, gr, bitsd(A[8]), bitsd(B[8]), thresh)) {
-                    uf_union(g.parent, ra, rb);
+                    uf_union(par, ra, rb);
                     s_changed = 1;
                 }
             }
@@ -288,7 +328,7 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
                 int c = 0;
                 for (int k0 = 0; k0 < m; k0 += 32) {
                     const int i = k0 + lane;
-                    c += __popc(__ballot_sync(0xffffffffu, i < m && g.parent[i] == root));
+                    c += __popc(__ballot_sync(0xffffffffu, i < m && par[i] == root));
                 }
                 if (lane == 0) s_cnt[r] = c;
             }
@@ -306,7 +346,7 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
                 int c = s_off[r];
                 for (int k0 = 0; k0 < m; k0 += 32) {
                     const int i = k0 + lane;
-                    const bool in_r = i < m && g.parent[i] == root;
+                    const bool in_r = i < m && par[i] == root;
                     const unsigned bm = __ballot_sync(0xffffffffu, in_r);
                     if (in_r) g.list[c + __popc(bm & ((1u << lane) - 1u))] = i;
                     c += __popc(bm);
@@ -314,11 +354,34 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
             }
         }
         __syncthreads();
-        // ---- greedy loop per component, one warp each
-        for (int r = warp; r < K; r += GWARPS) {
-            const int* L = g.list + s_off[r];
-            const int mc = s_cnt[r];
-            if (mc < 2) continue;
+        __syncthreads();
+        // ---- components with >= 2 members -> global work list (one warp each in K4b)
+        if (tid == 0) {
+            int c = 0;
+            for (int r = 0; r < K; ++r) c += s_cnt[r] >= 2;
+            s_cbase = c ? atomicAdd(n_comp, c) : 0;
+            for (int r = 0, q = s_cbase; r < K; ++r)
+                if (s_cnt[r] >= 2) comp[q++] = make_longlong2(a0, ((long long)s_off[r] << 32) | (unsigned)s_cnt[r]);
+        }
+    }
+}
+
+// K4b: the greedy loop of one component per warp, over the components of every frame (the
+// merges of different components commute; inside a component the definition's order is kept).
+__global__ void __launch_bounds__(GT) k_group_greedy(const longlong2* __restrict__ comp, const int* __restrict__ n_comp,
+                                                     double thresh, GroupScratch gs) {
+    const int lane = threadIdx.x & 31;
+    const double tguard = thresh * (1.0 + 0x1p-40);
+    const int nc = *n_comp;
+    for (int r = (blockIdx.x * GT + threadIdx.x) >> 5; r < nc; r += (gridDim.x * GT) >> 5) {
+        const longlong2 cr = comp[r];
+        const long long a0 = cr.x;
+        GroupScratch g = gs;
+        g.sx += a0; g.sy += a0; g.sw += a0; g.sh += a0; g.cnt += a0; g.smax += a0;
+        g.nn += a0; g.nnd += a0; g.eyes += a0; g.parent += a0; g.list += a0; g.box += 9 * a0;
+        const int* L = g.list + (int)(cr.y >> 32);
+        const int mc = (int)(cr.y & 0xffffffffLL);
+        {
             auto dist = [&](const Eyes& a, int j) -> double {
                 const Eyes b = g.eyes[j];
                 const double lim = tguard * (a.d < b.d ? a.d : b.d);
@@ -432,9 +495,23 @@ __global__ void __launch_bounds__(GT) k_group(const fd_detection* __restrict__ i
                 }
             }
         }
-        __syncthreads();
-        // ---- emit clusters in first-member order (warp 0, ballot compaction over the frame)
-        if (warp == 0) {
+    }
+}
+
+// K4c: one warp per frame: clusters with >= min_neighbors members, in first-member order.
+__global__ void __launch_bounds__(GT) k_group_emit(const fd_detection* __restrict__ in, long long n,
+                                                   const long long* __restrict__ seg_start,
+                                                   const int* __restrict__ n_seg_p, int min_neighbors, GroupScratch gs,
+                                                   int* seg_count, fd_detection* __restrict__ tmp) {
+    const int lane = threadIdx.x & 31;
+    const int n_seg = *n_seg_p;
+    for (int sgi = (blockIdx.x * GT + threadIdx.x) >> 5; sgi < n_seg; sgi += (gridDim.x * GT) >> 5) {
+        const long long a0 = seg_start[sgi];
+        const long long a1 = sgi + 1 < n_seg ? seg_start[sgi + 1] : n;
+        const int m = (int)(a1 - a0);
+        GroupScratch g = gs;
+        g.sx += a0; g.sy += a0; g.sw += a0; g.sh += a0; g.cnt += a0; g.smax += a0;
+        {
             int q = 0;
             for (int k0 = 0; k0 < m; k0 += 32) {
                 const int i = k0 + lane;
@@ -518,7 +595,8 @@ struct GroupLayout {
     int* seg_count;
     long long* seg_off;
     fd_detection* tmp;
-    int* misc;                 // [0] n_seg, [1] seg_next
+    longlong2* comp;           // component work list: (frame start, list offset << 32 | members)
+    int* misc;                 // [0] n_seg, [1] seg_next, [2] components
     GroupLayout(void* scratch, long long n) {
         char* p = reinterpret_cast<char*>(scratch);
         auto take = [&](size_t bytes) {
@@ -543,13 +621,15 @@ struct GroupLayout {
         seg_count = reinterpret_cast<int*>(take(a * 4));
         seg_off = reinterpret_cast<long long*>(take(a * 8));
         tmp = reinterpret_cast<fd_detection*>(take(a * sizeof(fd_detection)));
+        comp = reinterpret_cast<longlong2*>(take(a * sizeof(longlong2)));
         misc = reinterpret_cast<int*>(take(256));
     }
 };
 
 size_t group_scratch_bytes(long long n) {
     const size_t a = (size_t)(n > 0 ? n : 1);
-    return a * (4 * 8 + 4 + 4 + 4 + 8 + sizeof(Eyes) + 4 + 4 + 72 + 8 + 4 + 8 + sizeof(fd_detection)) + 24 * 256;
+    return a * (4 * 8 + 4 + 4 + 4 + 8 + sizeof(Eyes) + 4 + 4 + 72 + 8 + 4 + 8 + sizeof(fd_detection) + sizeof(longlong2)) +
+           24 * 256;
 }
 
 // phase 1: frame segments (runs of equal frame index)
@@ -570,7 +650,11 @@ cudaError_t launch_group_run(const fd_detection* in, long long n, double thresh,
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int grid = (int)(n < (long long)sms * 4 ? n : (long long)sms * 4);
-    k_group<<<grid, GT, 0, st>>>(in, n, L.seg_start, L.misc, thresh, min_neighbors, L.g, L.misc + 1, L.seg_count, L.tmp);
+    cudaError_t e = cudaFuncSetAttribute(k_group_comp, cudaFuncAttributeMaxDynamicSharedMemorySize, GPS * 16);
+    if (e != cudaSuccess) return e;
+    k_group_comp<<<grid, GT, GPS * 16, st>>>(in, n, L.seg_start, L.misc, thresh, L.g, L.misc + 1, L.comp, L.misc + 2);
+    k_group_greedy<<<sms * 8, GT, 0, st>>>(L.comp, L.misc + 2, thresh, L.g);
+    k_group_emit<<<grid, GT, 0, st>>>(in, n, L.seg_start, L.misc, min_neighbors, L.g, L.seg_count, L.tmp);
     k_seg_offsets<<<1, 32, 0, st>>>(L.misc, L.seg_count, L.seg_off, d_total);
     k_seg_copy<<<grid < sms * 4 ? grid : sms * 4, 256, 0, st>>>(L.misc, L.seg_start, L.seg_count, L.seg_off, L.tmp, out, cap);
     return cudaGetLastError();

@@ -22,6 +22,10 @@
 namespace fdk {
 
 constexpr int TAIL_THREADS = 256;
+template <int V>
+struct IntC {
+    static constexpr int value = V;
+};
 constexpr int TAIL_REGION = ((WIN + 1) * TAIL_RP + 31) & ~31;   // words per warp
 
 template <bool DEPTH>
@@ -41,24 +45,36 @@ __global__ void __launch_bounds__(TAIL_THREADS) k_tail(const __grid_constant__ T
         const uint32_t* src = p.ws + L.ws_off + (long long)g * 2 * (L.H + 1) * L.P + (long long)(wyi * p.step) * L.P +
                               wxi * p.step;
         __syncwarp();                         // previous window's region reads done
-        if (lane <= WIN) {
-#pragma unroll 5
-            for (int r = 0; r <= WIN; ++r) R[r * TAIL_RP + lane] = __ldg(src + (long long)r * L.P + lane);
+        if (lane <= WIN) {           // 25 independent row loads in flight, then 25 stores
+            uint32_t v[WIN + 1];
+#pragma unroll
+            for (int r = 0; r <= WIN; ++r) v[r] = __ldg(src + (long long)r * L.P + lane);
+#pragma unroll
+            for (int r = 0; r <= WIN; ++r) R[r * TAIL_RP + lane] = v[r];
         }
         __syncwarp();
-        // leaf of stump c0 + lane of stage sd (0 beyond the stage)
-        auto leaf_of = [&](const StageDev& sd, int c0) -> float {
+        // leaf of stump c0 + lane of stage sd (0 beyond the stage); MC >= the stage's largest
+        // corner count (unused corner slots are offset 0, coefficient 0), so the corner loads do
+        // not wait for the stump's own count
+        auto leaf_mc = [&](const StageDev& sd, int c0, auto mc_tag) -> float {
+            constexpr int MC = decltype(mc_tag)::value;
             if (c0 + lane >= sd.n) return 0.0f;
             const uint32_t* t = p.trec + sd.first + c0 + lane;
-            const int nc = (int)__ldg(t);
             uint32_t f = 0;
-            for (int c = 0; c < nc; ++c) {
+#pragma unroll
+            for (int c = 0; c < MC; ++c) {
                 const uint32_t w = __ldg(t + (size_t)(4 + c) * p.ns);
                 f += (uint32_t)((int)w >> 16) * R[w & 0xffffu];
             }
             const float tt = __fmul_rn(__int_as_float((int)__ldg(t + (size_t)p.ns)), nf);
             return (__int2float_rn((int)f) < tt) ? __int_as_float((int)__ldg(t + (size_t)2 * p.ns))
                                                  : __int_as_float((int)__ldg(t + (size_t)3 * p.ns));
+        };
+        auto leaf_of = [&](const StageDev& sd, int c0) -> float {
+            if (sd.mc <= 6) return leaf_mc(sd, c0, IntC<6>{});
+            if (sd.mc <= 8) return leaf_mc(sd, c0, IntC<8>{});
+            if (sd.mc <= 9) return leaf_mc(sd, c0, IntC<9>{});
+            return leaf_mc(sd, c0, IntC<MAX_CORNERS>{});
         };
         int s2 = s;
         float sum = 0.0f;

@@ -125,6 +125,35 @@ def test_depth_maps_generic_k2(monkeypatch):
     compare_depth(cascades(3), fr, 1.1)
 
 
+# K2 schedules (fd_api.cpp run_groups): every one computes the same depth maps and detections
+K2_SCHEDULES = {
+    "stage1_only": {"FD_S0": "1"},                          # k_stage1 stage 1, k_deep1 from stage 2
+    "stage1_to_5_tail": {"FD_S0": "5", "FD_S1_TAIL": "1"},  # k_stage1 stages 1-5, then k_tail only
+    "no_tail": {"FD_TAIL": "0"},                            # k_deep1 finishes every window
+    "warp_specialised": {"FD_K2_WS": "1"},                  # k_ws
+    "warp_specialised_s0_1": {"FD_K2_WS": "1", "FD_WS_S0": "1"},
+    "fused": {"FD_K2_SPLIT": "0"},                          # k_cascade
+    "one_slot_pipeline": {"FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
+    "two_slot_pipeline": {"FD_GROUP_FRAMES": "1"},          # 3 frame groups over 2 slots/streams
+}
+
+
+@pytest.mark.parametrize("jit", ["1", "0"])
+@pytest.mark.parametrize("name", sorted(K2_SCHEDULES))
+def test_k2_schedules(name, jit, monkeypatch):
+    for k, v in K2_SCHEDULES[name].items():
+        monkeypatch.setenv(k, v)
+    monkeypatch.setenv("FD_JIT", jit)
+    fr, _ = gen(2, 5, 3)
+    compare_depth(cascades(2), fr, 1.2)
+    gc, oc = cascades(2)
+    got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, 1.2, 1, capacity=1 << 20))
+    ref, _ = oracle.detect(oc, fr, 24, 1.2, 1, nthreads=os.cpu_count())
+    assert np.array_equal(got, ref)
+    fr, _ = gen(3, 40, 1)
+    compare_depth(cascades(3), fr, 1.1)
+
+
 @pytest.mark.parametrize("step", [2, 3, 4])
 def test_depth_maps_step(step):
     fr, _ = gen(2, 7, 2)

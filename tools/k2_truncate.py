@@ -40,7 +40,7 @@ for arg in sys.argv[1:] or ["1", "2", "3", "4", "6", "10", "25"]:
         sts = stages[:k]
     body = "\n".join(h for h in hdr if h.strip()) + f"\nstages {k}\n" + "\n".join("\n".join(st) for st in sts) + "\n"
     casc = fd.Cascade(body)
-    run = (lambda: fd.fd_detect(casc, d, 24, s, 1, capacity=1 << 20)) if os.environ.get("MODE") == "detect" else \
+    run = (lambda: fd.fd_detect(casc, d, 24, s, 1, capacity=1 << 26)) if os.environ.get("MODE") == "detect" else \
         (lambda: fd.fd_detect_depth(casc, d, 24, s, 1))
     run()
     torch.cuda.synchronize()
@@ -49,4 +49,5 @@ for arg in sys.argv[1:] or ["1", "2", "3", "4", "6", "10", "25"]:
         run()
     torch.cuda.synchronize()
     p = fd.fd_profile_read()
-    print(f"{arg:>5s}: K2 {p['cascade'][1] / 3 / F * 1000:.1f} us/frame")
+    us = {k: p[k][1] / 3 / F * 1000 for k in ("cascade", "deep", "tail") if k in p and p[k][0]}
+    print(f"{arg:>5s}: K2 {sum(us.values()):.1f} us/frame  " + "  ".join(f"{k} {v:.1f}" for k, v in us.items()))
