@@ -138,6 +138,19 @@ fd_status fd_detect_depth(fd_cascade c, const uint8_t* d_frames, int n, int W, i
                           int min_size, double scale_factor, int step, uint8_t* d_depth,
                           float* d_score, void* stream);
 
+/* Depth-map analytics (Fig. 7: "the
+ * distribution of the deepest stage reached by all GPU threads when evaluating the pixels of a
+ * given video frame for each considered scale", aggregated over the frames).  d_depth: the
+ * fd_detect_depth output for n frames of W x H (same min_size, scale_factor, step), caller-owned
+ * device memory.  d_hist: caller-owned device int64[n_levels][n_stages + 1]; hist[k][d] += the
+ * number of windows of level k (over the n frames) whose depth is d (d > n_stages counts into
+ * bin n_stages).  The rejection rate of stage s at scale k is hist[k][s] / sum_d hist[k][d].
+ * d_hist is overwritten (not accumulated).  Exact integer counts.  Asynchronous.
+ * Errors: FD_EINVAL for NULL pointers, n < 1, n_stages < 1 or > 254, and the fd_pyramid_plan
+ * argument checks. */
+fd_status fd_depth_histogram(const uint8_t* d_depth, int n, int W, int H, int min_size, double scale_factor,
+                             int step, int n_stages, int64_t* d_hist, void* stream);
+
 /* End-to-end entry with HOST buffers: copies h_frames to the device, runs fd_detect, copies
  * the detections back to h_out (capacity elements).  Synchronises `stream`. */
 fd_status fd_detect_host(fd_cascade c, const uint8_t* h_frames, int n, int W, int H, int pitch,
@@ -165,14 +178,16 @@ fd_status fd_detect_group_host(fd_cascade c, const uint8_t* h_frames, int n, int
 /* Kernel accounting (process-wide, all devices): number of launches of each kernel class
  * since the last fd_profile_reset and, if time_kernels != 0, their summed device time
  * measured with CUDA events recorded on the launching stream around each launch.
- * FD_K_SORT is the CUB radix sort (library code, counted as one call).  The cascade evaluator
- * is FD_K_CASCADE (the dense first stage, k_stage1), FD_K_DEEP (the deeper stages over batches
- * of tiles, k_deep) and FD_K_TAIL (the deep stages of the few windows left per batch, one warp
- * per window). */
+ * FD_K_SORT is the CUB radix sort (library code, counted as one call).  K1 is FD_K_COLSUM
+ * (k_marg: resampling + per-tile marginals), FD_K_CARRY (k_carry + k_corner) and FD_K_BAND
+ * (k_tile: ii / sqii).  The cascade evaluator is FD_K_CASCADE (k_stage1: stages 1-2 dense and
+ * compacted; or k_ws / k_cascade in the alternative schedules), FD_K_DEEP (k_deep1: the deeper
+ * stages, one tile per CTA) and FD_K_TAIL (k_tail: the few windows left per tile, one warp per
+ * window).  FD_K_DEPTH_HIST is fd_depth_histogram. */
 typedef enum {
     FD_K_COLSUM = 0, FD_K_CARRY = 1, FD_K_BAND = 2, FD_K_CASCADE = 3,
     FD_K_SORT = 4, FD_K_DETS = 5, FD_K_GROUP = 6, FD_K_PYRAMID = 7, FD_K_TAIL = 8,
-    FD_K_DEEP = 9, FD_K_COUNT = 10
+    FD_K_DEEP = 9, FD_K_DEPTH_HIST = 10, FD_K_COUNT = 11
 } fd_kernel_kind;
 typedef struct {
     int64_t launches[FD_K_COUNT];

@@ -234,6 +234,25 @@ def detect_depth(casc: Cascade, frames: np.ndarray, min_size: int = 24, scale: f
     return depth, score, near
 
 
+def depth_histogram(depth: np.ndarray, n_frames: int, W: int, H: int, n_stages: int, min_size: int = 24,
+                    scale: float = 1.1, step: int = 1) -> np.ndarray:
+    """Fig. 7: for every scale k, how many windows (over all frames)
+    reached depth d -- "the distribution of the deepest stage reached ... for each considered
+    scale".  Plain definition: split each frame's depth map at the level window counts and count
+    each depth value (np.bincount).  int64 [levels, n_stages + 1]; depths above n_stages count
+    into the last bin."""
+    counts = [p[3] for p in plan(W, H, min_size, scale, step)]
+    per = sum(counts)
+    d = np.minimum(np.asarray(depth, np.int64).reshape(n_frames, per), n_stages)
+    out = np.zeros((len(counts), n_stages + 1), np.int64)
+    off = 0
+    for k, c in enumerate(counts):
+        for f in range(n_frames):
+            out[k] += np.bincount(d[f, off:off + c], minlength=n_stages + 1)
+        off += c
+    return out
+
+
 def group(dets: np.ndarray, eyes_thresh: float = 0.5, min_neighbors: int = 1) -> np.ndarray:
     """c10: greedy S_eyes grouping per frame (input sorted by frame)."""
     L = _load()

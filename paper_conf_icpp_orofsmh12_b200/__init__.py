@@ -48,7 +48,7 @@ class _Plan(C.Structure):
                 ("windows", C.c_int64 * FD_MAX_LEVELS), ("total_windows", C.c_int64)]
 
 
-K_NAMES = ["colsum", "carry", "band", "cascade", "sort", "dets", "group", "pyramid", "tail", "deep"]
+K_NAMES = ["colsum", "carry", "band", "cascade", "sort", "dets", "group", "pyramid", "tail", "deep", "depth_hist"]
 
 
 class _Profile(C.Structure):
@@ -84,12 +84,13 @@ def lib():
             L.fd_release_workspaces.argtypes = []
             L.fd_detect_group_host.argtypes = [P, P, i32, i32, i32, i32, i32, dbl, i32, dbl, i32, P, i64,
                                                C.POINTER(i64), C.POINTER(i64), P]
+            L.fd_depth_histogram.argtypes = [P, i32, i32, i32, i32, dbl, i32, i32, P, P]
             L.fd_profile_reset.argtypes = [i32]
             L.fd_profile_read.argtypes = [C.POINTER(_Profile)]
             for fn in ("fd_load_cascade", "fd_free_cascade", "fd_cascade_info", "fd_pyramid_plan",
                        "fd_build_pyramid", "fd_integral", "fd_detect", "fd_detect_ex", "fd_detect_depth",
                        "fd_detect_host", "fd_group", "fd_release_workspaces", "fd_detect_group_host",
-                       "fd_profile_reset", "fd_profile_read"):
+                       "fd_profile_reset", "fd_profile_read", "fd_depth_histogram"):
                 getattr(L, fn).restype = i32
             _lib = L
     return _lib
@@ -240,6 +241,19 @@ def fd_detect_depth(casc: Cascade, frames, min_size: int = 24, scale_factor: flo
     _check(lib().fd_detect_depth(casc.handle, _ptr(frames), n, W, H, pitch, min_size, float(scale_factor), step,
                                  _ptr(depth), _ptr(score), _stream(stream)))
     return depth[:tot], score[:tot]
+
+
+def fd_depth_histogram(depth, n_frames: int, W: int, H: int, n_stages: int, min_size: int = 24,
+                       scale_factor: float = 1.1, step: int = 1, stream=None):
+    """Fig. 7 analytics of an fd_detect_depth map: int64 [n_levels, n_stages + 1], entry [k, d] =
+    windows of level k (over the n_frames) whose depth is d."""
+    torch = _torch()
+    assert depth.dtype == torch.uint8 and depth.is_cuda and depth.is_contiguous()
+    levels = len(fd_pyramid_plan(W, H, min_size, scale_factor, step))
+    hist = torch.zeros((max(levels, 1), n_stages + 1), dtype=torch.int64, device=depth.device)
+    _check(lib().fd_depth_histogram(_ptr(depth), n_frames, W, H, min_size, float(scale_factor), step, n_stages,
+                                    _ptr(hist), _stream(stream)))
+    return hist[:levels]
 
 
 def fd_detect_host(casc: Cascade, frames, min_size: int = 24, scale_factor: float = 1.1, step: int = 1,

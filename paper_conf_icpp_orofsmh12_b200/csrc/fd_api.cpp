@@ -929,6 +929,46 @@ fd_status fd_detect_depth(fd_cascade c, const uint8_t* d_frames, int n, int W, i
     return run_groups(c, w, d_frames, n, W, H, pitch, pl, step, true, d_depth, d_score, 0, nullptr, st);
 }
 
+fd_status fd_depth_histogram(const uint8_t* d_depth, int n, int W, int H, int min_size, double scale_factor,
+                             int step, int n_stages, int64_t* d_hist, void* stream) {
+    if (!d_depth || !d_hist) return fail(FD_EINVAL, "depth or histogram pointer is NULL");
+    if (n < 1) return fail(FD_EINVAL, "n must be >= 1");
+    if (n > 65535) return fail(FD_EINVAL, "at most 65535 frames per call");
+    if (n_stages < 1 || n_stages > 254) return fail(FD_EINVAL, "n_stages %d not in [1, 254]", n_stages);
+    fd_plan pl;
+    fd_status r = make_plan(W, H, min_size, scale_factor, step, &pl);
+    if (r != FD_OK) return r;
+    if (pl.n_levels == 0) return FD_OK;
+    cudaStream_t st = (cudaStream_t)stream;
+    Workspace* w = nullptr;
+    r = get_ws(st, &w);
+    if (r != FD_OK) return r;
+    std::lock_guard<std::mutex> lk(w->mu);
+    // level window offsets within a frame, and the most levels one 4096-window chunk can span
+    long long* h_w0 = reinterpret_cast<long long*>(w->h_geo.get());
+    long long acc = 0;
+    for (int k = 0; k < pl.n_levels; ++k) {
+        h_w0[k] = acc;
+        acc += pl.windows[k];
+    }
+    int max_span = 1;
+    for (int k = 0; k < pl.n_levels; ++k) {
+        long long reach = h_w0[k] + 4096;
+        int j = k;
+        while (j + 1 < pl.n_levels && h_w0[j + 1] < reach) ++j;
+        max_span = std::max(max_span, j - k + 2);
+    }
+    max_span = std::min(max_span, pl.n_levels);
+    CK(w->flev.ensure(sizeof(double) * FD_MAX_LEVELS));
+    CK(cudaMemcpyAsync(w->flev.p, h_w0, sizeof(long long) * pl.n_levels, cudaMemcpyHostToDevice, st));
+    {
+        ProfScope ps(FD_K_DEPTH_HIST, st);
+        CK(launch_depth_hist(d_depth, n, acc, w->flev.as<long long>(), pl.n_levels, n_stages,
+                             reinterpret_cast<long long*>(d_hist), max_span, st));
+    }
+    return FD_OK;
+}
+
 fd_status fd_detect_host(fd_cascade c, const uint8_t* h_frames, int n, int W, int H, int pitch, int min_size,
                          double scale_factor, int step, fd_detection* h_out, int64_t capacity, int64_t* n_out,
                          void* stream) {

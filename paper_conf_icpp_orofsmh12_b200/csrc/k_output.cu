@@ -589,6 +589,50 @@ __global__ void k_seg_copy(const int* __restrict__ n_seg_p, const long long* __r
     }
 }
 
+// ------------------------------------------------------------------------------ depth analytics
+// hist[k][d] += #windows of level k with depth d (Fig. 7).  Grid (chunks of the frame's windows,
+// frames); a shared histogram per block over the levels its chunk spans.
+constexpr int HIST_CHUNK = 4096;
+__global__ void __launch_bounds__(256) k_depth_hist(const uint8_t* __restrict__ depth, long long win_per_frame,
+                                                    const long long* __restrict__ win0, int n_levels, int nb,
+                                                    unsigned long long* __restrict__ hist) {
+    extern __shared__ unsigned int sh[];                  // [levels spanned][nb]
+    const long long c0 = (long long)blockIdx.x * HIST_CHUNK;
+    const long long c1 = min(c0 + HIST_CHUNK, win_per_frame);
+    int k0 = 0;
+    while (k0 + 1 < n_levels && win0[k0 + 1] <= c0) ++k0;
+    int k1 = k0;
+    while (k1 + 1 < n_levels && win0[k1 + 1] < c1) ++k1;
+    const int span = k1 - k0 + 1;
+    for (int i = threadIdx.x; i < span * nb; i += blockDim.x) sh[i] = 0;
+    __syncthreads();
+    const uint8_t* dp = depth + (long long)blockIdx.y * win_per_frame;
+    int k = k0;
+    for (long long w = c0 + threadIdx.x; w < c1; w += blockDim.x) {
+        while (k > k0 && win0[k] > w) --k;             // w increases per thread: k only moves up
+        while (k < k1 && win0[k + 1] <= w) ++k;
+        const int d = min((int)dp[w], nb - 1);
+        atomicAdd(&sh[(k - k0) * nb + d], 1u);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < span * nb; i += blockDim.x)
+        if (sh[i]) atomicAdd(hist + (long long)(k0 + i / nb) * nb + i % nb, (unsigned long long)sh[i]);
+}
+
+cudaError_t launch_depth_hist(const uint8_t* depth, int n, long long win_per_frame, const long long* d_win0,
+                              int n_levels, int n_stages, long long* hist, int max_span, cudaStream_t st) {
+    const int nb = n_stages + 1;
+    cudaError_t e = cudaMemsetAsync(hist, 0, sizeof(long long) * n_levels * nb, st);
+    if (e != cudaSuccess || win_per_frame <= 0) return e;
+    const size_t smem = sizeof(unsigned int) * (size_t)max_span * nb;
+    e = cudaFuncSetAttribute(k_depth_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    const dim3 grid((unsigned)((win_per_frame + HIST_CHUNK - 1) / HIST_CHUNK), (unsigned)n);
+    k_depth_hist<<<grid, 256, smem, st>>>(depth, win_per_frame, d_win0, n_levels, nb,
+                                          reinterpret_cast<unsigned long long*>(hist));
+    return cudaGetLastError();
+}
+
 struct GroupLayout {
     GroupScratch g;
     long long* seg_start;

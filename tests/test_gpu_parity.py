@@ -154,6 +154,21 @@ def test_k2_schedules(name, jit, monkeypatch):
     compare_depth(cascades(3), fr, 1.1)
 
 
+@pytest.mark.parametrize("cfg,n,step", [(1, 3, 1), (2, 2, 2), (3, 1, 1)])
+def test_depth_histogram(cfg, n, step):
+    """f4: fd_depth_histogram (Fig. 7 analytics) equals the oracle's histogram of the oracle
+    depth map, and of the GPU's own depth map, exactly."""
+    W, H, s, _ = CFG[cfg]
+    fr, _ = gen(cfg, 2, n)
+    gc, oc = cascades(cfg)
+    d_fr = torch.from_numpy(fr).cuda()
+    depth, _ = fd.fd_detect_depth(gc, d_fr, 24, s, step)
+    hist = fd.fd_depth_histogram(depth, n, W, H, gc.n_stages, 24, s, step).cpu().numpy()
+    od, _, _ = oracle.detect_depth(oc, fr, 24, s, step, nthreads=os.cpu_count())
+    assert np.array_equal(hist, oracle.depth_histogram(od, n, W, H, gc.n_stages, 24, s, step))
+    assert np.array_equal(hist, oracle.depth_histogram(depth.cpu().numpy(), n, W, H, gc.n_stages, 24, s, step))
+
+
 @pytest.mark.parametrize("step", [2, 3, 4])
 def test_depth_maps_step(step):
     fr, _ = gen(2, 7, 2)

@@ -284,6 +284,36 @@ def test_all_pass_and_all_reject_cascades():
     assert len(d) == 2 * tot and (d == 0).all() and (sc == 0.5).all()
 
 
+def test_depth_histogram_pins():
+    """f4 (Fig. 7 analytics): hand example, the all-pass / all-reject cascades, and the
+    closed-form per-level window counts of tests/golden/pyramid_counts.txt as row sums."""
+    # 25 x 25 frame, scale 1.1: one level of 2 x 2 windows; depths [0, 3, 3, 1] (+ a 200 clamp)
+    h = oracle.depth_histogram(np.array([0, 3, 3, 1], np.uint8), 1, 25, 25, 3, 24, 1.1, 1)
+    assert h.tolist() == [[1, 1, 0, 2]]
+    h = oracle.depth_histogram(np.array([0, 200, 3, 1, 2, 2, 2, 2], np.uint8), 2, 25, 25, 3, 24, 1.1, 1)
+    assert h.tolist() == [[1, 1, 4, 2]]
+    W, H, s = 160, 120, 1.25
+    fr, _ = fdgen.frames(9, 3, 2, W, H)
+    st = ([(1, 1, 10, 10, -1), (1, 1, 5, 10, 2)], 0.1, 0.5, 0.5)
+    allpass = oracle.Cascade(cascade_text([(-math.inf, [st, st]), (-1e30, [st])]))
+    d, _, _ = oracle.detect_depth(allpass, fr, 24, s, 1)
+    h = oracle.depth_histogram(d, 2, W, H, 2, 24, s, 1)
+    per_level = [2 * l[3] for l in oracle.plan(W, H, 24, s, 1)]
+    assert h[:, 2].tolist() == per_level and h[:, :2].sum() == 0
+    allrej = oracle.Cascade(cascade_text([(math.inf, [st])]))
+    d, _, _ = oracle.detect_depth(allrej, fr, 24, s, 1)
+    h = oracle.depth_histogram(d, 2, W, H, 1, 24, s, 1)
+    assert h[:, 0].tolist() == per_level and h[:, 1].sum() == 0
+    # row sums = the closed-form window counts (golden) for the c1 geometry
+    row = [r for r in _golden("pyramid_counts.txt") if r[:4] == ["320", "240", "1.25", "1"]][0]
+    fr, _ = fdgen.frames(1, 0, 1, 320, 240)
+    casc = oracle.Cascade.from_file(os.path.join(ROOT, "cascades", "c1.fdc"))
+    d, _, _ = oracle.detect_depth(casc, fr, 24, 1.25, 1, nthreads=4)
+    h = oracle.depth_histogram(d, 1, 320, 240, casc.n_stages, 24, 1.25, 1)
+    assert len(h) == int(row[4]) and h.sum() == int(row[5])
+    assert h.sum(axis=0)[casc.n_stages] == (d == casc.n_stages).sum()
+
+
 def test_detect_matches_depth_maps_and_order():
     fr, _ = fdgen.frames(1, 0, 2, 320, 240)
     casc = oracle.Cascade.from_file(os.path.join(ROOT, "cascades", "c1.fdc"))
