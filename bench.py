@@ -49,6 +49,9 @@ def parse_args():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=2, help="frames timed on the CPU oracle")
+    ap.add_argument("--cascade", default="c3", choices=["c3", "c6"],
+                    help="c3: the paper-shaped 1446-stump cascade (c4 workload, default); c6: the "
+                         "OpenCV-shaped 2913-stump cascade (SURVEY 8(f) f3 workload)")
     return ap.parse_args()
 
 
@@ -178,9 +181,14 @@ def make_frames(rank: int, n: int, plan):
     return fr, faces
 
 
+CASCADES = {"c3": ("c4", "25-stage 1446-stump cascade (cascades/c3.fdc)"),
+            "c6": ("c6", "OpenCV-shaped 25-stage 2913-stump cascade (cascades/c6.fdc)")}
+
+
 def workload_config(frames_per_gpu: int, world: int):
-    return {"workload": f"c4: synthetic 1080p video, {frames_per_gpu} frames/GPU, Poisson(4) planted faces, "
-                        f"25-stage 1446-stump cascade (cascades/c3.fdc), scale 1.1, step 1, min_size 24",
+    name, desc = CASCADES[CFG["cascade"][:-4]]
+    return {"workload": f"{name}: synthetic 1080p video, {frames_per_gpu} frames/GPU, Poisson(4) planted faces, "
+                        f"{desc}, scale 1.1, step 1, min_size 24",
             "W": CFG["W"], "H": CFG["H"], "frames_per_gpu": frames_per_gpu, "global_frames": frames_per_gpu * world,
             "scale_factor": CFG["scale"], "step": CFG["step"], "min_size": CFG["min_size"],
             "parallelism": f"frame-sharded dp{world}" if world > 1 else "single GPU",
@@ -384,6 +392,7 @@ def run_ours(args):
 
 def main():
     args = parse_args()
+    CFG["cascade"] = f"{args.cascade}.fdc"
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)

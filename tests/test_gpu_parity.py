@@ -154,6 +154,24 @@ def test_k2_schedules(name, jit, monkeypatch):
     compare_depth(cascades(3), fr, 1.1)
 
 
+def test_c6_workload_1080p():
+    """f3 workload: the OpenCV-shaped 2913-stump cascade on c4 frames -- depth maps bit-exact,
+    detections identical, stage counters equal to the oracle's depth histogram."""
+    W, H, s = 1920, 1080, 1.1
+    lv = oracle.plan(W, H, 24, s, 1)
+    fr, _ = fdgen.frames(4, 100, 2, W, H, lv, faces="poisson", face_param=4, max_face_level=30)
+    text = open(os.path.join(ROOT, "cascades", "c6.fdc")).read()
+    pair = (fd.Cascade(text), oracle.Cascade(text))
+    compare_depth(pair, fr[:1], s)
+    gc, oc = pair
+    sc = torch.zeros(gc.n_stages + 1, dtype=torch.int64, device="cuda")
+    got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1, capacity=1 << 20, stage_counts=sc))
+    ref, _ = oracle.detect(oc, fr, 24, s, 1, nthreads=os.cpu_count())
+    assert np.array_equal(got, ref)
+    od, _, _ = oracle.detect_depth(oc, fr, 24, s, 1, nthreads=os.cpu_count())
+    assert sc.cpu().tolist() == [int((od >= k).sum()) for k in range(gc.n_stages + 1)]
+
+
 @pytest.mark.parametrize("cfg,n,step", [(1, 3, 1), (2, 2, 2), (3, 1, 1)])
 def test_depth_histogram(cfg, n, step):
     """f4: fd_depth_histogram (Fig. 7 analytics) equals the oracle's histogram of the oracle

@@ -284,6 +284,21 @@ def test_all_pass_and_all_reject_cascades():
     assert len(d) == 2 * tot and (d == 0).all() and (sc == 0.5).all()
 
 
+def test_c6_cascade_shape():
+    """f3 workload: the OpenCV-shaped cascade has the paper's "25 stages ... 2913 weak
+    classifiers" (P:L1106-1110) and only Table I features (2 or 3 rectangles)."""
+    casc = oracle.Cascade.from_file(os.path.join(ROOT, "cascades", "c6.fdc"))
+    assert casc.n_stages == 25
+    sizes, nrects = [], []
+    for line in open(os.path.join(ROOT, "cascades", "c6.fdc")):
+        t = line.split()
+        if t and t[0] == "stage":
+            sizes.append(int(t[1]))
+        elif t and t[0] == "stump":
+            nrects.append(int(t[1]))
+    assert sum(sizes) == 2913 == len(nrects) and set(nrects) <= {2, 3}
+
+
 def test_depth_histogram_pins():
     """f4 (Fig. 7 analytics): hand example, the all-pass / all-reject cascades, and the
     closed-form per-level window counts of tests/golden/pyramid_counts.txt as row sums."""

@@ -43,6 +43,13 @@ CONFIGS = {
             max_boot=64, max_face_level=12),
     3: dict(W=1920, H=1080, scale=1.1, sizes=[10 + 4 * k for k in range(24)] + [102],
             p=[0.0548, 0.270] + [0.5] * 23, bg_frames=2, max_boot=48, max_face_level=30),
+    # c6: the OpenCV-shaped cascade the paper compares against, "25 stages ...
+    # 2913 weak classifiers", stage sizes of the public OpenCV frontal-face
+    # cascade; weaker early rejection (p1 = 0.25, p2 = 0.35) for the paper's ~2.5x more work
+    #
+    6: dict(W=1920, H=1080, scale=1.1, sizes=[9, 16, 27, 32, 52, 53, 62, 72, 83, 91, 99, 115, 127, 135, 136, 137,
+                                              159, 155, 169, 196, 197, 181, 199, 211, 200],
+            p=[0.25, 0.35] + [0.5] * 23, bg_frames=2, max_boot=48, max_face_level=30),
 }
 MIN_POOL = 1000
 N_SUB = 20_000
