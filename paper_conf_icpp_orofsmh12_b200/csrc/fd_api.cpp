@@ -639,10 +639,8 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     P.lane_min = std::max(1, std::min(env_int("FD_LANE_MIN", half + 1), half + 1));
     P.tail_cap = tail_cap;
     P.tail_n = std::max(1, env_int("FD_TAIL_N", 8));
-    // split path: k_stage1 runs stages [0, s0) (FD_S0, default 2); with FD_S1_TAIL=1 it hands the
-    // windows entering stage s0 straight to k_tail (no k_deep launch)
-    P.s0 = split ? std::max(1, env_int("FD_S0", 2)) : (wsk ? std::max(1, env_int("FD_WS_S0", 2)) : 1);
-    P.s1_tail = (split && use_tail && env_int("FD_S1_TAIL", 0) != 0) ? 1 : 0;
+    // k_stage1 / k_ws run stages [0, s0): FD_S0 / FD_WS_S0 = 2 (default) or 1
+    P.s0 = split ? (env_int("FD_S0", 2) >= 2 ? 2 : 1) : (wsk ? (env_int("FD_WS_S0", 2) >= 2 ? 2 : 1) : 1);
     TailParams TP;
     TP.cap = tail_cap;
     TP.step = step;
@@ -713,7 +711,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
                 ProfScope ps(FD_K_CASCADE, gs);
                 e = jit_k2_launch(jit, P, depth, wsk ? JIT_WS : (split ? JIT_STAGE1 : JIT_FUSED), gs, &err);
             }
-            if (e == cudaSuccess && split && !P.s1_tail) {
+            if (e == cudaSuccess && split) {
                 ProfScope ps(FD_K_DEEP, gs);
                 e = jit_k2_launch(jit, P, depth, deep1 ? JIT_DEEP1 : JIT_DEEP, gs, &err);
             }
@@ -723,8 +721,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
             LAUNCH(FD_K_CASCADE, gs, launch_ws(P, depth, step, gs));
         } else if (split) {
             LAUNCH(FD_K_CASCADE, gs, launch_stage1(P, depth, step, gs));
-            if (!P.s1_tail)
-                LAUNCH(FD_K_DEEP, gs, deep1 ? launch_deep1(P, depth, step, gs) : launch_deep(P, depth, step, gs));
+            LAUNCH(FD_K_DEEP, gs, deep1 ? launch_deep1(P, depth, step, gs) : launch_deep(P, depth, step, gs));
         } else {
             LAUNCH(FD_K_CASCADE, gs, launch_cascade(P, depth, step, gr, gs));
         }

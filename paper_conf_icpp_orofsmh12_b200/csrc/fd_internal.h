@@ -84,15 +84,17 @@ struct TileGeo {
 #define FD_K2_CTAS 4                        // fused K2: resident CTAs per SM the launch bounds target
 #endif
 
-// k_stage1 (K2a): one tile's ii + sqii planes and its survivor list (window index, nf bits)
-// (the sqii plane, dead once every nf is taken, holds the stage-2 survivor list)
+// k_stage1 (K2a): two ii planes (the current tile's and the prefetched next tile's), one sqii
+// plane (dead once the variance is taken, so the next tile's sqii lands in it during stages 1-2)
+// and the stage-1 survivor list (u16 window index + f32 nf)
 template <int STEP>
 struct TileGeoA {
     static constexpr int PBUF = k2_pbuf(STEP);
     static constexpr int NW = k2_tx(STEP) * k2_ty(STEP);
-    static_assert(PBUF * 4 >= NW * 8, "stage-2 survivor list fits in the sqii plane");
-    static constexpr size_t OFF_SURV = (size_t)2 * PBUF * 4;
-    static constexpr size_t SMEM = OFF_SURV + (size_t)NW * 8;
+    static constexpr size_t OFF_Q = (size_t)2 * PBUF * 4;
+    static constexpr size_t OFF_SNF = OFF_Q + (size_t)PBUF * 4;
+    static constexpr size_t OFF_SIDX = OFF_SNF + (size_t)NW * 4;
+    static constexpr size_t SMEM = OFF_SIDX + (size_t)NW * 2;
 };
 
 // k_deep (K2b): NB ii slots, the pool of their stage-1 survivors, per-stage lists, group leaves
@@ -213,8 +215,7 @@ struct alignas(16) CascadeParams {
     unsigned long long* stage_counts;       // n_stages + 1, may be null
     int n_pstages;                          // stages [0, n_pstages) are also in pstages
     int tail_n;                             // a batch with <= tail_n windows left goes to the tail queue
-    int s0;                                 // first stage of the deep kernels (k_stage1 runs [0, s0))
-    int s1_tail;                            // 1: k_stage1 hands its stage-s0 windows to the tail queue (no k_deep)
+    int s0;                                 // first stage of the deep kernels (k_stage1 runs [0, s0), s0 <= 2)
     uint4* tail_q;                          // tail queue (k_tail.cu), may be null
     unsigned int* tail_count;               // entries appended (may exceed tail_cap: the excess stays in K2)
     int tail_cap;

@@ -483,63 +483,74 @@ __global__ void __launch_bounds__(k2_threads(STEP), FD_K2_CTAS) k_cascade(const 
 // ======================================================================== split K2, kernel a
 // k_stage1: the dense first stage and the second stage, the throughput part of the cascade
 // (c3: 10 of the 11.8 stumps per window, 94.5% of windows stop at stage 1, 71% of the rest at
-// stage 2).  Persistent over every (frame, level, tile) of the group; per tile one
-// TMA of the ii and sqii planes, variance normalisation (oracle c5), stage 1 evaluated densely
-// (WPT windows per thread down a column, run-time specialised code for step 1), its survivors
-// ballot-compacted into a shared list, stage 2 evaluated over that list one lane per window
-// (p.s0 == 2), and the survivors of the last stage run here -- window index and nf -- appended
-// to a global list with one atomic per tile; tile_rec[tile] = (offset, count).
+// stage 2).  Persistent over every (frame, level, tile) of the group:
+//   * the tile's ii and sqii planes arrive by TMA; the variance normalisation (oracle c5) reads
+//     sqii, after which the NEXT tile is claimed and its ii (into the other ii buffer) and sqii
+//     (into the now dead sqii plane) are fetched while this tile's stages run;
+//   * stage 1 is evaluated densely (WPT windows per thread down a column, run-time specialised
+//     code for step 1) and its survivors ballot-compacted into a shared list;
+//   * stage 2 (p.s0 == 2) runs over that list one lane per window; the survivors of the last
+//     stage run here -- window index and nf -- go to a global list at an offset reserved per tile
+//     (tile_rec[tile] = (offset, count)) for k_deep1.
 template <int STEP, bool DEPTH>
 __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_constant__ CascadeParams p) {
     using G = TileGeoA<STEP>;
     constexpr int TW = tile_w(STEP), TX = k2_tx(STEP), TY = k2_ty(STEP), WPT = k2_wpt(STEP);
     constexpr int WARPS_X = TX / 32, PLANE = tile_w(STEP) * tile_h(STEP), THREADS = k2_threads(STEP);
     extern __shared__ __align__(1024) uint8_t smem_raw[];
-    uint32_t* T = reinterpret_cast<uint32_t*>(smem_raw);                     // ii plane
-    uint32_t* Q = T + G::PBUF;                                               // sqii plane (mod 2^32)
-    uint2* sv = reinterpret_cast<uint2*>(smem_raw + G::OFF_SURV);            // [NW] stage-1 survivors
-    uint2* sv2 = reinterpret_cast<uint2*>(Q);                                // [NW] stage-2 survivors (over sqii)
-    __shared__ __align__(8) uint64_t mbar;
-    __shared__ int s_tile, s_c3[3], s_off;
-    __shared__ int s_frame[1], s_lvl[1], s_wx0[1], s_wy0[1];
+    uint32_t* Q = reinterpret_cast<uint32_t*>(smem_raw + G::OFF_Q);           // sqii plane (mod 2^32)
+    float* snf = reinterpret_cast<float*>(smem_raw + G::OFF_SNF);             // [NW] stage-1 survivors: nf
+    uint16_t* sidx = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_SIDX);    //       and window index
+    __shared__ __align__(8) uint64_t mbar[2];
+    __shared__ int s_tile[2], s_frame[2], s_lvl[2], s_wx0[2], s_wy0[2];
+    __shared__ int s_c1, s_c2, s_off, s_prev, s_prev_off;
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const StageDev& st0 = p.pstages[0];
     const ParamRec prec{p};
     const GlobalRec grec{p.stumps};
-    const WinOut<STEP, DEPTH> out{p, s_frame, s_lvl, s_wx0, s_wy0};
-    if (tid == 0) {
-        mbar_init(&mbar, 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    uint32_t phase = 0;
-    for (;;) {
-        __syncthreads();                          // buffers, survivor lists and s_* free
-        if (tid == 0) {
-            s_c3[0] = 0;
-            s_c3[1] = 0;
-            s_c3[2] = 0;
-            const int tn = (int)atomicAdd(p.tile_counter, 1u);
-            s_tile = tn;
-            if (tn < p.total_tiles) {
-                const TileAt t = tile_at<STEP>(p, tn);
-                s_frame[0] = p.frame_base + t.g;
-                s_lvl[0] = t.k;
-                s_wx0[0] = t.wx0;
-                s_wy0[0] = t.wy0;
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                mbar_expect_tx(&mbar, 2 * PLANE * 4);
-                tma_load_4d(T, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar);
-                tma_load_4d(Q, p.tmaps + t.k, t.x, t.y, 1, t.g, &mbar);
-            }
+    // tid 0: claim the next tile for ii buffer b and start its TMAs (ii -> buffer b, sqii -> Q)
+    auto claim = [&](int b) {
+        const int tn = (int)atomicAdd(p.tile_counter, 1u);
+        s_tile[b] = tn;
+        if (tn < p.total_tiles) {
+            const TileAt t = tile_at<STEP>(p, tn);
+            s_frame[b] = p.frame_base + t.g;
+            s_lvl[b] = t.k;
+            s_wx0[b] = t.wx0;
+            s_wy0[b] = t.wy0;
+            uint32_t* Tb = reinterpret_cast<uint32_t*>(smem_raw) + b * G::PBUF;
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_expect_tx(&mbar[b], 2 * PLANE * 4);
+            tma_load_4d(Tb, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar[b]);
+            tma_load_4d(Q, p.tmaps + t.k, t.x, t.y, 1, t.g, &mbar[b]);
         }
-        __syncthreads();
-        const int tn = s_tile;
+    };
+    if (tid == 0) {
+        mbar_init(&mbar[0], 1);
+        mbar_init(&mbar[1], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        s_prev = -1;
+        claim(0);
+    }
+    uint32_t phases = 0;
+    for (int it = 0;; ++it) {
+        const int b = it & 1;
+        __syncthreads();                          // (A) previous tile done: list, counters, its ii buffer free
+        const int tn = s_tile[b];
+        if (tid == 0) {
+            if (s_prev >= 0) p.tile_rec[s_prev] = make_uint2((unsigned)s_prev_off, (unsigned)s_c2);
+            s_prev = -1;
+            s_c1 = 0;
+            s_c2 = 0;
+        }
         if (tn >= p.total_tiles) break;
-        mbar_wait(&mbar, phase);
-        phase ^= 1;
-        const int k = s_lvl[0];
+        const WinOut<STEP, DEPTH> out{p, s_frame + b, s_lvl + b, s_wx0 + b, s_wy0 + b};
+        const uint32_t* T = reinterpret_cast<const uint32_t*>(smem_raw) + b * G::PBUF;
+        mbar_wait(&mbar[b], (phases >> b) & 1u);
+        phases ^= 1u << b;
+        const int k = s_lvl[b];
         const int nx = __ldg(&p.lv[k].nx), ny = __ldg(&p.lv[k].ny);
-        const int wx0 = s_wx0[0], wy0 = s_wy0[0];
+        const int wx0 = s_wx0[b], wy0 = s_wy0[b];
         const int lx = lane + 32 * (warp % WARPS_X);
         const int ly0 = (warp / WARPS_X) * WPT;
         const int base = ly0 * STEP * TW + lx * STEP;
@@ -554,6 +565,8 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
             nf[i] = v > 0 ? __fsqrt_rn(__ll2float_rn(v)) : 1.0f;
             sm[i] = 0.0f;
         }
+        __syncthreads();                          // (B) every sqii read done: prefetch the next tile
+        if (tid == 0) claim(b ^ 1);
 #ifdef FD_JIT_STAGE1
         jit_stage1(T + base, nf, sm);
 #else
@@ -576,107 +589,71 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
             const unsigned m = __ballot_sync(0xffffffffu, pass);
             if (m) {
                 int pos = 0;
-                if (lane == 0) pos = atomicAdd(&s_c3[1], __popc(m));
+                if (lane == 0) pos = atomicAdd(&s_c1, __popc(m));
                 pos = __shfl_sync(0xffffffffu, pos, 0);
-                if (pass) sv[pos + __popc(m & ((1u << lane) - 1u))] = make_uint2((unsigned)idx, (unsigned)__float_as_int(nf[i]));
+                if (pass) {
+                    const int at = pos + __popc(m & ((1u << lane) - 1u));
+                    sidx[at] = (uint16_t)idx;
+                    snf[at] = nf[i];
+                }
             }
         }
-        __syncthreads();                          // stage-1 survivors complete; sqii plane dead
-        // stages [1, s_end) over the survivor lists (sv -> sv2 -> sv ...), one lane per window;
-        // s_c3[s % 3] = windows entering stage s
-        int c = s_c3[1];
-        int s = 1;
-        const int s_end = min(p.s0, p.n_stages);
-        for (; s < s_end && c > 0; ++s) {
-            const uint2* lin = (s & 1) ? sv : sv2;
-            uint2* lout = (s & 1) ? sv2 : sv;
-            StageDev sd;
-            if (s < p.n_pstages) {
-                sd.first = p.pstages[s].first;
-                sd.n = p.pstages[s].n;
-                sd.T = p.pstages[s].T;
-                sd.mc = p.pstages[s].mc;
-            } else {
-                sd = p.stages[s];
+        __syncthreads();                          // (C) stage-1 survivor list complete
+        const int c = s_c1;
+        if (tid == 0) {
+            // reserve c global entries for this tile's survivors (an upper bound after stage 2)
+            s_off = c ? (int)atomicAdd(p.surv_count, (unsigned)c) : 0;
+            if (p.stage_counts) {
+                atomicAdd(p.stage_counts, (unsigned long long)min(TX, nx - wx0) * (unsigned long long)min(TY, ny - wy0));
+                if (p.s0 == 2 && c) atomicAdd(p.stage_counts + 1, (unsigned long long)c);
             }
-            const bool last = s == p.n_stages - 1;
-            if (tid == 0) {
-                s_c3[(s + 2) % 3] = 0;
-                if (p.stage_counts) atomicAdd(p.stage_counts + s, (unsigned long long)c);
-            }
+        }
+        __syncthreads();                          // (D) offset visible
+        const int off = s_off;
+        if (p.s0 < 2 || p.n_stages < 2) {
+            for (int e = tid; e < c; e += THREADS) p.surv[off + e] = make_uint2(sidx[e], (unsigned)__float_as_int(snf[e]));
+            if (tid == 0) s_c2 = c;
+        } else {
+            // stage 2 over the list, one lane per window; survivors straight to the global list
+            const StageDev& sd = p.pstages[1];
+            const bool last = p.n_stages == 2;
             for (int e0 = warp * 32; e0 < c; e0 += THREADS) {
                 const int e = e0 + lane;
                 const bool act = e < c;
-                uint2 v = make_uint2(0u, 0u);
-                float sum = 0.0f;
+                int idx = 0;
+                float nfw = 1.0f, sum = 0.0f;
                 if (act) {
-                    v = lin[e];
-                    const int idx = (int)v.x;
+                    idx = sidx[e];
+                    nfw = snf[e];
                     const int bo = (idx / TX) * STEP * TW + (idx % TX) * STEP;
-                    const float nfw = __int_as_float((int)v.y);
 #if FD_JIT_DEEP > 1
-                    if (s < FD_JIT_DEEP)
-                        sum = jit_deep(s, T + bo, nfw);
-                    else
+                    sum = jit_deep(1, T + bo, nfw);
+#else
+                    sum = sd.first + sd.n <= p.n_pstumps ? eval_stage(T, bo, nfw, prec, sd.first, sd.n, sd.mc)
+                                                         : eval_stage(T, bo, nfw, grec, sd.first, sd.n, sd.mc);
 #endif
-                        sum = sd.first + sd.n <= p.n_pstumps ? eval_stage(T, bo, nfw, prec, sd.first, sd.n, sd.mc)
-                                                             : eval_stage(T, bo, nfw, grec, sd.first, sd.n, sd.mc);
                 }
                 const bool pass = act && (sum >= sd.T);
-                if (act && !pass) out.reject(0, (int)v.x, s, sum);
+                if (act && !pass) out.reject(0, idx, 1, sum);
                 if (last) {
-                    if (pass) out.emit(0, (int)v.x, sum);
+                    if (pass) out.emit(0, idx, sum);
                     continue;
                 }
                 const unsigned m = __ballot_sync(0xffffffffu, pass);
                 if (m) {
                     int pos = 0;
-                    if (lane == 0) pos = atomicAdd(&s_c3[(s + 1) % 3], __popc(m));
+                    if (lane == 0) pos = atomicAdd(&s_c2, __popc(m));
                     pos = __shfl_sync(0xffffffffu, pos, 0);
-                    if (pass) lout[pos + __popc(m & ((1u << lane) - 1u))] = v;
+                    if (pass)
+                        p.surv[off + pos + __popc(m & ((1u << lane) - 1u))] =
+                            make_uint2((unsigned)idx, (unsigned)__float_as_int(nfw));
                 }
             }
-            __syncthreads();
-            c = last ? 0 : s_c3[(s + 1) % 3];
-        }
-        const uint2* lst = (s & 1) ? sv : sv2;    // the c windows entering stage s
-        if (p.s1_tail && c > 0) {
-            // hand the windows entering stage s to the tail queue (k_tail finishes them, one warp
-            // per window); what does not fit is finished here, one warp per window
-            if (tid == 0) {
-                if (p.stage_counts) atomicAdd(p.stage_counts + s, (unsigned long long)c);
-                s_off = (int)atomicAdd(p.tail_count, (unsigned)c);
-                p.tile_rec[tn] = make_uint2(0u, 0u);
-                if (p.stage_counts)
-                    atomicAdd(p.stage_counts, (unsigned long long)min(TX, nx - wx0) * (unsigned long long)min(TY, ny - wy0));
-            }
-            __syncthreads();
-            const int tpos = s_off;
-            const unsigned fl = ((unsigned)(s_frame[0] - p.frame_base) << 16) | ((unsigned)k << 8) | (unsigned)s;
-            for (int e = tid; e < c && tpos + e < p.tail_cap; e += THREADS) {
-                const uint2 v = lst[e];
-                const int idx = (int)v.x;
-                p.tail_q[tpos + e] = make_uint4(fl, ((unsigned)(wy0 + idx / TX) << 16) | (unsigned)(wx0 + idx % TX), v.y, 0u);
-            }
-            for (int e = warp; e < c; e += THREADS / 32) {
-                if (tpos + e < p.tail_cap) continue;
-                const uint2 v = lst[e];
-                const int idx = (int)v.x;
-                finish_window_warp<STEP, DEPTH>(p, T, (idx / TX) * STEP * TW + (idx % TX) * STEP,
-                                                __int_as_float((int)v.y), s, 0, idx, out);
-            }
-            continue;
         }
         if (tid == 0) {
-            const unsigned off = c ? atomicAdd(p.surv_count, (unsigned)c) : 0u;
-            p.tile_rec[tn] = make_uint2(off, (unsigned)c);
-            s_off = (int)off;
-            if (p.stage_counts)
-                atomicAdd(p.stage_counts, (unsigned long long)min(TX, nx - wx0) * (unsigned long long)min(TY, ny - wy0));
+            s_prev = tn;                          // tile_rec written after the next barrier (A)
+            s_prev_off = off;
         }
-        __syncthreads();
-        const int off = s_off;
-        for (int e = tid; e < c; e += THREADS) p.surv[off + e] = lst[e];
     }
 }
 

@@ -128,7 +128,6 @@ def test_depth_maps_generic_k2(monkeypatch):
 # K2 schedules (fd_api.cpp run_groups): every one computes the same depth maps and detections
 K2_SCHEDULES = {
     "stage1_only": {"FD_S0": "1"},                          # k_stage1 stage 1, k_deep1 from stage 2
-    "stage1_to_5_tail": {"FD_S0": "5", "FD_S1_TAIL": "1"},  # k_stage1 stages 1-5, then k_tail only
     "no_tail": {"FD_TAIL": "0"},                            # k_deep1 finishes every window
     "warp_specialised": {"FD_K2_WS": "1"},                  # k_ws
     "warp_specialised_s0_1": {"FD_K2_WS": "1", "FD_WS_S0": "1"},
