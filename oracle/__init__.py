@@ -52,6 +52,7 @@ def _load():
             L.fdo_plan.argtypes = [i32, i32, i32, dbl, i32, i32, P, P, P, P]
             L.fdo_resample.argtypes = [P, i32, i32, i32, dbl, i32, i32, P]
             L.fdo_integral.argtypes = [P, i32, i32, i32, P, P]
+            L.fdo_filter_binomial.argtypes = [P, i32, i32]
             L.fdo_rect_sum.restype = C.c_uint32
             L.fdo_rect_sum.argtypes = [P, i32, i32, i32, i32, i32]
             L.fdo_window_nf.restype = f32
@@ -130,6 +131,14 @@ def resample(frame: np.ndarray, f: float, Wk: int, Hk: int) -> np.ndarray:
     H, W = frame.shape
     out = np.zeros((Hk, Wk), np.uint8)
     _load().fdo_resample(_p(frame), W, H, W, float(f), Wk, Hk, _p(out))
+    return out
+
+
+def filter_binomial(img: np.ndarray) -> np.ndarray:
+    """f2 filtering stage (reading R3b): 3x3 binomial / 16, round half up, clamp-to-edge."""
+    out = np.array(img, dtype=np.uint8, order="C", copy=True)
+    H, W = out.shape
+    _load().fdo_filter_binomial(_p(out), W, H)
     return out
 
 

@@ -107,6 +107,18 @@ fdo_cascade* fdo_cascade_parse(const char* text, size_t len, char* err, int errl
     c->win_h = (int32_t)wh;
     if (!next_line(&cur, line, sizeof line)) PERR("line %d: missing stages", cur.line);
     s = line;
+    if (tok_word(&s, "filter")) {         /* optional: 'filter none' | 'filter binomial3' */
+        if (tok_word(&s, "binomial3") && at_end(s))
+            c->filter = 1;
+        else if (tok_word(&s, "none") && at_end(s))
+            c->filter = 0;
+        else
+            PERR("line %d: expected 'filter none' or 'filter binomial3'", cur.line);
+        if (!next_line(&cur, line, sizeof line)) PERR("line %d: missing stages", cur.line);
+        s = line;
+    } else {
+        s = line;
+    }
     if (!tok_word(&s, "stages") || !tok_long(&s, &v) || !at_end(s) || v < 1 || v > 4096)
         PERR("line %d: expected 'stages N' (1..4096)", cur.line);
     c->n_stages = (int32_t)v;
@@ -328,6 +340,34 @@ void fdo_eval_level(const fdo_cascade* c, const uint32_t* ii, const uint64_t* sq
 }
 
 /* ------------------------------------------------------------------------------------ */
+/* f2: filtering stage (P:L362-367 names it, gives no taps; reading R3b): binomial 3x3,     */
+/* out(x,y) = (sum_{i,j in -1..1} w_i w_j in(clamp(x+i), clamp(y+j)) + 8) >> 4,              */
+/* w_-1 = w_1 = 1, w_0 = 2, written out directly (no separable pass, no reordering).         */
+/* ------------------------------------------------------------------------------------ */
+
+void fdo_filter_binomial(uint8_t* img, int W, int H) {
+    static const int w[3] = {1, 2, 1};
+    uint8_t* src = (uint8_t*)malloc((size_t)W * H);
+    if (!src) return;
+    memcpy(src, img, (size_t)W * H);
+    for (int y = 0; y < H; ++y)
+        for (int x = 0; x < W; ++x) {
+            int sum = 0;
+            for (int j = -1; j <= 1; ++j)
+                for (int i = -1; i <= 1; ++i) {
+                    int xx = x + i, yy = y + j;
+                    if (xx < 0) xx = 0;
+                    if (xx > W - 1) xx = W - 1;
+                    if (yy < 0) yy = 0;
+                    if (yy > H - 1) yy = H - 1;
+                    sum += w[i + 1] * w[j + 1] * src[(size_t)yy * W + xx];
+                }
+            img[(size_t)y * W + x] = (uint8_t)((sum + 8) >> 4);
+        }
+    free(src);
+}
+
+/* ------------------------------------------------------------------------------------ */
 /* Whole path over frames: jobs = (frame, level), run on host threads, merged in order.  */
 /* ------------------------------------------------------------------------------------ */
 
@@ -369,6 +409,7 @@ static void run_job(run_t* R, int job) {
         goto done;
     }
     fdo_resample(frame, R->W, R->H, R->pitch, R->f[k], Wk, Hk, lvl);
+    if (R->c->filter) fdo_filter_binomial(lvl, Wk, Hk);
     fdo_integral(lvl, Wk, Hk, Wk, ii, sq);
     fdo_eval_level(R->c, ii, sq, Wk, Hk, R->step, dep, sco, nr);
     if (own) {

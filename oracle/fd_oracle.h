@@ -27,6 +27,7 @@ typedef struct { int32_t nrect; fdo_rect r[3]; float theta, left, right; } fdo_s
 typedef struct { int32_t n, first; float T; } fdo_stage;
 typedef struct {
     int32_t win_w, win_h, n_stages, n_stumps;
+    int32_t filter;          /* 0: identity; 1: binomial 3x3 after scaling (.fdc 'filter binomial3') */
     fdo_stage* stages;
     fdo_stump* stumps;
 } fdo_cascade;
@@ -37,6 +38,11 @@ typedef struct {
     float score;
     int32_t aux;
 } fdo_detection;
+
+/* f2: the filtering stage between scaling and the integral image (P:L362-367,
+ * taps not given; reading R3b): 3x3 binomial [1 2 1]^T [1 2 1] / 16 with round-half-up
+ * ((sum + 8) >> 4) and clamp-to-edge, in place on a W x H (pitch W) level image. */
+void fdo_filter_binomial(uint8_t* img, int W, int H);
 
 /* .fdc text -> cascade (NULL on error, message in err). */
 fdo_cascade* fdo_cascade_parse(const char* text, size_t len, char* err, int errlen);

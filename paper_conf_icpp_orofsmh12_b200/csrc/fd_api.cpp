@@ -162,6 +162,7 @@ bool parse_float(const std::string& t, float* v, bool allow_inf) {
 
 struct fd_cascade_s {
     int device = 0;
+    int filter = 0;                         // filtering stage after scaling: 0 none, 1 binomial 3x3
     std::vector<HStump> stumps;
     std::vector<HStage> stages;
     std::mutex mu;
@@ -229,6 +230,15 @@ fd_status parse_cascade(const char* text, size_t len, fd_cascade_s* c) {
     if (!L || L->tok.size() != 3 || L->tok[0] != "window" || L->tok[1] != "24" || L->tok[2] != "24")
         return fail(FD_EFORMAT, "line %d: expected 'window 24 24'", L ? L->no : 0);
     L = need("stages");
+    if (L && !L->tok.empty() && L->tok[0] == "filter") {      // optional filtering stage (f2, reading R3b)
+        if (L->tok.size() == 2 && L->tok[1] == "binomial3")
+            c->filter = 1;
+        else if (L->tok.size() == 2 && L->tok[1] == "none")
+            c->filter = 0;
+        else
+            return fail(FD_EFORMAT, "line %d: expected 'filter none' or 'filter binomial3'", L->no);
+        L = need("stages");
+    }
     long ns = 0;
     if (!L || L->tok.size() != 2 || L->tok[0] != "stages" || !parse_int(L->tok[1], &ns) || ns < 1 || ns > 250)
         return fail(FD_EFORMAT, "line %d: expected 'stages N' with 1 <= N <= 250", L ? L->no : 0);
@@ -568,6 +578,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     const int ngroups = (n + G - 1) / G;
     PlanDev& PD = *w->plan;
     make_plan_dev(pl, W, H, pitch, step, G, &PD);
+    PD.filter = c->filter;
     // two pipeline slots on two streams when there is more than one group (FD_PIPE=0: one)
     const int nslots = (ngroups > 1 && env_int("FD_PIPE", 1) != 0) ? 2 : 1;
     // K2 split in two kernels (k_stage1: dense first stage, k_deep: batched deeper stages;

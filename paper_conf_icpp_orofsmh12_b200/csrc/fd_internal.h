@@ -176,6 +176,7 @@ struct PlanDev {
     int k1tiles_per_frame;  // K1 tiles (band x chunk) per frame
     long long ws_elems;     // group workspace elements (all levels, all g)
     int G;                  // frames per group (tensor-map extent)
+    int filter;             // K1: 1 = binomial 3x3 filtering stage after scaling (f2)
     LevelDev lv[FD_MAX_LEVELS];
 };
 

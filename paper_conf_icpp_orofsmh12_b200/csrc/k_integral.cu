@@ -92,6 +92,7 @@ __device__ __forceinline__ int find_level_k1(const PlanDev& p, int t) {
 __global__ void __launch_bounds__(K1_THREADS) k_marg(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
                                                      K1Scratch s) {
     __shared__ uint32_t red_s[8][CHUNK], red_q[8][CHUNK];
+    __shared__ uint8_t raw[BAND + 2][CHUNK + 4];       // filtering stage: resampled rows with a 1-px halo
     const int g = blockIdx.y;
     const int k = find_level_k1(p, blockIdx.x);
     const LevelDev& L = p.lv[k];
@@ -110,12 +111,41 @@ __global__ void __launch_bounds__(K1_THREADS) k_marg(const uint8_t* __restrict__
     uint32_t cols[4] = {0, 0, 0, 0}, colq[4] = {0, 0, 0, 0};
     uint32_t* rowsum = s.row + (size_t)g * p.row_frame + L.row_off + (size_t)(b * L.nchunks + c) * 2 * BAND;
     uint8_t* lvl = s.lvl + (size_t)g * p.lvl_frame + L.lvl_off;
+    if (p.filter) {
+        // f2 filtering stage (reading R3b): the resampled level at rows y0-1 .. y0+rows and columns
+        // x0-1 .. x0+CHUNK, clamped to the level (clamp-to-edge), then the 3x3 binomial below
+        for (int r = warp; r < rows + 2; r += K1_THREADS / 32) {
+            const int yy = min(max(y0 - 1 + r, 0), L.H - 1);
+            for (int q = lane; q < CHUNK + 2; q += 32) {
+                const int xx = min(max(x0 - 1 + q, 0), L.W - 1);
+                raw[r][q] = (uint8_t)level_pixel(frame, p.pitch, p.W, p.H, L.r16, xx, yy);
+            }
+        }
+        __syncthreads();
+    }
 #pragma unroll
     for (int i = 0; i < BAND / 8; ++i) {
         const int r = warp + 8 * i;
         if (r < rows) {
             uint32_t pv[4];
-            tile_row_pixels(frame, p, L, y0 + r, x, cs, pv);
+            if (p.filter) {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const int q = x + j - x0 + 1;            // raw column of pixel x + j
+                    uint32_t v = 0;
+                    if (x + j < L.W) {
+#pragma unroll
+                        for (int dy = 0; dy < 3; ++dy) {
+                            const uint32_t h = raw[r + dy][q - 1] + 2u * raw[r + dy][q] + raw[r + dy][q + 1];
+                            v += (dy == 1 ? 2u : 1u) * h;
+                        }
+                        v = (v + 8u) >> 4;
+                    }
+                    pv[j] = v;
+                }
+            } else {
+                tile_row_pixels(frame, p, L, y0 + r, x, cs, pv);
+            }
             if (x < L.P)       // level image row, 4 pixels per lane as one aligned word (0 past W)
                 *reinterpret_cast<uint32_t*>(lvl + (size_t)(y0 + r) * L.P + x) =
                     pv[0] | (pv[1] << 8) | (pv[2] << 16) | (pv[3] << 24);

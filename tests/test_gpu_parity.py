@@ -153,6 +153,31 @@ def test_k2_schedules(name, jit, monkeypatch):
     compare_depth(cascades(3), fr, 1.1)
 
 
+def filtered(cfg):
+    """The cfg cascade with the f2 filtering stage switched on ('filter binomial3')."""
+    key = ("filtered", cfg)
+    if key not in _casc:
+        text = open(os.path.join(ROOT, "cascades", f"c{cfg}.fdc")).read()
+        text = text.replace("window 24 24\n", "window 24 24\nfilter binomial3\n", 1)
+        _casc[key] = (fd.Cascade(text), oracle.Cascade(text))
+    return _casc[key]
+
+
+@pytest.mark.parametrize("cfg,W,H,s", [(1, 320, 240, 1.25), (2, 640, 480, 1.2), (2, 131, 517, 1.17),
+                                       (2, 401, 37, 1.3), (3, 1920, 1080, 1.1)])
+def test_filter_stage_bit_exact(cfg, W, H, s):
+    """f2: with the binomial filtering stage the depth maps (hence K1's filtered levels and
+    integral images) and the detections equal the oracle's bit for bit."""
+    n = 1 if cfg == 3 else 2
+    fr = np.stack([fdgen.background(cfg, 700 + i, W, H) for i in range(n)]) if (W, H) != CFG[cfg][:2] \
+        else gen(cfg, 9, n)[0]
+    compare_depth(filtered(cfg), fr, s)
+    gc, oc = filtered(cfg)
+    got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1, capacity=1 << 20))
+    ref, _ = oracle.detect(oc, fr, 24, s, 1, nthreads=os.cpu_count())
+    assert np.array_equal(got, ref)
+
+
 def test_c6_workload_1080p():
     """f3 workload: the OpenCV-shaped 2913-stump cascade on c4 frames -- depth maps bit-exact,
     detections identical, stage counters equal to the oracle's depth histogram."""

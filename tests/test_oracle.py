@@ -284,6 +284,36 @@ def test_all_pass_and_all_reject_cascades():
     assert len(d) == 2 * tot and (d == 0).all() and (sc == 0.5).all()
 
 
+def test_filter_binomial_pins():
+    """f2 filtering stage (reading R3b): weights sum to 16, so constants are fixed points; the
+    binomial kernel reproduces linear functions exactly away from the border; an impulse gives
+    the 1-2-1 x 1-2-1 stencil with round-half-up; clamp-to-edge at the border (hand values)."""
+    c = np.full((30, 40), 173, np.uint8)
+    assert np.array_equal(oracle.filter_binomial(c), c)
+    x = np.arange(40)
+    ramp = np.tile((3 * x + 7).astype(np.uint8), (30, 1))
+    f = oracle.filter_binomial(ramp)
+    assert np.array_equal(f[:, 1:-1], ramp[:, 1:-1])
+    # left border: (1*7 + 2*7 + 1*10) * 4 / 16 = 7.75 -> (124 + 8) >> 4 = 8; right: 124,124,121 -> 123
+    assert (f[:, 0] == 8).all() and (f[:, -1] == ((4 * (124 + 2 * 124 + 121) + 8) >> 4)).all()
+    imp = np.zeros((7, 7), np.uint8)
+    imp[3, 3] = 255
+    want = np.zeros((7, 7), np.uint8)
+    want[2:5, 2:5] = [[16, 32, 16], [32, 64, 32], [16, 32, 16]]
+    assert np.array_equal(oracle.filter_binomial(imp), want)
+    # a cascade with 'filter binomial3' evaluates on filtered levels: a constant frame stays
+    # constant, so every window has nf = 1 and the same depth as without the filter
+    st = ([(1, 1, 10, 10, -1), (1, 1, 5, 10, 2)], 0.1, 0.5, -0.5)
+    text = cascade_text([(0.0, [st])])
+    filt = text.replace("window 24 24\n", "window 24 24\nfilter binomial3\n")
+    fr = np.full((1, 48, 64), 90, np.uint8)
+    a, _, _ = oracle.detect_depth(oracle.Cascade(text), fr, 24, 1.25, 1)
+    b, _, _ = oracle.detect_depth(oracle.Cascade(filt), fr, 24, 1.25, 1)
+    assert np.array_equal(a, b)
+    with pytest.raises(Exception):
+        oracle.Cascade(text.replace("window 24 24\n", "window 24 24\nfilter gauss\n"))
+
+
 def test_c6_cascade_shape():
     """f3 workload: the OpenCV-shaped cascade has the paper's "25 stages ... 2913 weak
     classifiers" (P:L1106-1110) and only Table I features (2 or 3 rectangles)."""
