@@ -132,6 +132,7 @@ K2_SCHEDULES = {
     "warp_specialised": {"FD_K2_WS": "1"},                  # k_ws
     "warp_specialised_s0_1": {"FD_K2_WS": "1", "FD_WS_S0": "1"},
     "fused": {"FD_K2_SPLIT": "0"},                          # k_cascade
+    "batched_deep": {"FD_K2_DEEP1": "0"},                   # k_stage1 + batched k_deep
     "one_slot_pipeline": {"FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
     "two_slot_pipeline": {"FD_GROUP_FRAMES": "1"},          # 3 frame groups over 2 slots/streams
 }
