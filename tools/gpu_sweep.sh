@@ -1,7 +1,9 @@
-# usage: bash tools/gpu_sweep.sh VAR v1 v2 ... -- bench K2 ms per setting of an env variable
-var=$1; shift
+# Bench A/B sweep on one B200: each argument is a set of environment settings for one run, e.g.
+#   bash tools/gpu_sweep.sh "FD_PIPE=0" "FD_PIPE=1" "FD_K2_WS=1 FD_PIPE=0"
+# FRAMES (default 512) frames per step, 3 timed steps, 2 warm-up; prints fps and per-kernel ms.
 mkdir -p gpurun_out
-for v in "$@"; do
-  env $var=$v timeout 300 python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu > gpurun_out/sw.json 2>gpurun_out/sw.err
-  python -c "import json;d=json.load(open('gpurun_out/sw.json'));k=d['kernel_ms_per_step'];print('$var=$v', round(d['value'],1), {a:round(b,2) for a,b in k.items()})" || tail -5 gpurun_out/sw.err
+for cfg in "$@"; do
+  env $cfg timeout 300 python bench.py --frames "${FRAMES:-512}" --steps 3 --warmup 2 --no-cpu --no-e2e \
+    > gpurun_out/sw.json 2> gpurun_out/sw.err || tail -3 gpurun_out/sw.err
+  python -c "import json;d=json.load(open('gpurun_out/sw.json'));k=d['kernel_ms_per_step'];print('$cfg', round(d['value'],1), {a: round(b, 2) for a, b in k.items()})"
 done
