@@ -217,7 +217,7 @@ def run_reference(args):
     out = {"impl": "reference", "metric": METRIC, "value": v, "unit": "frames/s", "n_gpus": args.gpus,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * dt / args.steps,
            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32+f32",
-           "data": "synthetic", "config": workload_config(1, 1),
+           "data": "synthetic", "config": workload_config(args.frames, 1),
            "cpu_baseline": {"value": v, "unit": "frames/s", "cores": cores, "kind": "oracle",
                             "sample": f"1 frame per step ({args.steps} timed, {args.warmup} warm-up) of the c4 "
                                       "workload, plain C oracle, detect + group, threads over (frame, level)"},
