@@ -82,7 +82,8 @@ def _p(a: np.ndarray):
 
 class _CascadeC(C.Structure):
     _fields_ = [("win_w", C.c_int32), ("win_h", C.c_int32), ("n_stages", C.c_int32),
-                ("n_stumps", C.c_int32), ("stages", C.c_void_p), ("stumps", C.c_void_p)]
+                ("n_stumps", C.c_int32), ("filter", C.c_int32), ("soft", C.c_int32),
+                ("stages", C.c_void_p), ("stumps", C.c_void_p)]
 
 
 class Cascade:

@@ -119,6 +119,14 @@ fdo_cascade* fdo_cascade_parse(const char* text, size_t len, char* err, int errl
     } else {
         s = line;
     }
+    if (tok_word(&s, "soft")) {           /* optional: soft cascade (f4, reading R8b) */
+        if (!at_end(s)) PERR("line %d: expected 'soft'", cur.line);
+        c->soft = 1;
+        if (!next_line(&cur, line, sizeof line)) PERR("line %d: missing stages", cur.line);
+        s = line;
+    } else {
+        s = line;
+    }
     if (!tok_word(&s, "stages") || !tok_long(&s, &v) || !at_end(s) || v < 1 || v > 4096)
         PERR("line %d: expected 'stages N' (1..4096)", cur.line);
     c->n_stages = (int32_t)v;
@@ -293,7 +301,11 @@ void fdo_window_nf_values(const uint32_t* ii, const uint64_t* sqii, int P,
 }
 
 /* c7 stump (GentleBoost regression stump [6]) and c8 stages with early
- * rejection: sum = sum + leaf in stump order (fp32), pass iff sum >= T. */
+ * rejection: sum = sum + leaf in stump order (fp32), pass iff sum >= T.
+ * Soft cascade (f4; the paper's future work, ref [32] Bourdev & Brandt; reading
+ * R8b): the sum is NOT restarted at a stage boundary -- it runs over every stump evaluated so
+ * far and T_s is the rejection threshold of the running sum after stage s (one-stump stages
+ * give the per-stump rejection trace of [32]). */
 int fdo_eval_window(const fdo_cascade* c, const uint32_t* ii, const uint64_t* sqii, int P,
                     int wx, int wy, float* score, int* near) {
     const float nf = fdo_window_nf(ii, sqii, P, wx, wy);
@@ -301,7 +313,7 @@ int fdo_eval_window(const fdo_cascade* c, const uint32_t* ii, const uint64_t* sq
     float sum = 0.0f;
     for (int s = 0; s < c->n_stages; ++s) {
         const fdo_stage* st = &c->stages[s];
-        sum = 0.0f;
+        if (!c->soft) sum = 0.0f;
         for (int j = 0; j < st->n; ++j) {
             const fdo_stump* sp = &c->stumps[st->first + j];
             const int32_t f = fdo_feature(ii, P, wx, wy, sp->r, sp->nrect);

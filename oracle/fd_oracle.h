@@ -28,6 +28,8 @@ typedef struct { int32_t n, first; float T; } fdo_stage;
 typedef struct {
     int32_t win_w, win_h, n_stages, n_stumps;
     int32_t filter;          /* 0: identity; 1: binomial 3x3 after scaling (.fdc 'filter binomial3') */
+    int32_t soft;            /* 0: stage sums restart at 0 (R8); 1: soft cascade (.fdc 'soft'), the sum runs
+                                over all stumps and T_s is a rejection threshold on the running sum (R8b) */
     fdo_stage* stages;
     fdo_stump* stumps;
 } fdo_cascade;

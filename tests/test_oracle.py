@@ -27,9 +27,9 @@ def _golden(name):
     return rows
 
 
-def cascade_text(stages):
-    """stages: list of (T, [ (rects, theta, left, right), ... ])"""
-    out = ["FDC 1", "window 24 24", f"stages {len(stages)}"]
+def cascade_text(stages, soft=False):
+    """stages: list of (T, [ (rects, theta, left, right), ... ]); soft: soft cascade (R8b)"""
+    out = ["FDC 1", "window 24 24"] + (["soft"] if soft else []) + [f"stages {len(stages)}"]
     for T, stumps in stages:
         out.append(f"stage {len(stumps)} {float(T)!r}" if math.isfinite(T) else f"stage {len(stumps)} {'inf' if T > 0 else '-inf'}")
         for rects, th, l, r in stumps:
@@ -268,6 +268,80 @@ def test_stage_pass_on_equality_and_early_exit():
     casc = oracle.Cascade(cascade_text([(0.5, [st, st]), (0.26, [st]), (-1.0, [st])]))
     d, score, near = oracle.eval_window(casc, ii, sq, 0, 0)
     assert d == 1 and score == np.float32(0.25)
+
+
+def test_soft_cascade_worked_example():
+    """f4 soft cascade (ref [32]; reading R8b) on the c7 worked-example window,
+    hand-computed: leaves 0.5 then 0.25 (both 'left', f = -61710 < theta*nf = -36720).
+    Hard: stage 2 sum 0.25 < 0.7 -> depth 1, score 0.25.  Soft: running sum 0.5 >= 0.4, then
+    0.75 >= 0.7 -> accepted, depth 2, score 0.75.  With T_2 = 0.8: 0.75 < 0.8 -> depth 1, 0.75."""
+    ii, sq = oracle.integral(_worked_window())
+    edge = [(1, 1, 22, 22, -1), (1, 1, 11, 22, 2)]
+    stages = [(0.4, [(edge, -0.5, 0.5, -1.0)]), (0.7, [(edge, -0.5, 0.25, -1.0)])]
+    d, score, _ = oracle.eval_window(oracle.Cascade(cascade_text(stages)), ii, sq, 0, 0)
+    assert d == 1 and score == np.float32(0.25)
+    d, score, _ = oracle.eval_window(oracle.Cascade(cascade_text(stages, soft=True)), ii, sq, 0, 0)
+    assert d == 2 and score == np.float32(0.75)
+    stages[1] = (0.8, stages[1][1])
+    d, score, _ = oracle.eval_window(oracle.Cascade(cascade_text(stages, soft=True)), ii, sq, 0, 0)
+    assert d == 1 and score == np.float32(0.75)
+
+
+def _soft_from_c2(n_stages=8):
+    """A soft cascade built from the first stages of the c2 cascade: the running-sum threshold
+    of stage s is the sum of the hard thresholds up to s (so pass rates stay meaningful)."""
+    lines = open(os.path.join(ROOT, "cascades", "c2.fdc")).read().splitlines()
+    out, s, acc, body = [], -1, 0.0, []
+    for ln in lines:
+        t = ln.split()
+        if not t or t[0] in ("FDC", "window", "stages"):
+            continue
+        if t[0] == "stage":
+            s += 1
+            if s >= n_stages:
+                break
+            acc += float.fromhex(t[2]) if "0x" in t[2] else float(t[2])
+            body.append(f"stage {t[1]} {np.float32(acc).item()!r}")
+        elif s < n_stages:
+            body.append(ln)
+    return "\n".join(["FDC 1", "window 24 24", "soft", f"stages {n_stages}"] + body) + "\n"
+
+
+def test_soft_cascade_equals_prefix_hard_cascades():
+    """R8b pinned against the hard-cascade definition (R8, itself pinned above): the soft running
+    sum after stage t is the fp32 sequential sum of the leaves of stumps 1..S_t in order, i.e.
+    the score of a ONE-stage hard cascade holding those stumps with T = -inf.  So the soft depth
+    of a window is the first t with that prefix score < T_t, and its score is that prefix score
+    (the full sum if every stage passes).  Checked on every window of a 160x120 frame."""
+    W, H, s = 160, 120, 1.25
+    fr, _ = fdgen.frames(2, 5, 1, W, H)
+    soft_text = _soft_from_c2(6)
+    soft = oracle.Cascade(soft_text)
+    d, sc, _ = oracle.detect_depth(soft, fr, 24, s, 1, nthreads=4)
+    lines = soft_text.splitlines()
+    stage_rows = [i for i, ln in enumerate(lines) if ln.startswith("stage ")]
+    T = [float(lines[i].split()[2]) for i in stage_rows]
+    prefix_scores = []
+    for t in range(len(stage_rows)):
+        end = stage_rows[t + 1] if t + 1 < len(stage_rows) else len(lines)
+        stumps = [ln for ln in lines[stage_rows[0]:end] if ln.startswith("stump ")]
+        hard = "\n".join(["FDC 1", "window 24 24", "stages 1", f"stage {len(stumps)} -inf"] + stumps) + "\n"
+        _, ps, _ = oracle.detect_depth(oracle.Cascade(hard), fr, 24, s, 1, nthreads=4)
+        prefix_scores.append(ps)
+    P = np.stack(prefix_scores)                      # [stages, windows]
+    fail = P < np.asarray(T, np.float32)[:, None]
+    exp_d = np.where(fail.any(axis=0), fail.argmax(axis=0), len(T))
+    exp_sc = P[np.minimum(exp_d, len(T) - 1), np.arange(P.shape[1])]
+    assert np.array_equal(d, exp_d.astype(d.dtype))
+    assert np.array_equal(sc.view(np.uint32), exp_sc.view(np.uint32))
+    # non-trivial: windows stop at several depths and some pass everything
+    assert len(np.unique(d)) >= 4
+    # a one-stage soft cascade is the hard cascade
+    one = "\n".join(lines[:stage_rows[1]]) + "\n"
+    one = one.replace("stages 6", "stages 1")
+    d1, s1, _ = oracle.detect_depth(oracle.Cascade(one), fr, 24, s, 1, nthreads=4)
+    d0, s0, _ = oracle.detect_depth(oracle.Cascade(one.replace("soft\n", "")), fr, 24, s, 1, nthreads=4)
+    assert np.array_equal(d1, d0) and np.array_equal(s1.view(np.uint32), s0.view(np.uint32))
 
 
 def test_all_pass_and_all_reject_cascades():
