@@ -49,9 +49,10 @@ def parse_args():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=2, help="frames timed on the CPU oracle")
-    ap.add_argument("--cascade", default="c3", choices=["c3", "c6"],
+    ap.add_argument("--cascade", default="c3", choices=["c3", "c6", "c3s"],
                     help="c3: the paper-shaped 1446-stump cascade (c4 workload, default); c6: the "
-                         "OpenCV-shaped 2913-stump cascade (SURVEY 8(f) f3 workload)")
+                         "OpenCV-shaped 2913-stump cascade (SURVEY 8(f) f3 workload); c3s: c3 as a soft "
+                         "cascade (SURVEY 8(f) f4, reading R8b, k_soft)")
     return ap.parse_args()
 
 
@@ -182,7 +183,8 @@ def make_frames(rank: int, n: int, plan):
 
 
 CASCADES = {"c3": ("c4", "25-stage 1446-stump cascade (cascades/c3.fdc)"),
-            "c6": ("c6", "OpenCV-shaped 25-stage 2913-stump cascade (cascades/c6.fdc)")}
+            "c6": ("c6", "OpenCV-shaped 25-stage 2913-stump cascade (cascades/c6.fdc)"),
+            "c3s": ("c4-soft", "25-stage 1446-stump soft cascade (cascades/c3s.fdc, running-sum thresholds)")}
 
 
 def workload_config(frames_per_gpu: int, world: int):
@@ -324,6 +326,10 @@ def run_ours(args):
         r["frac"] = r["achieved"] / issue_peak if r["achieved"] else None
     tr_s1, tr_deep, tr_k1 = ncu_traffic()
     roof1["traffic"], roofd["traffic"] = tr_s1, tr_deep
+    if CFG["cascade"] == "c3s.fdc":       # one kernel, k_soft, runs every stage
+        roof1.update(kernel="k_soft (K2, all stages, soft cascade)", algorithmic_ops_per_launch=(ops1 + opsd) / n1,
+                     achieved=(ops1 + opsd) / (t1 / 1e3) / 1e9 if t1 else None, traffic=None)
+        roof1["frac"] = roof1["achieved"] / issue_peak if roof1["achieved"] else None
     dominant, other = (roofd, roof1) if td > t1 else (roof1, roofd)
     k1_ms = prof["colsum"][1] + prof["carry"][1] + prof["band"][1]
     k1_bytes = level_bytes(plan) * F * args.steps

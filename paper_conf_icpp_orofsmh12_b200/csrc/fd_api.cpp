@@ -163,6 +163,7 @@ bool parse_float(const std::string& t, float* v, bool allow_inf) {
 struct fd_cascade_s {
     int device = 0;
     int filter = 0;                         // filtering stage after scaling: 0 none, 1 binomial 3x3
+    int soft = 0;                           // 1: soft cascade (f4, reading R8b), stage sums carried over
     std::vector<HStump> stumps;
     std::vector<HStage> stages;
     std::mutex mu;
@@ -237,6 +238,11 @@ fd_status parse_cascade(const char* text, size_t len, fd_cascade_s* c) {
             c->filter = 0;
         else
             return fail(FD_EFORMAT, "line %d: expected 'filter none' or 'filter binomial3'", L->no);
+        L = need("stages");
+    }
+    if (L && !L->tok.empty() && L->tok[0] == "soft") {        // optional soft cascade (f4, reading R8b)
+        if (L->tok.size() != 1) return fail(FD_EFORMAT, "line %d: expected 'soft'", L->no);
+        c->soft = 1;
         L = need("stages");
     }
     long ns = 0;
@@ -586,12 +592,15 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     // default (FD_K2_SPLIT=1): k_stage1 + k_deep1 (+ k_tail).  FD_K2_WS=1: the warp-specialised
     // k_ws (stage-1 and deep warp groups in one kernel; measured slower on B200, kept as an
     // alternative schedule under the same parity tests); FD_K2_SPLIT=0: the fused k_cascade
-    const bool wsk = env_int("FD_K2_WS", 0) != 0;
-    const bool split = !wsk && env_int("FD_K2_SPLIT", 1) != 0;
+    // a soft cascade (R8b) runs its own schedule, k_soft (k_soft.cu): one lane per window, the
+    // running sum carried across stages, no survivor lists, no tail queue, no specialisation
+    const bool soft = c->soft != 0;
+    const bool wsk = !soft && env_int("FD_K2_WS", 0) != 0;
+    const bool split = !soft && !wsk && env_int("FD_K2_SPLIT", 1) != 0;
     const bool deep1 = env_int("FD_K2_DEEP1", 1) != 0;      // k_deep1 (tile per small CTA) or batched k_deep
     // tail queue (k_tail): FD_TAIL=0 keeps every window inside K2; FD_TAIL_N = windows left in a
     // batch at which it hands them over; FD_TAIL_CAP = queue entries (16 B each) per group
-    const bool use_tail = env_int("FD_TAIL", 1) != 0;
+    const bool use_tail = !soft && env_int("FD_TAIL", 1) != 0;
     const int tail_cap = use_tail ? std::max(1024, env_int("FD_TAIL_CAP", 1 << 22)) : 0;
     K1Scratch k1s[2];
     std::vector<CUtensorMap> maps((size_t)PD.n_levels);
@@ -670,7 +679,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     TP.stage_counts = d_stage_counts;
     // step 1: the K2 specialised for this cascade (compiled once, FD_JIT=0 selects the generic kernel)
     JitK2* jit = nullptr;
-    if (step == 1 && env_int("FD_JIT", 1) != 0) {
+    if (step == 1 && !soft && env_int("FD_JIT", 1) != 0) {
         std::lock_guard<std::mutex> lk(c->mu);
         if (!c->jit_tried) {
             c->jit_tried = true;
@@ -715,7 +724,9 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         P.surv = split ? sl.surv.as<uint2>() : nullptr;
         P.tile_rec = split ? sl.tilerec.as<uint2>() : nullptr;
         const int gr = grid < P.total_tiles ? grid : P.total_tiles;
-        if (jit) {
+        if (soft) {
+            LAUNCH(FD_K_CASCADE, gs, launch_soft(P, depth, step, gs));
+        } else if (jit) {
             std::string err;
             cudaError_t e;
             {

@@ -11,6 +11,7 @@ import pytest
 
 import fdgen
 import oracle
+import softcasc
 
 torch = pytest.importorskip("torch")
 import paper_conf_icpp_orofsmh12_b200 as fd  # noqa: E402
@@ -339,6 +340,67 @@ def test_three_rect_and_one_rect_stumps():
     text = _casc_text([("-0.5", stumps[:2]), ("0.1", stumps[2:]), ("-0.2", stumps)])
     fr = np.stack([fdgen.background(3, 70 + i, 300, 200) for i in range(2)])
     compare_depth((fd.Cascade(text), oracle.Cascade(text)), fr, 1.15)
+
+
+# ------------------------------------------------------------------ f4: soft cascade (k_soft)
+def test_soft_worked_example():
+    """Reading R8b, hand-computed (tests/test_oracle.py test_soft_cascade_worked_example): the
+    worked-example window at (5, 3) gives leaves 0.5 then 0.25; hard: depth 1, score 0.25;
+    soft: running sum 0.75 >= 0.7, depth 2, score 0.75."""
+    img = np.full((30, 40), 0, np.uint8)
+    img[3:27, 5 + 12:5 + 24] = 255
+    edge = [(1, 1, 22, 22, -1), (1, 1, 11, 22, 2)]
+    body = _casc_text([("0.4", [(edge, -0.5, 0.5, -1.0)]), ("0.7", [(edge, -0.5, 0.25, -1.0)])])
+    soft = body.replace("window 24 24\n", "window 24 24\nsoft\n")
+    nx = 40 - 24 + 1
+    fr = torch.from_numpy(img[None]).cuda()
+    d, sc = fd.fd_detect_depth(fd.Cascade(body), fr, 24, 1.5, 1)
+    assert int(d.cpu()[3 * nx + 5]) == 1 and float(sc.cpu()[3 * nx + 5]) == 0.25
+    d, sc = fd.fd_detect_depth(fd.Cascade(soft), fr, 24, 1.5, 1)
+    assert int(d.cpu()[3 * nx + 5]) == 2 and float(sc.cpu()[3 * nx + 5]) == 0.75
+    od, osc, _ = oracle.detect_depth(oracle.Cascade(soft), img, 24, 1.5, 1)
+    assert np.array_equal(d.cpu().numpy(), od) and np.array_equal(sc.cpu().numpy(), osc)
+
+
+@pytest.mark.parametrize("cfg,name,n_st,per_stump,W,H,s,step", [
+    (1, "c1.fdc", None, False, None, None, None, 1),
+    (1, "c1.fdc", None, True, None, None, None, 1),       # one-stump stages: per-stump rejection trace
+    (2, "c2.fdc", None, False, None, None, None, 1),
+    (2, "c2.fdc", 6, True, 131, 517, 1.17, 1),            # ragged size, 180 one-stump stages
+    (2, "c2.fdc", None, False, None, None, None, 2),
+    (2, "c2.fdc", 10, False, 401, 37, 1.3, 3),
+])
+def test_soft_depth_maps_bit_exact(cfg, name, n_st, per_stump, W, H, s, step):
+    text = softcasc.soft_from(name, n_st, per_stump)
+    fr, _ = gen(cfg, 21, 2, W, H, s)
+    s = s or CFG[cfg][2]
+    gd, od = compare_depth((fd.Cascade(text), oracle.Cascade(text)), fr, s, step)
+    assert np.array_equal(gd, od) and len(np.unique(od)) >= 3
+
+
+def test_soft_bench_cascade_1080p():
+    """cascades/c3s.fdc (the `bench.py --cascade c3s` workload: calibrated running-sum thresholds)
+    on a 1080p frame with planted faces: depth map and scores bit-exact against the oracle."""
+    text = open(os.path.join(ROOT, "cascades", "c3s.fdc")).read()
+    fr, _ = gen(3, 41, 1)
+    gd, od = compare_depth((fd.Cascade(text), oracle.Cascade(text)), fr, CFG[3][2])
+    assert np.array_equal(gd, od) and (od == 25).any()
+
+
+def test_soft_detections_1080p():
+    """The full 25-stage c3 cascade as a soft cascade at 1080p: detection lists (sorted, back-
+    projected, with scores) identical to the oracle, and the stage counters equal to the oracle's
+    depth histogram."""
+    text = softcasc.soft_from("c3.fdc")
+    W, H, s, _ = CFG[3]
+    fr, _ = gen(3, 31, 1)
+    gc, oc = fd.Cascade(text), oracle.Cascade(text)
+    sc = torch.zeros(gc.n_stages + 1, dtype=torch.int64, device="cuda")
+    got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1, capacity=1 << 22, stage_counts=sc))
+    ref, _ = oracle.detect(oc, fr, 24, s, 1, nthreads=os.cpu_count())
+    assert len(ref) > 0 and np.array_equal(got, ref), f"{len(got)} vs {len(ref)} detections"
+    od, _, _ = oracle.detect_depth(oc, fr, 24, s, 1, nthreads=os.cpu_count())
+    assert sc.cpu().tolist() == [int((od >= k).sum()) for k in range(gc.n_stages + 1)]
 
 
 # ------------------------------------------------------------------ K4: grouping

@@ -12,6 +12,7 @@ import pytest
 
 import fdgen
 import oracle
+import softcasc
 
 GOLD = os.path.join(os.path.dirname(__file__), "golden")
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -287,26 +288,6 @@ def test_soft_cascade_worked_example():
     assert d == 1 and score == np.float32(0.75)
 
 
-def _soft_from_c2(n_stages=8):
-    """A soft cascade built from the first stages of the c2 cascade: the running-sum threshold
-    of stage s is the sum of the hard thresholds up to s (so pass rates stay meaningful)."""
-    lines = open(os.path.join(ROOT, "cascades", "c2.fdc")).read().splitlines()
-    out, s, acc, body = [], -1, 0.0, []
-    for ln in lines:
-        t = ln.split()
-        if not t or t[0] in ("FDC", "window", "stages"):
-            continue
-        if t[0] == "stage":
-            s += 1
-            if s >= n_stages:
-                break
-            acc += float.fromhex(t[2]) if "0x" in t[2] else float(t[2])
-            body.append(f"stage {t[1]} {np.float32(acc).item()!r}")
-        elif s < n_stages:
-            body.append(ln)
-    return "\n".join(["FDC 1", "window 24 24", "soft", f"stages {n_stages}"] + body) + "\n"
-
-
 def test_soft_cascade_equals_prefix_hard_cascades():
     """R8b pinned against the hard-cascade definition (R8, itself pinned above): the soft running
     sum after stage t is the fp32 sequential sum of the leaves of stumps 1..S_t in order, i.e.
@@ -315,7 +296,7 @@ def test_soft_cascade_equals_prefix_hard_cascades():
     (the full sum if every stage passes).  Checked on every window of a 160x120 frame."""
     W, H, s = 160, 120, 1.25
     fr, _ = fdgen.frames(2, 5, 1, W, H)
-    soft_text = _soft_from_c2(6)
+    soft_text = softcasc.soft_from("c2.fdc", 6)
     soft = oracle.Cascade(soft_text)
     d, sc, _ = oracle.detect_depth(soft, fr, 24, s, 1, nthreads=4)
     lines = soft_text.splitlines()
