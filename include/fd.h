@@ -79,10 +79,13 @@ typedef struct {
 } fd_plan;
 
 /* Parse a cascade in .fdc text (format in DESIGN.md "Cascade format": FDC 1 / window 24 24 /
- * optional "filter none|binomial3" / stages N / per stage "stage n T" / per stump
- * "stump r (x y w h wt)*r theta left right").  "filter binomial3" switches on the filtering
+ * optional "filter none|binomial3" / optional "soft" / stages N / per stage "stage n T" / per
+ * stump "stump r (x y w h wt)*r theta left right").  "filter binomial3" switches on the filtering
  * stage between scaling and the integral images (reading R3b) for
  * fd_detect / fd_detect_depth with this cascade; fd_build_pyramid and fd_integral are unfiltered.
+ * "soft" makes it a soft cascade (the paper's future work, ref [32]; SURVEY 8(f)
+ * f4, reading R8b): the stage sum is not restarted, T_s thresholds the running sum over every
+ * stump so far; depth = stages passed, score = the running sum at exit.  At most 250 stages.
  * Stages of growing size evaluated in order with early rejection;
  * stumps are GentleBoost regression stumps on Haar features.
  * Uploads the packed cascade to the CURRENT device.  text need not be NUL-terminated.
