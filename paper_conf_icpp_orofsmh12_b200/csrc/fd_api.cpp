@@ -594,13 +594,15 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     // alternative schedule under the same parity tests); FD_K2_SPLIT=0: the fused k_cascade
     // a soft cascade (R8b) runs its own schedule, k_soft (k_soft.cu): one lane per window, the
     // running sum carried across stages, no survivor lists, no tail queue, no specialisation
+    // FD_K2_QUEUE=1 runs a hard cascade on the same schedule (alternative, measured)
     const bool soft = c->soft != 0;
-    const bool wsk = !soft && env_int("FD_K2_WS", 0) != 0;
-    const bool split = !soft && !wsk && env_int("FD_K2_SPLIT", 1) != 0;
+    const bool queue = soft || env_int("FD_K2_QUEUE", 0) != 0;
+    const bool wsk = !queue && env_int("FD_K2_WS", 0) != 0;
+    const bool split = !queue && !wsk && env_int("FD_K2_SPLIT", 1) != 0;
     const bool deep1 = env_int("FD_K2_DEEP1", 1) != 0;      // k_deep1 (tile per small CTA) or batched k_deep
     // tail queue (k_tail): FD_TAIL=0 keeps every window inside K2; FD_TAIL_N = windows left in a
     // batch at which it hands them over; FD_TAIL_CAP = queue entries (16 B each) per group
-    const bool use_tail = !soft && env_int("FD_TAIL", 1) != 0;
+    const bool use_tail = !queue && env_int("FD_TAIL", 1) != 0;
     const int tail_cap = use_tail ? std::max(1024, env_int("FD_TAIL_CAP", 1 << 22)) : 0;
     K1Scratch k1s[2];
     std::vector<CUtensorMap> maps((size_t)PD.n_levels);
@@ -679,7 +681,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     TP.stage_counts = d_stage_counts;
     // step 1: the K2 specialised for this cascade (compiled once, FD_JIT=0 selects the generic kernel)
     JitK2* jit = nullptr;
-    if (step == 1 && !soft && env_int("FD_JIT", 1) != 0) {
+    if (step == 1 && !queue && env_int("FD_JIT", 1) != 0) {
         std::lock_guard<std::mutex> lk(c->mu);
         if (!c->jit_tried) {
             c->jit_tried = true;
@@ -724,8 +726,8 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         P.surv = split ? sl.surv.as<uint2>() : nullptr;
         P.tile_rec = split ? sl.tilerec.as<uint2>() : nullptr;
         const int gr = grid < P.total_tiles ? grid : P.total_tiles;
-        if (soft) {
-            LAUNCH(FD_K_CASCADE, gs, launch_soft(P, depth, step, gs));
+        if (queue) {
+            LAUNCH(FD_K_CASCADE, gs, launch_soft(P, depth, step, soft, gs));
         } else if (jit) {
             std::string err;
             cudaError_t e;

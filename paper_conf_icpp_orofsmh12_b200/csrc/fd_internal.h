@@ -289,7 +289,7 @@ cudaError_t launch_stage1(const CascadeParams& p, bool depth_mode, int step, cud
 cudaError_t launch_deep(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
 cudaError_t launch_deep1(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
 cudaError_t launch_ws(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
-cudaError_t launch_soft(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);  // k_soft.cu (R8b)
+cudaError_t launch_soft(const CascadeParams& p, bool depth_mode, int step, bool soft, cudaStream_t st);  // k_soft.cu (R8b)
 cudaError_t launch_depth_hist(const uint8_t* depth, int n, long long win_per_frame, const long long* d_win0,
                               int n_levels, int n_stages, long long* hist, int max_span, cudaStream_t st);
 int cascade_grid(bool depth_mode, int step);       // persistent grid size (SMs x resident CTAs)

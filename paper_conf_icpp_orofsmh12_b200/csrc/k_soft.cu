@@ -23,7 +23,7 @@ namespace fdk {
 
 constexpr int SOFT_MAX_STAGES = 256;      // the .fdc parser allows at most 250 stages
 
-template <int STEP, bool DEPTH>
+template <int STEP, bool DEPTH, bool SOFT>
 __global__ void __launch_bounds__(k2_threads(STEP), 2) k_soft(const __grid_constant__ CascadeParams p) {
     using G = TileGeo<STEP>;
     constexpr int TW = tile_w(STEP), TX = k2_tx(STEP), TY = k2_ty(STEP), WPT = k2_wpt(STEP), NW = G::NW;
@@ -165,6 +165,7 @@ __global__ void __launch_bounds__(k2_threads(STEP), 2) k_soft(const __grid_const
             if (!alive) continue;
             const StageDev sd = s < p.n_pstages ? p.pstages[s] : p.stages[s];
             if (counting) atomicAdd(&s_sc[s], 1u);
+            if (!SOFT) sum = 0.0f;                // hard cascade (R8): every stage sum starts at 0
             for (int j = sd.first; j < sd.first + sd.n; ++j)
                 sum = __fadd_rn(sum, eval_stump_mc<MAX_CORNERS>(T, b, nfw, grec, j));
             const bool pass = sum >= sd.T;
@@ -184,29 +185,36 @@ __global__ void __launch_bounds__(k2_threads(STEP), 2) k_soft(const __grid_const
     }
 }
 
-template <int STEP, bool DEPTH>
+template <int STEP, bool DEPTH, bool SOFT>
 static cudaError_t launch_soft_t(const CascadeParams& p, cudaStream_t st) {
     const size_t smem = TileGeo<STEP>::SMEM;
-    cudaError_t e = cudaFuncSetAttribute(k_soft<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(k_soft<STEP, DEPTH, SOFT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     int dev = 0, sms = 0, per = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_soft<STEP, DEPTH>, k2_threads(STEP), smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_soft<STEP, DEPTH, SOFT>, k2_threads(STEP), smem);
     int grid = sms * (per > 0 ? per : 1);
     if (grid > p.total_tiles) grid = p.total_tiles;
-    k_soft<STEP, DEPTH><<<grid, k2_threads(STEP), smem, st>>>(p);
+    k_soft<STEP, DEPTH, SOFT><<<grid, k2_threads(STEP), smem, st>>>(p);
     return cudaGetLastError();
 }
 
-cudaError_t launch_soft(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
+template <bool SOFT>
+static cudaError_t launch_q(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
     switch (step) {
-        case 1: return depth ? launch_soft_t<1, true>(p, st) : launch_soft_t<1, false>(p, st);
-        case 2: return depth ? launch_soft_t<2, true>(p, st) : launch_soft_t<2, false>(p, st);
-        case 3: return depth ? launch_soft_t<3, true>(p, st) : launch_soft_t<3, false>(p, st);
-        case 4: return depth ? launch_soft_t<4, true>(p, st) : launch_soft_t<4, false>(p, st);
+        case 1: return depth ? launch_soft_t<1, true, SOFT>(p, st) : launch_soft_t<1, false, SOFT>(p, st);
+        case 2: return depth ? launch_soft_t<2, true, SOFT>(p, st) : launch_soft_t<2, false, SOFT>(p, st);
+        case 3: return depth ? launch_soft_t<3, true, SOFT>(p, st) : launch_soft_t<3, false, SOFT>(p, st);
+        case 4: return depth ? launch_soft_t<4, true, SOFT>(p, st) : launch_soft_t<4, false, SOFT>(p, st);
         default: return cudaErrorInvalidValue;
     }
+}
+
+// soft = true: a soft cascade (R8b); false: a hard cascade on the same queue schedule
+// (FD_K2_QUEUE=1, an alternative K2 schedule measured against the default)
+cudaError_t launch_soft(const CascadeParams& p, bool depth, int step, bool soft, cudaStream_t st) {
+    return soft ? launch_q<true>(p, depth, step, st) : launch_q<false>(p, depth, step, st);
 }
 
 }  // namespace fdk

@@ -136,6 +136,7 @@ K2_SCHEDULES = {
     "batched_deep": {"FD_K2_DEEP1": "0"},                   # k_stage1 + batched k_deep
     "one_slot_pipeline": {"FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
     "two_slot_pipeline": {"FD_GROUP_FRAMES": "1"},          # 3 frame groups over 2 slots/streams
+    "queue": {"FD_K2_QUEUE": "1"},                          # k_soft's schedule on a hard cascade
 }
 
 
