@@ -47,12 +47,12 @@ def assert_scores_equal(gpu, ref, near, what):
     return len(bad)
 
 
-def compare_depth(casc_pair, frames, s, step=1):
+def compare_depth(casc_pair, frames, s, step=1, min_size=24):
     gc, oc = casc_pair
     d_fr = torch.from_numpy(frames).cuda()
-    depth, score = fd.fd_detect_depth(gc, d_fr, 24, s, step)
+    depth, score = fd.fd_detect_depth(gc, d_fr, min_size, s, step)
     torch.cuda.synchronize()
-    od, osc, onear = oracle.detect_depth(oc, frames, 24, s, step, nthreads=os.cpu_count())
+    od, osc, onear = oracle.detect_depth(oc, frames, min_size, s, step, nthreads=os.cpu_count())
     gd = depth.cpu().numpy()
     gs = score.cpu().numpy()
     mism = np.nonzero(gd != od)[0]
@@ -224,6 +224,27 @@ def test_depth_maps_step(step):
 def test_depth_maps_ragged_sizes(W, H, s):
     fr = np.stack([fdgen.background(2, 900 + i, W, H) for i in range(2)])
     compare_depth(cascades(2), fr, s)
+
+
+@pytest.mark.parametrize("min_size", [25, 30, 48, 97])
+def test_min_size_bit_exact(min_size):
+    """min_size > 24 (f_0 = min_size/24, so level 0 is itself resampled and
+    every back-projected rect is scaled): levels, depth maps and detection lists."""
+    W, H, s = 640, 480, 1.2
+    fr, _ = gen(2, 41, 2)
+    lv = fd.fd_build_pyramid(torch.from_numpy(fr).cuda(), min_size, s).cpu().numpy()
+    pl = oracle.plan(W, H, min_size, s, 1)
+    assert pl and abs(pl[0][0] - min_size / 24.0) < 1e-15
+    for i in range(2):
+        off = 0
+        for (f, wk, hk, _) in pl:
+            assert np.array_equal(lv[i, off:off + wk * hk].reshape(hk, wk), oracle.resample(fr[i], f, wk, hk))
+            off += wk * hk
+    compare_depth(cascades(2), fr, s, 1, min_size)
+    gc, oc = cascades(2)
+    got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), min_size, s, 1, capacity=1 << 20))
+    ref, _ = oracle.detect(oc, fr, min_size, s, 1, nthreads=os.cpu_count())
+    assert np.array_equal(got, ref), f"{len(got)} vs {len(ref)} detections"
 
 
 # ------------------------------------------------------------------ detections (fd_detect)
