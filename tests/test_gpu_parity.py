@@ -247,6 +247,19 @@ def test_min_size_bit_exact(min_size):
     assert np.array_equal(got, ref), f"{len(got)} vs {len(ref)} detections"
 
 
+@pytest.mark.parametrize("cfg,W,H,s", [(2, 320, 240, 1.02), (1, 640, 480, 1.025)])
+def test_many_levels_near_max(cfg, W, H, s):
+    """117 / 122 pyramid levels, close to FD_MAX_LEVELS = 128 (the plan tables, tile scheduler
+    and per-level offsets at their largest): depth maps and detection lists bit-exact."""
+    assert 110 < len(oracle.plan(W, H, 24, s, 1)) <= 128
+    fr = np.stack([fdgen.background(cfg, 950 + i, W, H) for i in range(2)])
+    compare_depth(cascades(cfg), fr, s)
+    gc, oc = cascades(cfg)
+    got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1, capacity=1 << 22))
+    ref, _ = oracle.detect(oc, fr, 24, s, 1, nthreads=os.cpu_count())
+    assert np.array_equal(got, ref), f"{len(got)} vs {len(ref)} detections"
+
+
 # ------------------------------------------------------------------ detections (fd_detect)
 @pytest.mark.parametrize("cfg", [1, 2, 3])
 def test_detections_identical(cfg):
