@@ -80,7 +80,7 @@ def test_pyramid_levels_bit_exact(cfg):
             off += wk * hk
 
 
-@pytest.mark.parametrize("W,H", [(24, 24), (7, 5), (333, 97), (129, 257), (640, 480), (1920, 1080)])
+@pytest.mark.parametrize("W,H", [(24, 24), (7, 5), (333, 97), (129, 257), (640, 480), (1920, 1080), (3840, 2160)])
 def test_integral_bit_exact(W, H):
     rng = np.random.default_rng(W * 1000 + H)
     img = rng.integers(0, 256, (3, H, W), dtype=np.uint8)
@@ -410,6 +410,15 @@ def test_soft_depth_maps_bit_exact(cfg, name, n_st, per_stump, W, H, s, step):
     fr, _ = gen(cfg, 21, 2, W, H, s)
     s = s or CFG[cfg][2]
     gd, od = compare_depth((fd.Cascade(text), oracle.Cascade(text)), fr, s, step)
+    assert np.array_equal(gd, od) and len(np.unique(od)) >= 3
+
+
+@pytest.mark.parametrize("W,H,s,min_size", [(640, 480, 1.2, 48), (320, 240, 1.02, 24)])
+def test_soft_min_size_and_many_levels(W, H, s, min_size):
+    """Soft cascade (R8b) with a resampled level 0 (min_size 48) and with 117 levels."""
+    text = softcasc.soft_from("c2.fdc", None, False)
+    fr = np.stack([fdgen.background(2, 970 + i, W, H) for i in range(2)])
+    gd, od = compare_depth((fd.Cascade(text), oracle.Cascade(text)), fr, s, 1, min_size)
     assert np.array_equal(gd, od) and len(np.unique(od)) >= 3
 
 
