@@ -133,7 +133,7 @@ struct TileGeoW {
 };
 
 #ifndef FD_K2D_CTAS
-#define FD_K2D_CTAS 6
+#define FD_K2D_CTAS 8
 #endif
 constexpr int K2D_THREADS = 128;
 template <int STEP>
