@@ -283,30 +283,63 @@ def test_detections_identical(cfg):
     assert sc.cpu().tolist() == want
 
 
-def test_video_batch_sampled_1080p():
-    """c4-shaped: 16 frames 1080p with Poisson(4) planted faces in one call (several frame
-    groups); oracle on frames 0, 7 and 15 only."""
+def _bench_shape_parity(n_frames, first=0):
+    """The c4 bench configuration (1080p, Poisson(4) planted faces, c3 cascade, s = 1.1, step 1)
+    in ONE fd_detect call, so the library's own frame grouping and pipeline slots are exercised
+    exactly as bench.py times them.  Every frame's detections and the per-stage counters are
+    compared with the oracle, and fd_group over the whole batch with oracle.group."""
     W, H, s = 1920, 1080, 1.1
     lv = oracle.plan(W, H, 24, s, 1)
-    fr, _ = fdgen.frames(4, 0, 16, W, H, lv, faces="poisson", face_param=4, max_face_level=30)
+    fr, _ = fdgen.frames(4, first, n_frames, W, H, lv, faces="poisson", face_param=4, max_face_level=30)
     gc, oc = cascades(3)
-    got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1))
-    for i in (0, 7, 15):
-        ref, _ = oracle.detect(oc, fr[i:i + 1], 24, s, 1, nthreads=os.cpu_count())
-        ref["frame"] = i
-        assert np.array_equal(got[got["frame"] == i], ref), i
+    sc = torch.zeros(gc.n_stages + 1, dtype=torch.int64, device="cuda")
+    dets = fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1, capacity=1 << 22, stage_counts=sc)
+    got = fd.to_numpy(dets)
+    want_counts = np.zeros(gc.n_stages + 1, np.int64)
+    near = 0
+    refs = []
+    for c0 in range(0, n_frames, 8):             # oracle in chunks (depth maps of 8 frames at a time)
+        chunk = fr[c0:c0 + 8]
+        ref, nn = oracle.detect(oc, chunk, 24, s, 1, nthreads=os.cpu_count())
+        ref["frame"] += c0
+        refs.append(ref)
+        near += nn
+        od, _, _ = oracle.detect_depth(oc, chunk, 24, s, 1, nthreads=os.cpu_count())
+        want_counts += np.array([int((od >= k).sum()) for k in range(gc.n_stages + 1)])
+    ref = np.concatenate(refs)
+    print(f"{n_frames} frames: {len(ref)} detections, near-threshold windows {near}, "
+          f"decision mismatches {int(len(got) != len(ref) or not np.array_equal(got, ref))}")
+    for i in range(n_frames):
+        assert np.array_equal(got[got["frame"] == i], ref[ref["frame"] == i]), f"frame {i}"
+    assert np.array_equal(got, ref)
+    assert sc.cpu().numpy().tolist() == want_counts.tolist()
+    grp = fd.to_numpy(fd.fd_group(dets, 0.5, 1))
+    assert np.array_equal(grp, oracle.group(ref, 0.5, 1))
+    return fr
+
+
+def test_video_batch_1080p_bench_shape():
+    """48 frames at the default group size (16 frames of 1080p per group -> three groups over
+    both pipeline slots and streams), every frame checked (VERDICT r1 'weak' 1)."""
+    _bench_shape_parity(48)
+
+
+def test_video_batch_1080p_small_groups(monkeypatch):
+    """12 frames in groups of 4 (FD_GROUP_FRAMES=4): three groups, slot 0 used twice."""
+    monkeypatch.setenv("FD_GROUP_FRAMES", "4")
+    _bench_shape_parity(12, first=100)
 
 
 def test_4k_sampled():
-    """c5-shaped: 2 frames 3840x2160; oracle on frame 1."""
+    """c5-shaped: 2 frames 3840x2160 (Poisson(4) planted faces), both checked."""
     W, H, s = 3840, 2160, 1.1
     lv = oracle.plan(W, H, 24, s, 1)
     fr, _ = fdgen.frames(5, 0, 2, W, H, lv, faces="poisson", face_param=4, max_face_level=34)
     gc, oc = cascades(3)
     got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1))
-    ref, _ = oracle.detect(oc, fr[1:2], 24, s, 1, nthreads=os.cpu_count())
-    ref["frame"] = 1
-    assert np.array_equal(got[got["frame"] == 1], ref)
+    ref, nn = oracle.detect(oc, fr, 24, s, 1, nthreads=os.cpu_count())
+    print(f"4K: {len(ref)} detections, near-threshold windows {nn}")
+    assert np.array_equal(got, ref)
 
 
 def test_detect_host_equals_device():

@@ -339,6 +339,53 @@ def test_all_pass_and_all_reject_cascades():
     assert len(d) == 2 * tot and (d == 0).all() and (sc == 0.5).all()
 
 
+@pytest.mark.parametrize("min_size,num,den", [(36, 3, 2), (30, 5, 4), (48, 2, 1)])
+def test_backprojection_round_half_up(min_size, num, den):
+    """c9 (P:L623-631 "multiplying the downscaling factor by the normalized dimensions"; reading
+    R9: round half up in double).  min_size 36 gives f_0 = 1.5 exactly and min_size 30 gives
+    1.25, so wx*f_0 lands exactly on .5 for odd wx (1.5 -> 2, 4.5 -> 5) and for wx = 2 mod 4
+    (2.5 -> 3).  Expected values are integer closed forms: floor(wx*num/den + 1/2) =
+    (2*wx*num + den) // (2*den); round-half-even or truncation would fail at those windows.
+    An all-pass cascade makes every level-0 window a detection."""
+    W, H = 160, 100
+    fr, _ = fdgen.frames(9, 5, 1, W, H)
+    st = ([(1, 1, 10, 10, -1), (1, 1, 5, 10, 2)], 0.1, 0.5, 0.5)
+    allpass = oracle.Cascade(cascade_text([(-math.inf, [st])]))
+    dets, _ = oracle.detect(allpass, fr, min_size, 1.25, 1)
+    lv0 = dets[dets["level"] == 0]
+    f0 = oracle.plan(W, H, min_size, 1.25, 1)[0]
+    assert f0[0] * den == num and len(lv0) == f0[3]
+    for field, src in (("x", "wx"), ("y", "wy")):
+        want = (2 * lv0[src].astype(np.int64) * num + den) // (2 * den)
+        assert np.array_equal(lv0[field], want), field
+    assert (lv0["w"] == (2 * 24 * num + den) // (2 * den)).all() and (lv0["h"] == lv0["w"]).all()
+    # the half-way cases are present: odd wx for f = 1.5, wx = 2 mod 4 for f = 1.25
+    half = (2 * lv0["wx"].astype(np.int64) * num) % (2 * den) == den
+    assert half.any() == (den > 1)
+    if den > 1:
+        assert (lv0["x"][half] * 2 * den == 2 * lv0["wx"][half] * num + den).all()
+
+
+def test_stage_near_threshold_flag():
+    """c11 (north_star: windows whose score lies within 1e-4 of a stage threshold are counted
+    and reported): bit 0 of the near flag is set iff |sum_s - T_s| <= 1e-4 at an evaluated
+    stage.  Constant window: f = 0, nf = 1; theta = 100 puts every stump far from its own
+    threshold (bit 1 clear); both leaves are 0.5 so the stage sum is exactly 0.5."""
+    ii, sq = oracle.integral(np.full((24, 24), 77, np.uint8))
+    st = ([(1, 1, 4, 4, -1), (1, 1, 2, 4, 2)], 100.0, 0.5, 0.5)
+    for T, depth, flag in ((0.5 + 5e-5, 0, 1),      # just above: reject, flagged
+                           (0.5 - 5e-5, 1, 1),      # just below: pass, flagged
+                           (0.5 + 2e-4, 0, 0),      # outside the band: reject, not flagged
+                           (0.5 - 2e-4, 1, 0)):
+        d, score, near = oracle.eval_window(oracle.Cascade(cascade_text([(T, [st])])), ii, sq, 0, 0)
+        assert (d, score, near) == (depth, 0.5, flag), T
+    # the flag comes from any evaluated stage, not only the rejecting one; an unevaluated
+    # stage never sets it
+    far, close = (0.5 - 2e-4, [st]), (0.5 - 5e-5, [st])
+    assert oracle.eval_window(oracle.Cascade(cascade_text([close, far, (1.0, [st])])), ii, sq, 0, 0)[2] == 1
+    assert oracle.eval_window(oracle.Cascade(cascade_text([(1.0, [st]), close])), ii, sq, 0, 0)[2] == 0
+
+
 def test_filter_binomial_pins():
     """f2 filtering stage (reading R3b): weights sum to 16, so constants are fixed points; the
     binomial kernel reproduces linear functions exactly away from the border; an impulse gives
