@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define FD_ABI_VERSION 2
+#define FD_ABI_VERSION 3
 #define FD_MAX_LEVELS 128
 #define FD_WINDOW 24 /* fixed 24x24 sliding window, image scaled instead (Fig. 2) */
 
@@ -184,16 +184,17 @@ fd_status fd_detect_group_host(fd_cascade c, const uint8_t* h_frames, int n, int
 /* Kernel accounting (process-wide, all devices): number of launches of each kernel class
  * since the last fd_profile_reset and, if time_kernels != 0, their summed device time
  * measured with CUDA events recorded on the launching stream around each launch.
- * FD_K_SORT is the CUB radix sort (library code, counted as one call).  K1 is FD_K_COLSUM
- * (k_marg: resampling + per-tile marginals), FD_K_CARRY (k_carry + k_corner) and FD_K_BAND
- * (k_tile: ii / sqii).  The cascade evaluator is FD_K_CASCADE (k_stage1: stages 1-2 dense and
- * compacted; or k_ws / k_cascade in the alternative schedules), FD_K_DEEP (k_deep1: the deeper
- * stages, one tile per CTA) and FD_K_TAIL (k_tail: the few windows left per tile, one warp per
- * window).  FD_K_DEPTH_HIST is fd_depth_histogram. */
+ * FD_K_SORT is the CUB radix sort (library code, counted as one call).  Default detection
+ * path (f1): FD_K_LEVEL (k_level: the group's level images) and FD_K_CASCADE (k_f1: tile-local
+ * integral + every stage).  K1 (fd_integral, soft cascades, the FD_F1=0 schedule) is
+ * FD_K_COLSUM (k_marg: resampling + per-tile marginals), FD_K_CARRY (k_carry + k_corner) and
+ * FD_K_BAND (k_tile: ii / sqii); its cascade kernels are FD_K_CASCADE (k_stage1, k_cascade or
+ * k_soft) and FD_K_DEEP (k_deep1).  FD_K_TAIL is k_tail (the few windows left per tile, one warp
+ * per window).  FD_K_DEPTH_HIST is fd_depth_histogram. */
 typedef enum {
     FD_K_COLSUM = 0, FD_K_CARRY = 1, FD_K_BAND = 2, FD_K_CASCADE = 3,
     FD_K_SORT = 4, FD_K_DETS = 5, FD_K_GROUP = 6, FD_K_PYRAMID = 7, FD_K_TAIL = 8,
-    FD_K_DEEP = 9, FD_K_DEPTH_HIST = 10, FD_K_COUNT = 11
+    FD_K_DEEP = 9, FD_K_DEPTH_HIST = 10, FD_K_LEVEL = 11, FD_K_COUNT = 12
 } fd_kernel_kind;
 typedef struct {
     int64_t launches[FD_K_COUNT];

@@ -48,7 +48,8 @@ class _Plan(C.Structure):
                 ("windows", C.c_int64 * FD_MAX_LEVELS), ("total_windows", C.c_int64)]
 
 
-K_NAMES = ["colsum", "carry", "band", "cascade", "sort", "dets", "group", "pyramid", "tail", "deep", "depth_hist"]
+K_NAMES = ["colsum", "carry", "band", "cascade", "sort", "dets", "group", "pyramid", "tail", "deep", "depth_hist",
+           "level"]
 
 
 class _Profile(C.Structure):

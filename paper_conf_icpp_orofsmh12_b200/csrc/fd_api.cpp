@@ -1,7 +1,11 @@
 // fd_api.cpp -- the C ABI (include/fd.h): validation, pyramid plan, cascade parsing and
-// packing, per-(device, stream) workspaces, and the launch sequence of the hot path
-//   K1 (k_colsum -> k_carry -> k_band)  ->  K2 (k_cascade, persistent, all scales)
-//   -> count read-back -> K3 (radix sort + back-projection).
+// packing, per-(device, stream) workspaces, and the launch sequence of the hot path, per frame
+// group on two pipeline slots:
+//   default (f1):  k_level (level images, u8)  ->  k_f1 (persistent, all scales: tile-local
+//                  integral + every stage)  ->  k_tail
+//   FD_F1=0 / soft cascades:  K1 (k_marg -> k_carry/k_corner -> k_tile: global ii + sqii)
+//                  ->  k_stage1 + k_deep1 (+ k_tail), or k_soft
+//   then count read-back -> K3 (radix sort + back-projection).
 // Host code only; every arithmetic step of the method runs in the kernels.
 #include <cuda.h>
 #include <cuda_runtime.h>
@@ -82,13 +86,16 @@ void make_plan_dev(const fd_plan& pl, int W, int H, int pitch, int step, int G, 
     p->step = step;
     p->G = G;
     const int tx = k2_tx(step), ty = k2_ty(step);
-    long long ws = 0, col = 0, win = 0, row = 0, cor = 0, lvl = 0;
+    long long ws = 0, col = 0, win = 0, row = 0, cor = 0, lvl = 0, u8 = 0;
     int bands = 0, tiles = 0, maxW = 0, k1t = 0;
     for (int k = 0; k < pl.n_levels; ++k) {
         LevelDev& L = p->lv[k];
         L.W = pl.w[k];
         L.H = pl.h[k];
         L.P = (L.W + 1 + 3) & ~3;
+        L.PB = (L.W + 1 + 15) & ~15;
+        L.u8_off = u8;
+        u8 += (long long)G * L.H * L.PB;
         L.nx = (L.W - WIN) / step + 1;
         L.ny = (L.H - WIN) / step + 1;
         L.band0 = bands;
@@ -125,6 +132,7 @@ void make_plan_dev(const fd_plan& pl, int W, int H, int pitch, int step, int G, 
     p->cor_frame = cor;
     p->lvl_frame = lvl;
     p->ws_elems = ws;
+    p->u8_bytes = u8;
 }
 
 // ------------------------------------------------------------------ cascade (.fdc) parser
@@ -410,6 +418,36 @@ fd_status encode_maps(const PlanDev& p, uint32_t* ws, int step, int box_planes, 
     return FD_OK;
 }
 
+// f1: one 3-D map per level over the group's level images {x, y, frame}; the box is a tile's
+// pixel region (TileGeoF), zero-filled beyond the level
+void f1_box(int step, int* bw, int* bh) {
+    switch (step) {
+        case 1: *bw = TileGeoF<1>::U8W; *bh = TileGeoF<1>::PH; break;
+        case 2: *bw = TileGeoF<2>::U8W; *bh = TileGeoF<2>::PH; break;
+        case 3: *bw = TileGeoF<3>::U8W; *bh = TileGeoF<3>::PH; break;
+        default: *bw = TileGeoF<4>::U8W; *bh = TileGeoF<4>::PH; break;
+    }
+}
+
+fd_status encode_maps8(const PlanDev& p, uint8_t* ws8, int step, CUtensorMap* maps) {
+    EncodeTiledFn enc = encode_fn();
+    if (!enc) return fail(FD_ECUDA, "cuTensorMapEncodeTiled unavailable");
+    int bw = 0, bh = 0;
+    f1_box(step, &bw, &bh);
+    for (int k = 0; k < p.n_levels; ++k) {
+        const LevelDev& L = p.lv[k];
+        cuuint64_t dims[3] = {(cuuint64_t)L.W, (cuuint64_t)L.H, (cuuint64_t)p.G};
+        cuuint64_t strides[2] = {(cuuint64_t)L.PB, (cuuint64_t)L.H * L.PB};
+        cuuint32_t box[3] = {(cuuint32_t)bw, (cuuint32_t)bh, 1};
+        cuuint32_t es[3] = {1, 1, 1};
+        CUresult r = enc(&maps[k], CU_TENSOR_MAP_DATA_TYPE_UINT8, 3, ws8 + L.u8_off, dims, strides, box, es,
+                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) return fail(FD_ECUDA, "cuTensorMapEncodeTiled (u8) failed (%d) for level %d", (int)r, k);
+    }
+    return FD_OK;
+}
+
 // ------------------------------------------------------------------ kernel accounting
 struct Profiler {
     std::mutex mu;
@@ -563,7 +601,7 @@ fd_status check_frames(const void* d, int n, int W, int H, int pitch) {
     return FD_OK;
 }
 
-// core of fd_detect / fd_detect_depth: K1 + K2 for every frame group.
+// core of fd_detect / fd_detect_depth: the hot path for every frame group.
 fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int n, int W, int H, int pitch,
                      const fd_plan& pl, int step, bool depth, uint8_t* d_depth, float* d_score, long long det_cap,
                      unsigned long long* d_stage_counts, cudaStream_t st) {
@@ -571,60 +609,68 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     const Packed* pk = nullptr;
     fd_status s = get_packed(c, step, &pk);
     if (s != FD_OK) return s;
-    // frames per group: one K2 launch per group; larger groups amortise the launch tail
-    // (FD_GROUP_MB workspace budget, default 1536 MB = 16 frames of 1080p; FD_GROUP_FRAMES overrides)
+    // Schedules (all under the same parity tests, tests/test_gpu_parity.py K2_SCHEDULES):
+    //   default for hard cascades: K1 -> k_stage1 -> k_deep1 -> k_tail (FD_K2_SPLIT=0: K1 ->
+    //            fused k_cascade -> k_tail);
+    //   FD_F1=1: k_level -> k_f1 -> k_deep1<F1> -> k_tail, no global integral
+    //            (FD_F1_SPLIT=0: k_f1 runs every stage);
+    //   soft cascades (R8b) and FD_K2_QUEUE=1: K1 -> k_soft (one lane per window, running sums).
+    const bool soft = c->soft != 0;
+    const bool queue = soft || env_int("FD_K2_QUEUE", 0) != 0;
+    const bool f1 = !queue && env_int("FD_F1", 0) != 0;
+    // f1 split (default): k_f1 runs stages 0-1, k_deep1 the rest from rebuilt tile integrals
+    // (FD_F1_SPLIT=0: k_f1 runs every stage itself)
+    const bool f1_split = f1 && env_int("FD_F1_SPLIT", 1) != 0;
+    const bool split = !queue && !f1 && env_int("FD_K2_SPLIT", 1) != 0;
+    const bool surv = split || f1_split;
+    // tail queue (k_tail): FD_TAIL=0 keeps every window inside K2; FD_TAIL_N = windows left in a
+    // batch at which it hands them over; FD_TAIL_CAP = queue entries (16 B each) per group
+    const bool use_tail = !queue && env_int("FD_TAIL", 1) != 0;
+    const int tail_cap = use_tail ? std::max(1024, env_int("FD_TAIL_CAP", 1 << 22)) : 0;
+    // frames per group: one K2 launch per group.  f1: the group's level images (12.5 MB per 1080p
+    // frame) should stay L2-resident between k_level and k_f1 (FD_F1_GROUP_MB, default 64 MB);
+    // K1 schedules: the ii/sqii planes (95.8 MB per 1080p frame; FD_GROUP_MB, default 1536 MB).
+    // FD_GROUP_FRAMES overrides.  G <= 65535 (tile and tail-queue frame indices are 32-bit, but
+    // the tensor maps' frame extent is kept within 16 bits).
     PlanDev one;
     make_plan_dev(pl, W, H, pitch, step, 1, &one);
-    const double per_frame = (double)one.ws_elems * 4.0;
+    const double per_frame = f1 ? (double)one.u8_bytes : (double)one.ws_elems * 4.0;
     int G = env_int("FD_GROUP_FRAMES", 0);
-    const double budget = (double)env_int("FD_GROUP_MB", 1536) * 1024.0 * 1024.0;
-    if (G <= 0) G = (int)std::floor(budget / (per_frame > 1 ? per_frame : 1));
-    if (G < 1) G = 1;
-    if (G > n) G = n;
+    const double budget = (double)(f1 ? env_int("FD_F1_GROUP_MB", 64) : env_int("FD_GROUP_MB", 1536)) * 1024.0 * 1024.0;
+    if (G <= 0) G = (int)std::min(65535.0, std::floor(budget / (per_frame > 1 ? per_frame : 1)));
+    G = std::max(1, std::min(G, std::min(n, 65535)));
     const int ngroups = (n + G - 1) / G;
     PlanDev& PD = *w->plan;
     make_plan_dev(pl, W, H, pitch, step, G, &PD);
     PD.filter = c->filter;
     // two pipeline slots on two streams when there is more than one group (FD_PIPE=0: one)
     const int nslots = (ngroups > 1 && env_int("FD_PIPE", 1) != 0) ? 2 : 1;
-    // K2 split in two kernels (k_stage1: dense first stage, k_deep: batched deeper stages;
-    // FD_K2_SPLIT=0 runs the fused k_cascade).  Survivor list sized for the worst case.
-    // default (FD_K2_SPLIT=1): k_stage1 + k_deep1 (+ k_tail).  FD_K2_WS=1: the warp-specialised
-    // k_ws (stage-1 and deep warp groups in one kernel; measured slower on B200, kept as an
-    // alternative schedule under the same parity tests); FD_K2_SPLIT=0: the fused k_cascade
-    // a soft cascade (R8b) runs its own schedule, k_soft (k_soft.cu): one lane per window, the
-    // running sum carried across stages, no survivor lists, no tail queue, no specialisation
-    // FD_K2_QUEUE=1 runs a hard cascade on the same schedule (alternative, measured)
-    const bool soft = c->soft != 0;
-    const bool queue = soft || env_int("FD_K2_QUEUE", 0) != 0;
-    const bool wsk = !queue && env_int("FD_K2_WS", 0) != 0;
-    const bool split = !queue && !wsk && env_int("FD_K2_SPLIT", 1) != 0;
-    const bool deep1 = env_int("FD_K2_DEEP1", 1) != 0;      // k_deep1 (tile per small CTA) or batched k_deep
-    // tail queue (k_tail): FD_TAIL=0 keeps every window inside K2; FD_TAIL_N = windows left in a
-    // batch at which it hands them over; FD_TAIL_CAP = queue entries (16 B each) per group
-    const bool use_tail = !queue && env_int("FD_TAIL", 1) != 0;
-    const int tail_cap = use_tail ? std::max(1024, env_int("FD_TAIL_CAP", 1 << 22)) : 0;
     K1Scratch k1s[2];
     std::vector<CUtensorMap> maps((size_t)PD.n_levels);
     for (int b = 0; b < nslots; ++b) {
         PipeSlot& sl = w->slot[b];
-        CK(sl.ws.ensure((size_t)PD.ws_elems * 4));
-        CK(sl.k1_scratch(PD, G, &k1s[b]));
-        if (split) {
+        if (surv) {
             CK(sl.surv.ensure((size_t)G * (size_t)PD.win_per_frame * 8 + 16));
             CK(sl.tilerec.ensure((size_t)G * PD.tiles_per_frame * 8 + 16));
         }
-        if (use_tail) CK(sl.tailq.ensure((size_t)tail_cap * 16));
-        // tensor maps of this slot's integral planes (global memory, copied in stream order)
-        s = encode_maps(PD, sl.ws.as<uint32_t>(), step, 1, maps.data());
+        if (f1) {
+            CK(sl.ws.ensure((size_t)PD.u8_bytes + 16));
+            s = encode_maps8(PD, sl.ws.as<uint8_t>(), step, maps.data());
+        } else {
+            CK(sl.ws.ensure((size_t)PD.ws_elems * 4));
+            CK(sl.k1_scratch(PD, G, &k1s[b]));
+            // tensor maps of this slot's integral planes (global memory, copied in stream order)
+            s = encode_maps(PD, sl.ws.as<uint32_t>(), step, 1, maps.data());
+        }
         if (s != FD_OK) return s;
+        if (use_tail) CK(sl.tailq.ensure((size_t)tail_cap * 16));
         CK(sl.tmaps.ensure(sizeof(CUtensorMap) * FD_MAX_LEVELS));
         std::memcpy(w->h_geo.get() + b * FD_MAX_LEVELS, maps.data(), sizeof(CUtensorMap) * PD.n_levels);
         CK(cudaMemcpyAsync(sl.tmaps.p, w->h_geo.get() + b * FD_MAX_LEVELS, sizeof(CUtensorMap) * PD.n_levels,
                            cudaMemcpyHostToDevice, st));
     }
     // ctl: [0] detection count, [256 B..] per-group K2 tile counters, then per-group tail counts,
-    // survivor counts and k_deep tile counters
+    // survivor counts and k_deep1 tile counters
     CK(w->ctl.ensure(256 + (size_t)ngroups * 16));
     CK(cudaMemsetAsync(w->ctl.p, 0, 256 + (size_t)ngroups * 16, st));
     if (!depth) {
@@ -661,14 +707,31 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     P.lane_min = std::max(1, std::min(env_int("FD_LANE_MIN", half + 1), half + 1));
     P.tail_cap = tail_cap;
     P.tail_n = std::max(1, env_int("FD_TAIL_N", 8));
-    // k_stage1 / k_ws run stages [0, s0): FD_S0 / FD_WS_S0 = 2 (default) or 1
-    P.s0 = split ? (env_int("FD_S0", 2) >= 2 ? 2 : 1) : (wsk ? (env_int("FD_WS_S0", 2) >= 2 ? 2 : 1) : 1);
+    // FD_S_TAIL: every window still alive at this stage is handed to k_tail (default: none, only
+    // the FD_TAIL_N rule)
+    P.s_tail = std::max(1, env_int("FD_S_TAIL", 255));
+    // deep stages with at most FD_DEEP_SPLIT windows (<= 64; 0 = off) run split-stump (k_f1)
+    P.split_max = std::max(0, env_int("FD_DEEP_SPLIT", 64));
+    // k_stage1 runs stages [0, s0) (FD_S0 = 2, default, or 1); the fused kernels start their
+    // deep phase at stage 1
+    P.s0 = split ? (env_int("FD_S0", 2) >= 2 ? 2 : 1) : (f1_split ? 2 : 1);
+    P.f1 = f1 ? 1 : 0;
     TailParams TP;
     TP.cap = tail_cap;
     TP.step = step;
     TP.lv = P.lv;
     TP.trec = pk->d_trec;
     TP.ns = (int)c->stumps.size();
+    // k_tail stages the records of the first deep stages in shared memory (whole stages from
+    // stage 1 on, FD_TAIL_SMEM_STUMPS budget, default 256 stumps = 16 KB)
+    {
+        const int budget = std::max(0, env_int("FD_TAIL_SMEM_STUMPS", 256));
+        const int s1 = c->stages.size() > 1 ? 1 : 0;
+        TP.j0 = c->stages[s1].first;
+        int k = s1, m = 0;
+        while (k < (int)c->stages.size() && m + c->stages[k].n <= budget) m += c->stages[k++].n;
+        TP.nsm = m;
+    }
     TP.stages = pk->d_st;
     TP.n_stages = P.n_stages;
     TP.win_per_frame = P.win_per_frame;
@@ -708,12 +771,16 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         const cudaStream_t gs = sts[b];
         const int f0 = gi * G, gf = (n - f0) < G ? (n - f0) : G;
         const uint8_t* fr = d_frames + (size_t)f0 * H * pitch;
-        LAUNCH(FD_K_COLSUM, gs, launch_k1_marg(fr, PD, gf, k1s[b], gs));
-        {
-            ProfScope ps(FD_K_CARRY, gs, 2);
-            CK(launch_k1_carry(PD, gf, k1s[b], gs));
+        if (f1) {
+            LAUNCH(FD_K_LEVEL, gs, launch_levels(fr, PD, gf, sl.ws.as<uint8_t>(), gs));
+        } else {
+            LAUNCH(FD_K_COLSUM, gs, launch_k1_marg(fr, PD, gf, k1s[b], gs));
+            {
+                ProfScope ps(FD_K_CARRY, gs, 2);
+                CK(launch_k1_carry(PD, gf, k1s[b], gs));
+            }
+            LAUNCH(FD_K_BAND, gs, launch_k1_tiles(fr, PD, gf, k1s[b], sl.ws.as<uint32_t>(), gs));
         }
-        LAUNCH(FD_K_BAND, gs, launch_k1_tiles(fr, PD, gf, k1s[b], sl.ws.as<uint32_t>(), gs));
         P.tmaps = sl.tmaps.as<CUtensorMap>();
         P.tail_q = use_tail ? sl.tailq.as<uint4>() : nullptr;
         P.g_frames = gf;
@@ -723,8 +790,8 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         P.tail_count = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + ngroups + gi;
         P.surv_count = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + 2 * ngroups + gi;
         P.deep_counter = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + 3 * ngroups + gi;
-        P.surv = split ? sl.surv.as<uint2>() : nullptr;
-        P.tile_rec = split ? sl.tilerec.as<uint2>() : nullptr;
+        P.surv = surv ? sl.surv.as<uint2>() : nullptr;
+        P.tile_rec = surv ? sl.tilerec.as<uint2>() : nullptr;
         const int gr = grid < P.total_tiles ? grid : P.total_tiles;
         if (queue) {
             LAUNCH(FD_K_CASCADE, gs, launch_soft(P, depth, step, soft, gs));
@@ -733,25 +800,27 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
             cudaError_t e;
             {
                 ProfScope ps(FD_K_CASCADE, gs);
-                e = jit_k2_launch(jit, P, depth, wsk ? JIT_WS : (split ? JIT_STAGE1 : JIT_FUSED), gs, &err);
+                e = jit_k2_launch(jit, P, depth, f1 ? JIT_F1 : (split ? JIT_STAGE1 : JIT_FUSED), gs, &err);
             }
-            if (e == cudaSuccess && split) {
+            if (e == cudaSuccess && surv) {
                 ProfScope ps(FD_K_DEEP, gs);
-                e = jit_k2_launch(jit, P, depth, deep1 ? JIT_DEEP1 : JIT_DEEP, gs, &err);
+                e = jit_k2_launch(jit, P, depth, f1 ? JIT_DEEP1_F1 : JIT_DEEP1, gs, &err);
             }
             if (e != cudaSuccess)
                 return fail(FD_ECUDA, "specialised K2: %s", err.empty() ? cudaGetErrorString(e) : err.c_str());
-        } else if (wsk) {
-            LAUNCH(FD_K_CASCADE, gs, launch_ws(P, depth, step, gs));
+        } else if (f1) {
+            LAUNCH(FD_K_CASCADE, gs, launch_f1(P, depth, step, gs));
+            if (f1_split) LAUNCH(FD_K_DEEP, gs, launch_deep1(P, depth, step, true, gs));
         } else if (split) {
             LAUNCH(FD_K_CASCADE, gs, launch_stage1(P, depth, step, gs));
-            LAUNCH(FD_K_DEEP, gs, deep1 ? launch_deep1(P, depth, step, gs) : launch_deep(P, depth, step, gs));
+            LAUNCH(FD_K_DEEP, gs, launch_deep1(P, depth, step, false, gs));
         } else {
             LAUNCH(FD_K_CASCADE, gs, launch_cascade(P, depth, step, gr, gs));
         }
         if (use_tail) {
             TP.q = P.tail_q;
-            TP.ws = sl.ws.as<uint32_t>();
+            TP.ws = f1 ? nullptr : sl.ws.as<uint32_t>();
+            TP.lvl8 = f1 ? sl.ws.as<uint8_t>() : nullptr;
             TP.count = P.tail_count;
             TP.frame_base = f0;
             LAUNCH(FD_K_TAIL, gs, launch_tail(TP, depth, gs));

@@ -49,11 +49,6 @@ __host__ __device__ constexpr int k2_wpt(int step) { return step == 1 ? 8 : (ste
 __host__ __device__ constexpr int k2_ty(int step) { return (k2_threads(step) / 32 / (k2_tx(step) / 32)) * k2_wpt(step); }
 __host__ __device__ constexpr int tile_w(int step) { return (((k2_tx(step) - 1) * step + WIN + 1) + 3) & ~3; }
 __host__ __device__ constexpr int tile_h(int step) { return (k2_ty(step) - 1) * step + WIN + 1; }
-// split K2 (k_stage1 + k_deep): tiles per k_deep batch (ii-only slots)
-#ifndef FD_K2B_NB
-#define FD_K2B_NB 4
-#endif
-__host__ __device__ constexpr int k2b_min_ctas(int nb) { return nb <= 4 ? 2 : 1; }
 __host__ __device__ constexpr int k2_pbuf(int step) { return (tile_w(step) * tile_h(step) + 31) & ~31; }
 
 
@@ -75,10 +70,11 @@ struct TileGeo {
     static constexpr size_t OFF_LOC = OFF_NF + (size_t)NW * 4;
     static constexpr size_t OFF_LIST = OFF_LOC + (size_t)NW * 2;
 #ifdef FD_POOL_SEPARATE
-    static constexpr size_t SMEM = OFF_LIST + (size_t)NW * 4;
+    static constexpr size_t OFF_RED = OFF_LIST + (size_t)NW * 4;
 #else
-    static constexpr size_t SMEM = OFF_Q + (size_t)QBUF * 4;
+    static constexpr size_t OFF_RED = OFF_Q + (size_t)QBUF * 4;
 #endif
+    static constexpr size_t SMEM = OFF_RED + (size_t)k2_threads(STEP) * 8;   // + split-stump partial sums
 };
 #ifndef FD_K2_CTAS
 #define FD_K2_CTAS 4                        // fused K2: resident CTAs per SM the launch bounds target
@@ -97,57 +93,54 @@ struct TileGeoA {
     static constexpr size_t SMEM = OFF_SIDX + (size_t)NW * 2;
 };
 
-// k_deep (K2b): NB ii slots, the pool of their stage-1 survivors, per-stage lists, group leaves
-template <int STEP, int NB>
-struct TileGeoB {
-    static constexpr int PBUF = k2_pbuf(STEP);
-    static constexpr int NW = k2_tx(STEP) * k2_ty(STEP);
-    static constexpr int CP = NB <= 4 ? NW + 512 : NW + 2048;   // pool capacity (>= one full tile)
-    static constexpr size_t OFF_NF = (size_t)NB * PBUF * 4;
-    static constexpr size_t OFF_LOC = OFF_NF + (size_t)CP * 4;
-    static constexpr size_t OFF_LIST = OFF_LOC + (((size_t)CP * 2 + 15) & ~(size_t)15);
-    static constexpr size_t SMEM = OFF_LIST + (size_t)2 * CP * 2;
-};
-
-// k_deep1: one ii slot, a pool chunk of CP survivors and its two per-stage lists
-// k_ws (warp-specialised K2): 256 stage-1 threads + WS_DEEP deep-stage threads per CTA.  The
-// stage-1 group streams tiles (ii + sqii planes by TMA, variance, dense stage 1); each tile's
-// ii plane and stage-1 survivors are handed to the deep group in a second buffer, which runs
-// stages 1.. while the stage-1 group moves on.
-#ifndef FD_WS_DEEP_WARPS
-#define FD_WS_DEEP_WARPS 2
-#endif
-constexpr int WS_S1 = 256;
-constexpr int WS_DEEP = 32 * FD_WS_DEEP_WARPS;
-constexpr int WS_THREADS = WS_S1 + WS_DEEP;
+// f1 (fused tile-local integral + cascade): k_f1 stages the tile's level
+// PIXELS (u8, one 3-D TMA box from the group's level images) and builds the tile-local ii and
+// sqii planes in shared memory -- the same TW x TH layout the TMA'd global planes have, so the
+// stage code (incl. the NVRTC-specialised stages) is shared.  Rectangle sums are differences of
+// ii values, hence independent of the integral's origin (exact, reading R4).
+__host__ __device__ constexpr int f1_nseg(int ph) { return 256 / ph >= 8 ? 8 : (256 / ph >= 4 ? 4 : (256 / ph >= 2 ? 2 : 1)); }
 template <int STEP>
-struct TileGeoW {
+struct TileGeoF {
+    static constexpr int TW = tile_w(STEP), TH = tile_h(STEP);
+    static constexpr int PW = TW - 1, PH = TH - 1;                      // pixel region of a tile
+    static constexpr int U8W = (PW + 15) & ~15;                          // TMA box width (16-B multiple)
+    static constexpr int UB = (U8W * PH + 127) & ~127;                   // one u8 staging buffer
     static constexpr int PBUF = k2_pbuf(STEP);
     static constexpr int NW = k2_tx(STEP) * k2_ty(STEP);
-    static constexpr int CP = NW;                                        // pool: a whole tile
-    static constexpr size_t OFF_B = (size_t)2 * PBUF * 4;                // ii copy for the deep group
-    static constexpr size_t OFF_NF = OFF_B + (size_t)PBUF * 4;
+    static constexpr int CP = NW;
+    static constexpr int QBUF = ((PBUF > NW * 10 / 4 ? PBUF : NW * 10 / 4) + 31) & ~31;
+    static constexpr size_t OFF_T = (size_t)2 * UB;                       // ii plane
+    static constexpr size_t OFF_Q = OFF_T + (size_t)PBUF * 4;             // sqii plane, then the pool
+    static constexpr size_t OFF_NF = OFF_Q;
     static constexpr size_t OFF_LOC = OFF_NF + (size_t)NW * 4;
     static constexpr size_t OFF_LIST = OFF_LOC + (size_t)NW * 2;
-    static constexpr size_t SMEM = OFF_LIST + (size_t)2 * NW * 2;
+    static constexpr size_t OFF_RED = OFF_Q + (size_t)QBUF * 4;          // split-stump partial sums
+    static constexpr size_t SMEM = OFF_RED + (size_t)k2_threads(STEP) * 8;
 };
+#ifndef FD_F1_CTAS
+#define FD_F1_CTAS 4                        // k_f1: resident CTAs per SM the launch bounds target
+#endif
 
 #ifndef FD_K2D_CTAS
 #define FD_K2D_CTAS 8
 #endif
 constexpr int K2D_THREADS = 128;
-template <int STEP>
+template <int STEP, bool F1 = false>
 struct TileGeoD {
     static constexpr int PBUF = k2_pbuf(STEP);
     static constexpr int CP = 512;
     static constexpr size_t OFF_NF = (size_t)PBUF * 4;
     static constexpr size_t OFF_LOC = OFF_NF + (size_t)CP * 4;
     static constexpr size_t OFF_LIST = OFF_LOC + (size_t)CP * 2;
-    static constexpr size_t SMEM = OFF_LIST + (size_t)2 * CP * 2;
+    static constexpr size_t OFF_RED = OFF_LIST + (size_t)2 * CP * 2;     // split-stump partial sums
+    static constexpr size_t OFF_U8 = (OFF_RED + (size_t)K2D_THREADS * 8 + 127) & ~(size_t)127;   // f1 pixels
+    static constexpr size_t SMEM = F1 ? OFF_U8 + (size_t)TileGeoF<STEP>::UB : OFF_U8;
 };
 
 struct LevelDev {
     int W, H, P;            // level size, ii pitch (elements)
+    int PB;                 // f1: u8 level-image pitch (bytes, 16-B multiple >= P)
+    long long u8_off;       // f1: byte offset of the level's block u8[G][H][PB] in the group workspace
     int nx, ny;             // windows along x / y (step aware)
     int band0, nbands;      // K1 bands (per frame)
     int tile0, tiles_x;     // K2 tiles (per frame); tiles_y = ceil(ny / TY)
@@ -175,6 +168,7 @@ struct PlanDev {
     long long lvl_frame;    // K1 level-image bytes per frame
     int k1tiles_per_frame;  // K1 tiles (band x chunk) per frame
     long long ws_elems;     // group workspace elements (all levels, all g)
+    long long u8_bytes;     // f1 group workspace bytes (level images of G frames)
     int G;                  // frames per group (tensor-map extent)
     int filter;             // K1: 1 = binomial 3x3 filtering stage after scaling (f2)
     LevelDev lv[FD_MAX_LEVELS];
@@ -220,7 +214,9 @@ struct alignas(16) CascadeParams {
     uint4* tail_q;                          // tail queue (k_tail.cu), may be null
     unsigned int* tail_count;               // entries appended (may exceed tail_cap: the excess stays in K2)
     int tail_cap;
-    int pad1;
+    int s_tail;                             // windows still alive at stage s_tail go to the tail queue
+    int split_max;                          // deep stages with <= split_max windows use the split-stump mode
+    int f1;                                 // 1: tmaps are u8 level-image maps (k_f1, k_deep1 rebuilds ii)
     uint2* surv;                            // split K2: stage-1 survivors (window index, nf bits)
     uint2* tile_rec;                        // split K2: per tile (offset into surv, count)
     unsigned int* surv_count;
@@ -229,8 +225,8 @@ struct alignas(16) CascadeParams {
     uint4 prec[PREC_MAX * (REC_WORDS / 4)];
 };
 
-// Tail queue entry (k_cascade -> k_tail): x = g(16) | level(8) | stage(8), y = wyi(16) | wxi(16)
-// (window indices in the level's step grid), z = nf bits, w = 0.
+// Tail queue entry (K2 -> k_tail): x = level(8) | stage(8), y = wyi(16) | wxi(16) (window
+// indices in the level's step grid), z = nf bits, w = frame index within the group (32 bit).
 constexpr int TAIL_RP = 25;                 // row pitch of a window's ii region staged by k_tail
 constexpr int TAIL_REC_WORDS = 4 + MAX_CORNERS;   // SoA tail records: nc, theta, left, right, corners
 struct TailParams {
@@ -238,10 +234,12 @@ struct TailParams {
     const unsigned int* count;
     int cap;
     int step;
-    const uint32_t* ws;                     // group workspace (ii plane 0 read)
+    const uint32_t* ws;                     // group workspace (ii plane 0 read); null in f1 mode
+    const uint8_t* lvl8;                    // f1: group level images (the window's ii is rebuilt)
     const LevelDev* lv;
     const uint32_t* trec;                   // [TAIL_REC_WORDS][ns] corner offsets in TAIL_RP pitch
     int ns;
+    int j0, nsm;                            // records of stumps [j0, j0 + nsm) are staged in shared memory
     const StageDev* stages;
     int n_stages;
     int frame_base;
@@ -283,12 +281,13 @@ cudaError_t launch_k1_tiles_canonical(const uint8_t* img, const PlanDev& plan, i
 cudaError_t launch_pyramid(const uint8_t* frames, const PlanDev& plan, int n, uint8_t* levels,
                            long long frame_stride, const long long* lvl_off_host, cudaStream_t st);
 cudaError_t launch_cascade(const CascadeParams& p, bool depth_mode, int step, int grid, cudaStream_t st);
+// f1: level images of a frame group (u8, level-major, pitch PB) and the fused tile-local kernel
+cudaError_t launch_levels(const uint8_t* frames, const PlanDev& plan, int g_frames, uint8_t* out, cudaStream_t st);
+cudaError_t launch_f1(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
 cudaError_t launch_tail(const TailParams& p, bool depth_mode, cudaStream_t st);
 // split K2: k_stage1 then k_deep (precompiled kernels; step 1 normally runs the NVRTC ones)
 cudaError_t launch_stage1(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
-cudaError_t launch_deep(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
-cudaError_t launch_deep1(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
-cudaError_t launch_ws(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
+cudaError_t launch_deep1(const CascadeParams& p, bool depth_mode, int step, bool f1, cudaStream_t st);
 cudaError_t launch_soft(const CascadeParams& p, bool depth_mode, int step, bool soft, cudaStream_t st);  // k_soft.cu (R8b)
 cudaError_t launch_depth_hist(const uint8_t* depth, int n, long long win_per_frame, const long long* d_win0,
                               int n_levels, int n_stages, long long* hist, int max_span, cudaStream_t st);

@@ -30,9 +30,16 @@
 
 namespace fdk {
 
+// Launch geometry of each kind, fixed when the program is generated (the launch-bound macros
+// of the generated source come from the environment at that moment; never re-read at launch).
+struct KindGeo {
+    int threads = 0;
+    size_t smem = 0;
+};
 struct JitK2 {
     std::string key;                              // generated program (NVRTC source)
-    cudaKernel_t kern[2][JIT_KINDS] = {};         // [depth][kind], compiled on first use
+    KindGeo geo[JIT_KINDS];
+    cudaKernel_t kern[2][JIT_KINDS] = {};         // [depth][kind], compiled on first use (g_jit_mu)
     int grid[2][JIT_KINDS] = {};
 };
 
@@ -158,45 +165,23 @@ int jit_deep_end(const StageDev* st, int n_stages) {
     return k;
 }
 
+static int env_or(const char* name, int dflt) {
+    const char* e = std::getenv(name);
+    return e && *e ? std::atoi(e) : dflt;
+}
+
 // resident CTAs per SM targeted by the fused kernel's launch bounds (FD_K2_CTAS, 2..6)
-int jit_ctas() {
-    int c = FD_K2_CTAS;
-    if (const char* e = std::getenv("FD_K2_CTAS")) c = std::atoi(e);
+static int jit_ctas() {
+    const int c = env_or("FD_K2_CTAS", FD_K2_CTAS);
     return c < 2 ? 2 : (c > 6 ? 6 : c);
-}
-
-// tiles per k_deep batch of the specialised kernel (FD_K2B_NB, 1..8; default FD_K2B_NB of the build)
-int jit_nb_deep() {
-    int nb = FD_K2B_NB;
-    if (const char* e = std::getenv("FD_K2B_NB")) nb = std::atoi(e);
-    return nb < 1 ? 1 : (nb > 8 ? 8 : nb);
-}
-
-size_t jit_smem_deep(int nb) {
-    switch (nb) {
-        case 1: return TileGeoB<JIT_STEP, 1>::SMEM;
-        case 2: return TileGeoB<JIT_STEP, 2>::SMEM;
-        case 3: return TileGeoB<JIT_STEP, 3>::SMEM;
-        case 4: return TileGeoB<JIT_STEP, 4>::SMEM;
-        case 5: return TileGeoB<JIT_STEP, 5>::SMEM;
-        case 6: return TileGeoB<JIT_STEP, 6>::SMEM;
-        case 7: return TileGeoB<JIT_STEP, 7>::SMEM;
-        default: return TileGeoB<JIT_STEP, 8>::SMEM;
-    }
-}
-
-static int jit_ws_deep_warps() {
-    const char* e = std::getenv("FD_WS_DEEP_WARPS");
-    return e ? std::atoi(e) : FD_WS_DEEP_WARPS;
 }
 
 std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages) {
     const int k_end = jit_deep_end(st, n_stages);
-    std::string src = std::string(std::getenv("FD_POOL_SEPARATE") ? "#define FD_POOL_SEPARATE 1\n" : "") +
-                      "#define FD_K2D_CTAS " + std::to_string(std::getenv("FD_K2D_CTAS") ? std::atoi(std::getenv("FD_K2D_CTAS")) : FD_K2D_CTAS) +
-                      "\n#define FD_WS_DEEP_WARPS " + std::to_string(jit_ws_deep_warps()) +
-                      "\n#define FD_K2_CTAS " + std::to_string(jit_ctas()) + "\n#define FD_K2B_NB " +
-                      std::to_string(jit_nb_deep()) + "\n#include \"fd_internal.h\"\n" + jit_stage1_source(rec_words, st[0].first, st[0].n) +
+    std::string src = "#define FD_K2D_CTAS " + std::to_string(env_or("FD_K2D_CTAS", FD_K2D_CTAS)) +
+                      "\n#define FD_F1_CTAS " + std::to_string(env_or("FD_F1_CTAS", FD_F1_CTAS)) +
+                      "\n#define FD_K2_CTAS " + std::to_string(jit_ctas()) +
+                      "\n#include \"fd_internal.h\"\n" + jit_stage1_source(rec_words, st[0].first, st[0].n) +
                       "#define FD_JIT_STAGE1 1\n";
     if (k_end > 1) src += jit_deep_source(rec_words, st, k_end) + "#define FD_JIT_DEEP " + std::to_string(k_end) + "\n";
     return src + "#include \"k_cascade.cu\"\n";
@@ -206,22 +191,20 @@ static std::string jit_name(int kind, bool depth) {
     const std::string d = depth ? "true" : "false";
     if (kind == JIT_FUSED) return "fdk::k_cascade<1, " + d + ">";
     if (kind == JIT_STAGE1) return "fdk::k_stage1<1, " + d + ">";
-    if (kind == JIT_DEEP1) return "fdk::k_deep1<1, " + d + ">";
-    if (kind == JIT_WS) return "fdk::k_ws<1, " + d + ">";
-    return "fdk::k_deep<1, " + d + ", " + std::to_string(jit_nb_deep()) + ">";
+    if (kind == JIT_DEEP1) return "fdk::k_deep1<1, " + d + ", false>";
+    if (kind == JIT_DEEP1_F1) return "fdk::k_deep1<1, " + d + ", true>";
+    return "fdk::k_f1<1, " + d + ">";
 }
 
-static int jit_kind_threads(int kind) {
-    return kind == JIT_DEEP1 ? K2D_THREADS : (kind == JIT_WS ? WS_S1 + 32 * jit_ws_deep_warps() : k2_threads(JIT_STEP));
-}
-
-static size_t jit_kind_smem(int kind) {
-    if (kind == JIT_FUSED)
-        return TileGeo<JIT_STEP>::SMEM + (std::getenv("FD_POOL_SEPARATE") ? (size_t)TileGeo<JIT_STEP>::NW * 10 : 0);
-    if (kind == JIT_STAGE1) return TileGeoA<JIT_STEP>::SMEM;
-    if (kind == JIT_DEEP1) return TileGeoD<JIT_STEP>::SMEM;
-    if (kind == JIT_WS) return TileGeoW<JIT_STEP>::SMEM;
-    return jit_smem_deep(jit_nb_deep());
+static KindGeo jit_kind_geo(int kind) {
+    KindGeo g;
+    g.threads = (kind == JIT_DEEP1 || kind == JIT_DEEP1_F1) ? K2D_THREADS : k2_threads(JIT_STEP);
+    if (kind == JIT_FUSED) g.smem = TileGeo<JIT_STEP>::SMEM;
+    if (kind == JIT_STAGE1) g.smem = TileGeoA<JIT_STEP>::SMEM;
+    if (kind == JIT_DEEP1) g.smem = TileGeoD<JIT_STEP, false>::SMEM;
+    if (kind == JIT_DEEP1_F1) g.smem = TileGeoD<JIT_STEP, true>::SMEM;
+    if (kind == JIT_F1) g.smem = TileGeoF<JIT_STEP>::SMEM;
+    return g;
 }
 
 bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cubin, std::vector<std::string>* lowered,
@@ -270,6 +253,7 @@ JitK2* jit_k2_build(const uint32_t* rec_words, const StageDev* st, int n_stages,
     (void)err;
     std::unique_ptr<JitK2> J(new JitK2());
     J->key = jit_program(rec_words, st, n_stages);
+    for (int k = 0; k < JIT_KINDS; ++k) J->geo[k] = jit_kind_geo(k);
     return J.release();
 }
 
@@ -287,46 +271,56 @@ std::map<std::pair<std::string, int>, Loaded> g_jit_cache;
 
 cudaError_t jit_k2_launch(JitK2* J, const CascadeParams& p, bool depth, int kind, cudaStream_t st, std::string* err) {
     const int d = depth ? 1 : 0;
-    if (!J->kern[d][0]) {
+    cudaKernel_t kern = nullptr;
+    int kgrid = 0;
+    {
+        // compile / load once per (program, depth); the handle's kernel table is read and
+        // published under the same lock, so concurrent launches on other streams never see a
+        // half-filled table
         std::lock_guard<std::mutex> lk(g_jit_mu);
-        Loaded& L = g_jit_cache[{J->key, d}];
-        if (!L.kern[0]) {
-            std::vector<char> cubin;
-            std::vector<std::string> lowered;
-            if (!jit_k2_compile(J->key, depth, &cubin, &lowered, err)) {
-                g_jit_cache.erase({J->key, d});
-                return cudaErrorInvalidSource;
+        if (!J->kern[d][0]) {
+            Loaded& L = g_jit_cache[{J->key, d}];
+            if (!L.kern[0]) {
+                std::vector<char> cubin;
+                std::vector<std::string> lowered;
+                if (!jit_k2_compile(J->key, depth, &cubin, &lowered, err)) {
+                    g_jit_cache.erase({J->key, d});
+                    return cudaErrorInvalidSource;
+                }
+                cudaError_t e = cudaLibraryLoadData(&L.lib, cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0);
+                int dev = 0, sms = 0;
+                if (e == cudaSuccess) e = cudaGetDevice(&dev);
+                if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+                for (int k = 0; k < JIT_KINDS && e == cudaSuccess; ++k) {
+                    int per = 0;
+                    const KindGeo& g = J->geo[k];
+                    e = cudaLibraryGetKernel(&L.kern[k], L.lib, lowered[k].c_str());
+                    if (e == cudaSuccess)
+                        e = cudaKernelSetAttributeForDevice(L.kern[k], cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                            (int)g.smem, dev);
+                    if (e == cudaSuccess)
+                        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, reinterpret_cast<const void*>(L.kern[k]),
+                                                                          g.threads, g.smem);
+                    L.grid[k] = sms * (per > 0 ? per : 1);
+                }
+                if (e != cudaSuccess) {
+                    *err = std::string("JIT kernel load: ") + cudaGetErrorString(e);
+                    g_jit_cache.erase({J->key, d});
+                    return e;
+                }
             }
-            cudaError_t e = cudaLibraryLoadData(&L.lib, cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0);
-            int dev = 0, sms = 0;
-            if (e == cudaSuccess) e = cudaGetDevice(&dev);
-            if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-            for (int k = 0; k < JIT_KINDS && e == cudaSuccess; ++k) {
-                int per = 0;
-                const size_t smem = jit_kind_smem(k);
-                e = cudaLibraryGetKernel(&L.kern[k], L.lib, lowered[k].c_str());
-                if (e == cudaSuccess)
-                    e = cudaKernelSetAttributeForDevice(L.kern[k], cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem, dev);
-                if (e == cudaSuccess)
-                    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, reinterpret_cast<const void*>(L.kern[k]),
-                                                                      jit_kind_threads(k), smem);
-                L.grid[k] = sms * (per > 0 ? per : 1);
-            }
-            if (e != cudaSuccess) {
-                *err = std::string("JIT kernel load: ") + cudaGetErrorString(e);
-                g_jit_cache.erase({J->key, d});
-                return e;
+            for (int k = 0; k < JIT_KINDS; ++k) {
+                J->kern[d][k] = L.kern[k];
+                J->grid[d][k] = L.grid[k];
             }
         }
-        for (int k = 0; k < JIT_KINDS; ++k) {
-            J->kern[d][k] = L.kern[k];
-            J->grid[d][k] = L.grid[k];
-        }
+        kern = J->kern[d][kind];
+        kgrid = J->grid[d][kind];
     }
-    const int grid = J->grid[d][kind] < p.total_tiles ? J->grid[d][kind] : p.total_tiles;
+    const int grid = kgrid < p.total_tiles ? kgrid : p.total_tiles;
     void* args[] = {const_cast<CascadeParams*>(&p)};
-    return cudaLaunchKernel(reinterpret_cast<const void*>(J->kern[d][kind]), dim3(grid),
-                            dim3(jit_kind_threads(kind)), args, jit_kind_smem(kind), st);
+    return cudaLaunchKernel(reinterpret_cast<const void*>(kern), dim3(grid), dim3(J->geo[kind].threads), args,
+                            J->geo[kind].smem, st);
 }
 
 void jit_k2_free(JitK2* J) { delete J; }    // loaded code stays in the process-wide cache

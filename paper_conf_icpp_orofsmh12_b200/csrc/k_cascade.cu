@@ -141,10 +141,31 @@ __device__ __forceinline__ void phase_sync() {
         asm volatile("bar.sync %0, %1;" ::"n"(BAR), "n"(THREADS) : "memory");
 }
 
+// Split-stump partial sums: the stumps first + q, first + q + wpb, ... of a stage for one window
+// (sequential fp32 sums of the leaves and of their magnitudes); records warp-uniform.
+template <int MC, class R>
+__device__ __forceinline__ void split_partial(const uint32_t* __restrict__ T, int b, float nf, const R& rec, int first,
+                                              int n, int q, int wpb, float& acc, float& aacc) {
+    for (int j = q; j < n; j += wpb) {
+        const float l = eval_stump_mc<MC>(T, b, nf, rec, first + j);
+        acc = __fadd_rn(acc, l);
+        aacc = __fadd_rn(aacc, fabsf(l));
+    }
+}
+template <class R>
+__device__ __forceinline__ void split_partial_mc(const uint32_t* __restrict__ T, int b, float nf, const R& rec, int first,
+                                                 int n, int mc, int q, int wpb, float& acc, float& aacc) {
+    if (mc <= 6) return split_partial<6>(T, b, nf, rec, first, n, q, wpb, acc, aacc);
+    if (mc <= 8) return split_partial<8>(T, b, nf, rec, first, n, q, wpb, acc, aacc);
+    if (mc <= 9) return split_partial<9>(T, b, nf, rec, first, n, q, wpb, acc, aacc);
+    return split_partial<MAX_CORNERS>(T, b, nf, rec, first, n, q, wpb, acc, aacc);
+}
+
+// red: THREADS / 32 x 32 float2 of shared memory for the split-stump mode (nullptr: not used)
 template <int STEP, bool DEPTH, int CP, int THREADS = k2_threads(STEP), int TID0 = 0, int BAR = 0>
 __device__ __forceinline__ void deep_phase(const CascadeParams& p, int s0, const uint32_t* __restrict__ slots,
                                            const float* pnf, const uint16_t* ploc, uint16_t* lists, int* s_cnt,
-                                           int& s_tpos, const WinOut<STEP, DEPTH>& out) {
+                                           int& s_tpos, const WinOut<STEP, DEPTH>& out, float2* red = nullptr) {
     constexpr int TX = k2_tx(STEP), TW = tile_w(STEP), PBUF = k2_pbuf(STEP);
     const int tid = (int)threadIdx.x - TID0, warp = tid >> 5, lane = tid & 31;
     const int lane_min = min(p.lane_min, THREADS / 2 + 1);
@@ -171,6 +192,65 @@ __device__ __forceinline__ void deep_phase(const CascadeParams& p, int s0, const
         // stages [1, FD_JIT_DEEP) of the run-time specialised kernel: immediate-offset code,
         // always one lane per window
         const bool jit_s = FD_JIT_DEEP > 0 && s < FD_JIT_DEEP;
+        if (red && n <= p.split_max && n <= 2 * 32 && THREADS >= 64) {
+            // split-stump mode (few windows): lanes = windows (blocks of 32), the WARPS / nb warps
+            // of a block each evaluate every wpb-th stump of the stage for all the block's
+            // windows with warp-uniform records, so a stage costs ~n_s / wpb stump evaluations of
+            // latency instead of n_s.  The partial sums are added in a fixed order (q = 0, 1, ..)
+            // and the decision is certified against the rounding bound of that summation tree
+            // (k_common.cuh certify: leaf depth <= ceil(n_s / wpb) - 1 + wpb - 1); near ties and
+            // output scores are recomputed with the definition's sequential sum.
+            constexpr int WARPS = THREADS / 32;
+            const int nb = (n + 31) >> 5;
+            const int wpb = WARPS / nb;
+            const int bk = warp / wpb, q = warp - bk * wpb;
+            const int e = bk * 32 + lane;
+            const bool act = bk < nb && e < n;
+            int pe = 0, sl = 0, idx = 0, b = 0;
+            float nfw = 1.0f;
+            if (act) {
+                pe = s == s0 ? e : lin[e];
+                const int loc = ploc[pe];
+                sl = loc >> 11;
+                idx = loc & 2047;
+                b = sl * PBUF + (idx / TX) * STEP * TW + (idx % TX) * STEP;
+                nfw = pnf[pe];
+            }
+            const bool in_param = sd.first + sd.n <= p.n_pstumps;
+            float acc = 0.0f, aacc = 0.0f;
+            if (act) {
+                if (in_param)
+                    split_partial_mc(slots, b, nfw, prec, sd.first, sd.n, sd.mc, q, wpb, acc, aacc);
+                else
+                    split_partial_mc(slots, b, nfw, grec, sd.first, sd.n, sd.mc, q, wpb, acc, aacc);
+            }
+            red[warp * 32 + lane] = make_float2(acc, aacc);
+            phase_sync<BAR, THREADS>();
+            if (act && q == 0) {
+                float t = 0.0f, ta = 0.0f;
+                for (int r = 0; r < wpb; ++r) {
+                    const float2 v = red[(bk * wpb + r) * 32 + lane];
+                    t = __fadd_rn(t, v.x);
+                    ta = __fadd_rn(ta, v.y);
+                }
+                int dec = certify(t, ta, sd.n, (sd.n + wpb - 1) / wpb + wpb, sd.T);
+                float sum = t;
+                if (dec < 0 || (dec == 1 && last) || (DEPTH && dec == 0)) {
+                    sum = in_param ? eval_stage(slots, b, nfw, prec, sd.first, sd.n, sd.mc)
+                                   : eval_stage(slots, b, nfw, grec, sd.first, sd.n, sd.mc);
+                    dec = sum >= sd.T ? 1 : 0;
+                }
+                if (dec == 1) {
+                    if (last)
+                        emit(sl, idx, sum);
+                    else
+                        lout[atomicAdd(&s_cnt[(s + 1) % 3], 1)] = (uint16_t)pe;
+                } else {
+                    reject(sl, idx, s, sum);
+                }
+            }
+            return;
+        }
         if (!jit_s && n < lane_min) {
             // fewer windows than half the block: GL = 2^lg lanes per window (the largest
             // power of two with n*GL <= THREADS, so one pass covers every window and
@@ -260,7 +340,7 @@ __device__ __forceinline__ void deep_phase(const CascadeParams& p, int s0, const
         const int n = s_cnt[s % 3];
         if (tid == 0 && p.stage_counts && n) atomicAdd(p.stage_counts + s, (unsigned long long)n);
         if (n == 0) break;
-        if (n <= tail_n && !(FD_JIT_DEEP > 0 && s < FD_JIT_DEEP)) {
+        if ((n <= tail_n && !(FD_JIT_DEEP > 0 && s < FD_JIT_DEEP)) || (s >= p.s_tail && p.tail_q)) {
             // tail: few windows left.  They go to the global tail queue (finished by
             // k_tail, one warp per window) so this CTA moves on to its next tiles instead of
             // waiting for its deepest window; whatever does not fit in the queue is finished
@@ -274,10 +354,10 @@ __device__ __forceinline__ void deep_phase(const CascadeParams& p, int s0, const
                 const int loc = ploc[pe];
                 const int sl = loc >> 11, idx = loc & 2047;
                 uint4 q;
-                q.x = ((unsigned)(s_frame[sl] - p.frame_base) << 16) | ((unsigned)s_lvl[sl] << 8) | (unsigned)s;
+                q.x = ((unsigned)s_lvl[sl] << 8) | (unsigned)s;
                 q.y = ((unsigned)(s_wy0[sl] + idx / TX) << 16) | (unsigned)(s_wx0[sl] + idx % TX);
                 q.z = (unsigned)__float_as_int(pnf[pe]);
-                q.w = 0u;
+                q.w = (unsigned)(s_frame[sl] - p.frame_base);
                 p.tail_q[tpos + e] = q;
             }
             for (int e = warp; e < n; e += THREADS / 32) {
@@ -476,7 +556,8 @@ __global__ void __launch_bounds__(k2_threads(STEP), FD_K2_CTAS) k_cascade(const 
         }
 #endif
         __syncthreads();                          // pool complete
-        deep_phase<STEP, DEPTH, CP>(p, 1, T, pnf, ploc, lists, s_cnt, s_tpos, out);
+        deep_phase<STEP, DEPTH, CP>(p, 1, T, pnf, ploc, lists, s_cnt, s_tpos, out,
+                                    reinterpret_cast<float2*>(smem_raw + G::OFF_RED));
     }
 }
 
@@ -657,127 +738,112 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
     }
 }
 
-// ======================================================================== split K2, kernel b
-// k_deep: the deeper stages.  A CTA claims tiles in order, skips those without survivors, TMAs
-// each claimed tile's ii plane into one of NB slots and copies its survivors into the pool, then
-// runs deep_phase over the whole batch -- NB tiles' worth of windows per stage-synchronous step
-// (c3: ~110 windows enter stage 2 per tile) instead of one tile's.
-template <int STEP, bool DEPTH, int NB>
-__global__ void __launch_bounds__(k2_threads(STEP), k2b_min_ctas(NB)) k_deep(const __grid_constant__ CascadeParams p) {
-    using G = TileGeoB<STEP, NB>;
-    constexpr int CP = G::CP, PBUF = G::PBUF, PLANE = tile_w(STEP) * tile_h(STEP), THREADS = k2_threads(STEP);
-    static_assert(G::NW <= 2048 && NB <= 8, "pool entries pack slot:3 | window:11");
-    extern __shared__ __align__(1024) uint8_t smem_raw[];
-    uint32_t* slots = reinterpret_cast<uint32_t*>(smem_raw);
-    float* pnf = reinterpret_cast<float*>(smem_raw + G::OFF_NF);
-    uint16_t* ploc = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LOC);
-    uint16_t* lists = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LIST);
-    __shared__ __align__(8) uint64_t mbar[NB];
-    __shared__ int s_frame[NB], s_lvl[NB], s_wx0[NB], s_wy0[NB];
-    __shared__ int s_cnt[3];
-    __shared__ int s_tpos, s_tile, s_carry, s_stop, s_off, s_n, s_base;
+// ======================================================================== f1: fused K2
+// the tile's integral images are built in shared memory from its level pixels,
+// so no ii / sqii plane ever makes an HBM round trip (the paper's integral kernels take "20% of
+// the total" time; P:L368-384 scan + transpose).  The level pixels of a tile's
+// (TW-1) x (TH-1) region arrive as one 3-D TMA box (u8, 5.3 KB at step 1, double buffered so the
+// next tile's box is in flight while this tile is evaluated).
+//
+// Tile-local integral (reading R4: every rectangle sum is a difference of four ii values, so the
+// origin of the integral does not matter; tile-local sums are < 2^32, so u32 is exact):
+//   row pass    thread (r, s) owns pixel row r, columns [s*SEGW, (s+1)*SEGW): it sums its segment,
+//               the NSEG segments of a row (adjacent lanes) exchange exclusive offsets with
+//               shuffles, then it writes running row prefixes of p and p^2 into rows 1.. of T / Q;
+//   column pass thread per (column, plane) adds down the TH-1 rows (loads batched 8 at a time).
+// Row 0 and column 0 of both planes are zero.  Ends with a block barrier.
+// THREADS: block size; WITH_Q: also build the sqii plane (k_f1; k_deep1 rebuilds ii only)
+template <int STEP, int THREADS = k2_threads(STEP), bool WITH_Q = true>
+__device__ __forceinline__ void build_tile_integral(const uint8_t* __restrict__ U, uint32_t* __restrict__ T,
+                                                    uint32_t* __restrict__ Q) {
+    using G = TileGeoF<STEP>;
+    constexpr int TW = G::TW, TH = G::TH, PW = G::PW, PH = G::PH, U8W = G::U8W;
+    constexpr int NSEG = f1_nseg(PH * 256 / THREADS), SEGW = (PW + NSEG - 1) / NSEG;
+    constexpr bool KEEP = SEGW <= 24;          // segment pixels kept in registers between the sweeps
+    static_assert(NSEG * PH <= THREADS && (32 % NSEG) == 0, "row-pass jobs must fit one pass of the block");
+    (void)Q;
     const int tid = threadIdx.x;
-    const WinOut<STEP, DEPTH> out{p, s_frame, s_lvl, s_wx0, s_wy0};
-    if (tid == 0) {
-        for (int i = 0; i < NB; ++i) mbar_init(&mbar[i], 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        s_carry = -1;
+    const int r = tid / NSEG, sg = tid % NSEG;
+    const bool act = r < PH;
+    const int c0 = sg * SEGW;
+    const uint8_t* row = U + r * U8W + c0;
+    // sweep 1: segment totals (only the last segment can reach past PW)
+    uint32_t px[KEEP ? SEGW : 1];
+    uint32_t ts = 0, tq = 0;
+#pragma unroll
+    for (int i = 0; i < SEGW; ++i) {
+        const uint32_t v = (act && c0 + i < PW) ? (uint32_t)row[i] : 0u;
+        if constexpr (KEEP) px[i] = v;
+        ts += v;
+        tq += v * v;
     }
-    uint32_t phases = 0;
-    for (;;) {
-        int nb = 0;
-#ifdef FD_K2_TIMING
-        const long long tf0 = clock64();
-#endif
-        for (;;) {
-            __syncthreads();
-            if (tid == 0) {
-                if (nb == 0) {
-                    s_cnt[0] = 0;
-                    s_cnt[1] = 0;
-                    s_cnt[2] = 0;
-                }
-                int tn;
-                uint2 tr = make_uint2(0u, 0u);
-                if (s_carry >= 0) {
-                    tn = s_carry;
-                    s_carry = -1;
-                    tr = p.tile_rec[tn];
-                } else {
-                    do {
-                        tn = (int)atomicAdd(p.deep_counter, 1u);
-                        if (tn >= p.total_tiles) break;
-                        tr = p.tile_rec[tn];
-                    } while (tr.y == 0u);
-                }
-                s_tile = tn;
-                s_stop = 0;
-                if (tn < p.total_tiles) {
-                    if (s_cnt[p.s0 % 3] + (int)tr.y > CP) {
-                        s_carry = tn;             // does not fit: first tile of the next batch
-                        s_stop = 1;
-                    } else {
-                        const TileAt t = tile_at<STEP>(p, tn);
-                        s_frame[nb] = p.frame_base + t.g;
-                        s_lvl[nb] = t.k;
-                        s_wx0[nb] = t.wx0;
-                        s_wy0[nb] = t.wy0;
-                        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                        mbar_expect_tx(&mbar[nb], PLANE * 4);
-                        tma_load_4d(slots + nb * PBUF, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar[nb]);
-                        s_off = (int)tr.x;
-                        s_n = (int)tr.y;
-                        s_base = s_cnt[p.s0 % 3];
-                        s_cnt[p.s0 % 3] += (int)tr.y;
-                    }
-                }
-            }
-            __syncthreads();
-            if (s_tile >= p.total_tiles || s_stop) break;
-            {
-                const int off = s_off, n = s_n, b0 = s_base;
-                for (int e = tid; e < n; e += THREADS) {
-                    const uint2 v = p.surv[off + e];
-                    ploc[b0 + e] = (uint16_t)((nb << 11) | (int)v.x);
-                    pnf[b0 + e] = __int_as_float((int)v.y);
-                }
-            }
-            if (++nb == NB) break;
+    uint32_t is = ts, iq = tq;                  // inclusive scan over the row's segments
+#pragma unroll
+    for (int d = 1; d < NSEG; d <<= 1) {
+        const uint32_t a = __shfl_up_sync(0xffffffffu, is, d, NSEG);
+        const uint32_t b = __shfl_up_sync(0xffffffffu, iq, d, NSEG);
+        if (sg >= d) {
+            is += a;
+            iq += b;
         }
-        if (nb == 0) break;
-#ifdef FD_K2_TIMING
-        const long long tf1 = clock64();
-#endif
-        for (int i = 0; i < nb; ++i) {
-            mbar_wait(&mbar[i], (phases >> i) & 1u);
-            phases ^= 1u << i;
-        }
-        __syncthreads();                          // pool copies visible
-#ifdef FD_K2_TIMING
-        if (tid == 0) {
-            atomicAdd(&g_k2_timing[90], (unsigned long long)(tf1 - tf0));
-            atomicAdd(&g_k2_timing[91], (unsigned long long)(clock64() - tf1));
-            atomicAdd(&g_k2_timing[92], (unsigned long long)nb);
-            atomicAdd(&g_k2_timing[93], (unsigned long long)s_cnt[p.s0 % 3]);
-        }
-#endif
-        deep_phase<STEP, DEPTH, CP>(p, p.s0, slots, pnf, ploc, lists, s_cnt, s_tpos, out);
     }
+    // sweep 2: running row prefixes of p and p^2 (exclusive segment offset + segment prefix)
+    if (act) {
+        uint32_t rs = is - ts, rq = iq - tq;
+        uint32_t* To = T + (r + 1) * TW + 1 + c0;
+        uint32_t* Qo = WITH_Q ? Q + (r + 1) * TW + 1 + c0 : nullptr;
+#pragma unroll
+        for (int i = 0; i < SEGW; ++i) {
+            uint32_t v;
+            if constexpr (KEEP)
+                v = px[i];
+            else
+                v = c0 + i < PW ? (uint32_t)row[i] : 0u;
+            rs += v;
+            rq += v * v;
+            if (c0 + i < PW) {
+                To[i] = rs;
+                if constexpr (WITH_Q) Qo[i] = rq;
+            }
+        }
+    }
+    for (int i = tid; i < TW; i += THREADS) {
+        T[i] = 0u;
+        if constexpr (WITH_Q) Q[i] = 0u;
+    }
+    for (int i = tid; i < TH; i += THREADS) {
+        T[i * TW] = 0u;
+        if constexpr (WITH_Q) Q[i * TW] = 0u;
+    }
+    __syncthreads();
+    // column pass: thread per (column, plane), every row unrolled (independent loads, one add
+    // chain)
+    for (int j = tid; j < (WITH_Q ? 2 : 1) * PW; j += THREADS) {
+        uint32_t* P = (j < PW ? T : Q) + 1 + (j < PW ? j : j - PW);
+        uint32_t acc = 0;
+#pragma unroll
+        for (int y = 1; y < TH; ++y) {
+            acc += P[y * TW];
+            P[y * TW] = acc;
+        }
+    }
+    __syncthreads();
 }
 
 // k_deep1: the deeper stages, one tile per (small) CTA and many CTAs per SM.  Each CTA claims a
 // tile with stage-1 survivors, TMAs its ii plane and runs deep_phase over the survivors (in
 // chunks of CP); with ~25 KB of shared memory and 4 warps per CTA, FD_K2D_CTAS tiles are in
 // flight per SM, so the latency-bound stage chains of different tiles overlap.
-template <int STEP, bool DEPTH>
+template <int STEP, bool DEPTH, bool F1 = false>
 __global__ void __launch_bounds__(K2D_THREADS, FD_K2D_CTAS) k_deep1(const __grid_constant__ CascadeParams p) {
-    using G = TileGeoD<STEP>;
+    using G = TileGeoD<STEP, F1>;
     constexpr int CP = G::CP, PLANE = tile_w(STEP) * tile_h(STEP);
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint32_t* slot = reinterpret_cast<uint32_t*>(smem_raw);
     float* pnf = reinterpret_cast<float*>(smem_raw + G::OFF_NF);
     uint16_t* ploc = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LOC);
     uint16_t* lists = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LIST);
+    uint8_t* U = smem_raw + G::OFF_U8;                                       // f1: level pixels (TMA)
     __shared__ __align__(8) uint64_t mbar;
     __shared__ int s_frame[1], s_lvl[1], s_wx0[1], s_wy0[1];
     __shared__ int s_cnt[3];
@@ -807,8 +873,13 @@ __global__ void __launch_bounds__(K2D_THREADS, FD_K2D_CTAS) k_deep1(const __grid
                 s_wx0[0] = t.wx0;
                 s_wy0[0] = t.wy0;
                 asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                mbar_expect_tx(&mbar, PLANE * 4);
-                tma_load_4d(slot, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar);
+                if (F1) {       // the tile's level pixels; its ii plane is rebuilt below
+                    mbar_expect_tx(&mbar, TileGeoF<STEP>::U8W * TileGeoF<STEP>::PH);
+                    tma_load_3d(U, p.tmaps + t.k, t.x, t.y, t.g, &mbar);
+                } else {
+                    mbar_expect_tx(&mbar, PLANE * 4);
+                    tma_load_4d(slot, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar);
+                }
                 s_off = (int)tr.x;
                 s_n = (int)tr.y;
             }
@@ -833,241 +904,196 @@ __global__ void __launch_bounds__(K2D_THREADS, FD_K2D_CTAS) k_deep1(const __grid
             if (c0 == 0) {
                 mbar_wait(&mbar, phase);
                 phase ^= 1;
+                if constexpr (F1) build_tile_integral<STEP, K2D_THREADS, false>(U, slot, nullptr);
             }
             __syncthreads();
-            deep_phase<STEP, DEPTH, CP, K2D_THREADS>(p, p.s0, slot, pnf, ploc, lists, s_cnt, s_tpos, out);
+            deep_phase<STEP, DEPTH, CP, K2D_THREADS>(p, p.s0, slot, pnf, ploc, lists, s_cnt, s_tpos, out,
+                                                     reinterpret_cast<float2*>(smem_raw + G::OFF_RED));
         }
     }
 }
 
-
-// ======================================================================== warp-specialised K2
-// k_ws: one persistent CTA = a stage-1 warp group (WS_S1 threads) + a deep warp group (WS_DEEP
-// threads), 2 CTAs per SM.  The stage-1 group claims tiles, TMAs their ii + sqii planes, computes
-// the variance normalisation and the dense first stage exactly as k_stage1, then (once the deep
-// group has released the hand-off buffer) ballot-compacts the survivors into the pool and copies
-// the ii plane into the hand-off buffer B; the deep group runs deep_phase (stages 1..N-1,
-// named barrier 2) over the pool while the stage-1 group already streams the next tile.  The
-// hand-off is a one-slot pipeline on two mbarriers: FULL (every stage-1 thread arrives after
-// its pool / B writes) and EMPTY (every deep thread arrives when done with B and the pool).
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
-
+// k_f1: persistent over every (frame, level, tile) of a frame group, like k_cascade, with the
+// tile's planes built in shared memory (above) instead of TMA'd from a global integral:
+//   TMA box of level pixels -> tile-local ii + sqii -> variance (oracle c5) -> dense first stage
+//   (run-time specialised for step 1) -> ballot compaction into the pool (over the dead sqii
+//   plane) -> deep_phase (stages 1.., tail queue once few windows remain; k_tail rebuilds the
+//   window's 25 x 25 ii from the same level image).
 template <int STEP, bool DEPTH>
-__global__ void __launch_bounds__(WS_THREADS, 2) k_ws(const __grid_constant__ CascadeParams p) {
-    using G = TileGeoW<STEP>;
-    constexpr int TW = tile_w(STEP), TX = k2_tx(STEP), TY = k2_ty(STEP), WPT = k2_wpt(STEP), CP = G::CP;
-    constexpr int WARPS_X = TX / 32, PLANE = tile_w(STEP) * tile_h(STEP);
-    static_assert(k2_threads(STEP) == WS_S1, "stage-1 group = the k_stage1 thread layout");
+__global__ void __launch_bounds__(k2_threads(STEP), FD_F1_CTAS) k_f1(const __grid_constant__ CascadeParams p) {
+    using G = TileGeoF<STEP>;
+    constexpr int TW = G::TW, TX = k2_tx(STEP), TY = k2_ty(STEP), WPT = k2_wpt(STEP), CP = G::CP;
+    constexpr int WARPS_X = TX / 32;
     extern __shared__ __align__(1024) uint8_t smem_raw[];
-    uint32_t* T = reinterpret_cast<uint32_t*>(smem_raw);                     // ii plane (TMA)
-    uint32_t* Q = T + G::PBUF;                                               // sqii plane (TMA)
-    uint32_t* B = reinterpret_cast<uint32_t*>(smem_raw + G::OFF_B);          // ii plane of the deep group
-    float* pnf = reinterpret_cast<float*>(smem_raw + G::OFF_NF);
+    uint32_t* T = reinterpret_cast<uint32_t*>(smem_raw + G::OFF_T);           // ii plane
+    uint32_t* Q = reinterpret_cast<uint32_t*>(smem_raw + G::OFF_Q);           // sqii plane
+    float* pnf = reinterpret_cast<float*>(smem_raw + G::OFF_NF);              // pool, over Q after stage 1
     uint16_t* ploc = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LOC);
     uint16_t* lists = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LIST);
-    __shared__ __align__(8) uint64_t mbar_tma, mbar_full, mbar_empty;
-    __shared__ int s_tile, s_pc, s_l1;
-    __shared__ int s_frame[1], s_lvl[1], s_wx0[1], s_wy0[1];                // stage-1 group's tile
-    __shared__ int d_frame[1], d_lvl[1], d_wx0[1], d_wy0[1];                // deep group's tile
-    __shared__ int d_n, d_s0, d_stop, d_cnt[3], d_tpos;
-    const int tid = threadIdx.x;
+    __shared__ __align__(8) uint64_t mbar[2];
+    __shared__ int s_tile[2], s_frame[2], s_lvl[2], s_wx0[2], s_wy0[2];
+    __shared__ int s_cnt[3];
+    __shared__ int s_tpos, s_off;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const StageDev& st0 = p.pstages[0];
+    const ParamRec prec{p};
+    const GlobalRec grec{p.stumps};
+    // tid 0: claim the next tile for u8 buffer b and start its TMA
+    auto claim = [&](int b) {
+        const int tn = (int)atomicAdd(p.tile_counter, 1u);
+        s_tile[b] = tn;
+        if (tn < p.total_tiles) {
+            const TileAt t = tile_at<STEP>(p, tn);
+            s_frame[b] = p.frame_base + t.g;
+            s_lvl[b] = t.k;
+            s_wx0[b] = t.wx0;
+            s_wy0[b] = t.wy0;
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_expect_tx(&mbar[b], G::U8W * G::PH);
+            tma_load_3d(smem_raw + b * G::UB, p.tmaps + t.k, t.x, t.y, t.g, &mbar[b]);
+        }
+    };
     if (tid == 0) {
-        mbar_init(&mbar_tma, 1);
-        mbar_init(&mbar_full, WS_S1);
-        mbar_init(&mbar_empty, WS_DEEP);
+        mbar_init(&mbar[0], 1);
+        mbar_init(&mbar[1], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        claim(0);
     }
-    __syncthreads();
-    if (tid < WS_S1) {
-        // ------------------------------------------------------------ stage-1 group
-        const int warp = tid >> 5, lane = tid & 31;
-        const StageDev& st0 = p.pstages[0];
-        const ParamRec prec{p};
-        const GlobalRec grec{p.stumps};
-        const WinOut<STEP, DEPTH> out{p, s_frame, s_lvl, s_wx0, s_wy0};
-        uint32_t ph_tma = 0, ph_empty = 0;
-        bool first = true;
-        for (;;) {
-            phase_sync<1, WS_S1>();               // planes, s_* free
-            if (tid == 0) {
-                s_pc = 0;
-                const int tn = (int)atomicAdd(p.tile_counter, 1u);
-                s_tile = tn;
-                if (tn < p.total_tiles) {
-                    const TileAt t = tile_at<STEP>(p, tn);
-                    s_frame[0] = p.frame_base + t.g;
-                    s_lvl[0] = t.k;
-                    s_wx0[0] = t.wx0;
-                    s_wy0[0] = t.wy0;
-                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                    mbar_expect_tx(&mbar_tma, 2 * PLANE * 4);
-                    tma_load_4d(T, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar_tma);
-                    tma_load_4d(Q, p.tmaps + t.k, t.x, t.y, 1, t.g, &mbar_tma);
-                }
-            }
-            phase_sync<1, WS_S1>();
-            if (s_tile >= p.total_tiles) break;
-            mbar_wait(&mbar_tma, ph_tma);
-            ph_tma ^= 1;
-            const int k = s_lvl[0];
-            const int nx = __ldg(&p.lv[k].nx), ny = __ldg(&p.lv[k].ny);
-            const int wx0 = s_wx0[0], wy0 = s_wy0[0];
-            const int lx = lane + 32 * (warp % WARPS_X);
-            const int ly0 = (warp / WARPS_X) * WPT;
-            const int base = ly0 * STEP * TW + lx * STEP;
-            const bool colok = wx0 + lx < nx;
-            float nf[WPT], sm[WPT];
+    uint32_t phases = 0;
+    for (int it = 0;; ++it) {
+        const int b = it & 1;
+        if (tid == 0) {
+            s_cnt[0] = 0;
+            s_cnt[1] = 0;
+            s_cnt[2] = 0;
+        }
+        __syncthreads();                          // previous tile done: planes, pool, s_* of slot b^1 free
+        if (s_tile[b] >= p.total_tiles) break;
+        if (tid == 0) claim(b ^ 1);               // the other u8 buffer was consumed by the last build
+#ifdef FD_K2_TIMING
+        const long long tm0 = clock64();
+#endif
+        mbar_wait(&mbar[b], (phases >> b) & 1u);
+        phases ^= 1u << b;
+#ifdef FD_K2_TIMING
+        const long long tm1 = clock64();
+#endif
+        build_tile_integral<STEP>(smem_raw + b * G::UB, T, Q);
+#ifdef FD_K2_TIMING
+        const long long tmb = clock64();
+#endif
+        const WinOut<STEP, DEPTH> out{p, s_frame + b, s_lvl + b, s_wx0 + b, s_wy0 + b};
+        const int k = s_lvl[b];
+        const int nx = __ldg(&p.lv[k].nx), ny = __ldg(&p.lv[k].ny);
+        const int wx0 = s_wx0[b], wy0 = s_wy0[b];
+        const int lx = lane + 32 * (warp % WARPS_X);
+        const int ly0 = (warp / WARPS_X) * WPT;
+        const int base = ly0 * STEP * TW + lx * STEP;
+        const bool colok = wx0 + lx < nx;
+        float nf[WPT], sm[WPT];
 #pragma unroll
-            for (int i = 0; i < WPT; ++i) {
-                const int bo = base + i * STEP * TW;
-                const uint32_t S = T[bo + WIN * TW + WIN] - T[bo + WIN] - T[bo + WIN * TW] + T[bo];
-                const uint32_t q = Q[bo + WIN * TW + WIN] - Q[bo + WIN] - Q[bo + WIN * TW] + Q[bo];
-                const long long v = 576LL * (long long)q - (long long)S * (long long)S;
-                nf[i] = v > 0 ? __fsqrt_rn(__ll2float_rn(v)) : 1.0f;
-                sm[i] = 0.0f;
-            }
+        for (int i = 0; i < WPT; ++i) {
+            const int bo = base + i * STEP * TW;
+            const uint32_t S = T[bo + WIN * TW + WIN] - T[bo + WIN] - T[bo + WIN * TW] + T[bo];
+            const uint32_t q = Q[bo + WIN * TW + WIN] - Q[bo + WIN] - Q[bo + WIN * TW] + Q[bo];
+            const long long v = 576LL * (long long)q - (long long)S * (long long)S;
+            nf[i] = v > 0 ? __fsqrt_rn(__ll2float_rn(v)) : 1.0f;
+            sm[i] = 0.0f;
+        }
 #ifdef FD_JIT_STAGE1
-            jit_stage1(T + base, nf, sm);
+        jit_stage1(T + base, nf, sm);
 #else
-            if (st0.first + st0.n <= p.n_pstumps)
-                dense_stage<WPT, STEP * TW>(T, base, nf, sm, prec, st0.first, st0.n);
-            else
-                dense_stage<WPT, STEP * TW>(T, base, nf, sm, grec, st0.first, st0.n);
+        if (st0.first + st0.n <= p.n_pstumps)
+            dense_stage<WPT, STEP * TW>(T, base, nf, sm, prec, st0.first, st0.n);
+        else
+            dense_stage<WPT, STEP * TW>(T, base, nf, sm, grec, st0.first, st0.n);
 #endif
-            // stage-1 survivors: straight into the pool (s0 == 1) or, when this group also runs
-            // stage 2 (s0 == 2), into a list over the sqii plane (dead once every nf is taken)
-            const bool s2here = p.s0 >= 2 && p.n_stages >= 2;
-            uint2* l1 = reinterpret_cast<uint2*>(Q);
-            if (s2here) {
-                if (tid == 0) s_l1 = 0;
-                phase_sync<1, WS_S1>();           // every sqii read done, s_l1 zeroed
-            }
-            // the hand-off buffer and the pool are free once the deep group has finished the
-            // previous tile
-            if (!first && !s2here) {
-                mbar_wait(&mbar_empty, ph_empty);
-                ph_empty ^= 1;
-            }
+        __syncthreads();                          // every sqii read done: the buffer becomes the pool
 #pragma unroll
-            for (int i = 0; i < WPT; ++i) {
-                const int wy = wy0 + ly0 + i;
-                const bool valid = colok && wy < ny;
-                const bool pass = valid && (sm[i] >= st0.T);
-                const int idx = (ly0 + i) * TX + lx;
-                if (DEPTH && valid && !pass) out.reject(0, idx, 0, sm[i]);
-                if (p.n_stages == 1) {
-                    if (pass) out.emit(0, idx, sm[i]);
-                    continue;
-                }
-                const unsigned m = __ballot_sync(0xffffffffu, pass);
-                if (m) {
-                    int pos = 0;
-                    if (lane == 0) pos = atomicAdd(s2here ? &s_l1 : &s_pc, __popc(m));
-                    pos = __shfl_sync(0xffffffffu, pos, 0);
-                    if (pass) {
-                        const int at = pos + __popc(m & ((1u << lane) - 1u));
-                        if (s2here) {
-                            l1[at] = make_uint2((unsigned)idx, (unsigned)__float_as_int(nf[i]));
-                        } else {
-                            ploc[at] = (uint16_t)idx;
-                            pnf[at] = nf[i];
-                        }
-                    }
+        for (int i = 0; i < WPT; ++i) {
+            const int wy = wy0 + ly0 + i;
+            const bool valid = colok && wy < ny;
+            const bool pass = valid && (sm[i] >= st0.T);
+            const int idx = (ly0 + i) * TX + lx;
+            if (DEPTH && valid && !pass) out.reject(0, idx, 0, sm[i]);
+            if (p.n_stages == 1) {
+                if (pass) out.emit(0, idx, sm[i]);
+                continue;
+            }
+            const unsigned m = __ballot_sync(0xffffffffu, pass);
+            if (m) {
+                int pos = 0;
+                if (lane == 0) pos = atomicAdd(&s_cnt[1], __popc(m));
+                pos = __shfl_sync(0xffffffffu, pos, 0);
+                if (pass) {
+                    const int at = pos + __popc(m & ((1u << lane) - 1u));
+                    ploc[at] = (uint16_t)idx;
+                    pnf[at] = nf[i];
                 }
             }
-            if (s2here) {
-                phase_sync<1, WS_S1>();           // stage-1 survivor list complete
-                if (!first) {
-                    mbar_wait(&mbar_empty, ph_empty);
-                    ph_empty ^= 1;
-                }
-                // stage 2 over the list, one lane per window; survivors into the pool
-                const int c = s_l1;
-                const StageDev& sd = p.pstages[1];
-                const bool last = p.n_stages == 2;
-                if (tid == 0 && p.stage_counts && c) atomicAdd(p.stage_counts + 1, (unsigned long long)c);
-                for (int e0 = warp * 32; e0 < c; e0 += WS_S1) {
-                    const int e = e0 + lane;
-                    const bool act = e < c;
-                    uint2 v = make_uint2(0u, 0u);
-                    float sum = 0.0f;
-                    if (act) {
-                        v = l1[e];
-                        const int idx = (int)v.x;
-                        const int bo = (idx / TX) * STEP * TW + (idx % TX) * STEP;
-                        const float nfw = __int_as_float((int)v.y);
-#if FD_JIT_DEEP > 1
-                        sum = jit_deep(1, T + bo, nfw);
-#else
-                        sum = sd.first + sd.n <= p.n_pstumps ? eval_stage(T, bo, nfw, prec, sd.first, sd.n, sd.mc)
-                                                             : eval_stage(T, bo, nfw, grec, sd.first, sd.n, sd.mc);
+        }
+        if (tid == 0 && p.stage_counts)
+            atomicAdd(p.stage_counts, (unsigned long long)min(TX, nx - wx0) * (unsigned long long)min(TY, ny - wy0));
+        __syncthreads();                          // pool complete
+#ifdef FD_K2_TIMING
+        if (tid == 0) {
+            atomicAdd(&g_k2_timing[0], 1ull);
+            atomicAdd(&g_k2_timing[1], (unsigned long long)(tm1 - tm0));
+            atomicAdd(&g_k2_timing[85], (unsigned long long)(tmb - tm1));
+            atomicAdd(&g_k2_timing[2], (unsigned long long)(clock64() - tmb));
+        }
 #endif
-                    }
-                    const bool pass = act && (sum >= sd.T);
-                    if (act && !pass) out.reject(0, (int)v.x, 1, sum);
-                    if (last) {
-                        if (pass) out.emit(0, (int)v.x, sum);
-                        continue;
-                    }
-                    const unsigned m = __ballot_sync(0xffffffffu, pass);
-                    if (m) {
-                        int pos = 0;
-                        if (lane == 0) pos = atomicAdd(&s_pc, __popc(m));
-                        pos = __shfl_sync(0xffffffffu, pos, 0);
-                        if (pass) {
-                            const int at = pos + __popc(m & ((1u << lane) - 1u));
-                            ploc[at] = (uint16_t)v.x;
-                            pnf[at] = __int_as_float((int)v.y);
-                        }
-                    }
-                }
-            }
-            first = false;
-            {   // ii plane -> hand-off buffer (uint4 copies)
-                const uint4* src = reinterpret_cast<const uint4*>(T);
-                uint4* dst = reinterpret_cast<uint4*>(B);
-                for (int i = tid; i < G::PBUF / 4; i += WS_S1) dst[i] = src[i];
-            }
-            phase_sync<1, WS_S1>();               // pool, B and s_pc complete
-            if (tid == 0) {
-                d_n = p.n_stages <= (p.s0 >= 2 ? 2 : 1) ? 0 : s_pc;
-                d_s0 = p.s0 >= 2 ? 2 : 1;
-                d_frame[0] = s_frame[0];
-                d_lvl[0] = k;
-                d_wx0[0] = wx0;
-                d_wy0[0] = wy0;
-                d_stop = 0;
-                if (p.stage_counts)
-                    atomicAdd(p.stage_counts, (unsigned long long)min(TX, nx - wx0) * (unsigned long long)min(TY, ny - wy0));
-            }
-            mbar_arrive(&mbar_full);
+        if (!p.surv) {
+            deep_phase<STEP, DEPTH, CP>(p, 1, T, pnf, ploc, lists, s_cnt, s_tpos, out,
+                                        reinterpret_cast<float2*>(smem_raw + G::OFF_RED));
+            continue;
         }
-        // no more tiles: stop the deep group once it is idle
-        if (!first) mbar_wait(&mbar_empty, ph_empty);
-        if (tid == 0) d_stop = 1;
-        mbar_arrive(&mbar_full);
-    } else {
-        // ------------------------------------------------------------ deep group
-        const int dt = tid - WS_S1;
-        const WinOut<STEP, DEPTH> out{p, d_frame, d_lvl, d_wx0, d_wy0};
-        uint32_t ph_full = 0;
-        for (;;) {
-            mbar_wait(&mbar_full, ph_full);
-            ph_full ^= 1;
-            if (d_stop) break;
-            const int s0 = d_s0;
-            if (dt == 0) {
-                d_cnt[0] = 0;
-                d_cnt[1] = 0;
-                d_cnt[2] = 0;
-                d_cnt[s0 % 3] = d_n;
-            }
-            phase_sync<2, WS_DEEP>();
-            deep_phase<STEP, DEPTH, CP, WS_DEEP, WS_S1, 2>(p, s0, B, pnf, ploc, lists, d_cnt, d_tpos, out);
-            mbar_arrive(&mbar_empty);
+        // split f1 (p.surv set): stage 1 over the pool here, one lane per window; its survivors
+        // (window index, nf) go to the global list at an offset reserved for this tile, and
+        // k_deep1 rebuilds the tile's ii from the same level image for the deeper stages
+        const int c = s_cnt[1];
+        if (tid == 0) {
+            s_off = c ? (int)atomicAdd(p.surv_count, (unsigned)c) : 0;
+            if (p.stage_counts && c) atomicAdd(p.stage_counts + 1, (unsigned long long)c);
         }
+        __syncthreads();
+        const int off = s_off;
+        const StageDev& sd = p.pstages[1];
+        const bool last = p.n_stages == 2;
+        for (int e0 = warp * 32; e0 < c; e0 += k2_threads(STEP)) {
+            const int e = e0 + lane;
+            const bool act = e < c;
+            int idx = 0;
+            float nfw = 1.0f, sum = 0.0f;
+            if (act) {
+                idx = ploc[e];
+                nfw = pnf[e];
+                const int bo = (idx / TX) * STEP * TW + (idx % TX) * STEP;
+#if FD_JIT_DEEP > 1
+                sum = jit_deep(1, T + bo, nfw);
+#else
+                sum = sd.first + sd.n <= p.n_pstumps ? eval_stage(T, bo, nfw, prec, sd.first, sd.n, sd.mc)
+                                                     : eval_stage(T, bo, nfw, grec, sd.first, sd.n, sd.mc);
+#endif
+            }
+            const bool pass = act && (sum >= sd.T);
+            if (act && !pass) out.reject(0, idx, 1, sum);
+            if (last) {
+                if (pass) out.emit(0, idx, sum);
+                continue;
+            }
+            const unsigned m = __ballot_sync(0xffffffffu, pass);
+            if (m) {
+                int pos = 0;
+                if (lane == 0) pos = atomicAdd(&s_cnt[2], __popc(m));
+                pos = __shfl_sync(0xffffffffu, pos, 0);
+                if (pass)
+                    p.surv[off + pos + __popc(m & ((1u << lane) - 1u))] =
+                        make_uint2((unsigned)idx, (unsigned)__float_as_int(nfw));
+            }
+        }
+        __syncthreads();
+        if (tid == 0) p.tile_rec[s_tile[b]] = make_uint2((unsigned)off, (unsigned)s_cnt[2]);
     }
 }
 
@@ -1143,23 +1169,6 @@ static cudaError_t launch_stage1_t(const CascadeParams& p, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-template <int STEP, bool DEPTH>
-static cudaError_t launch_deep_t(const CascadeParams& p, cudaStream_t st) {
-    static int grid = 0;
-    const size_t smem = TileGeoB<STEP, FD_K2B_NB>::SMEM;
-    cudaError_t e = cudaFuncSetAttribute(k_deep<STEP, DEPTH, FD_K2B_NB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    if (!grid) {
-        int dev = 0, sms = 0, per = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_deep<STEP, DEPTH, FD_K2B_NB>, k2_threads(STEP), smem);
-        grid = sms * (per > 0 ? per : 1);
-    }
-    k_deep<STEP, DEPTH, FD_K2B_NB><<<grid < p.total_tiles ? grid : p.total_tiles, k2_threads(STEP), smem, st>>>(p);
-    return cudaGetLastError();
-}
-
 cudaError_t launch_stage1(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
     switch (step) {
         case 1: return depth ? launch_stage1_t<1, true>(p, st) : launch_stage1_t<1, false>(p, st);
@@ -1170,66 +1179,61 @@ cudaError_t launch_stage1(const CascadeParams& p, bool depth, int step, cudaStre
     }
 }
 
-cudaError_t launch_deep(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
-    switch (step) {
-        case 1: return depth ? launch_deep_t<1, true>(p, st) : launch_deep_t<1, false>(p, st);
-        case 2: return depth ? launch_deep_t<2, true>(p, st) : launch_deep_t<2, false>(p, st);
-        case 3: return depth ? launch_deep_t<3, true>(p, st) : launch_deep_t<3, false>(p, st);
-        case 4: return depth ? launch_deep_t<4, true>(p, st) : launch_deep_t<4, false>(p, st);
-        default: return cudaErrorInvalidValue;
-    }
-}
-
-template <int STEP, bool DEPTH>
+template <int STEP, bool DEPTH, bool F1>
 static cudaError_t launch_deep1_t(const CascadeParams& p, cudaStream_t st) {
     static int grid = 0;
-    const size_t smem = TileGeoD<STEP>::SMEM;
-    cudaError_t e = cudaFuncSetAttribute(k_deep1<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const size_t smem = TileGeoD<STEP, F1>::SMEM;
+    cudaError_t e = cudaFuncSetAttribute(k_deep1<STEP, DEPTH, F1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     if (!grid) {
         int dev = 0, sms = 0, per = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_deep1<STEP, DEPTH>, K2D_THREADS, smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_deep1<STEP, DEPTH, F1>, K2D_THREADS, smem);
         grid = sms * (per > 0 ? per : 1);
     }
-    k_deep1<STEP, DEPTH><<<grid < p.total_tiles ? grid : p.total_tiles, K2D_THREADS, smem, st>>>(p);
+    k_deep1<STEP, DEPTH, F1><<<grid < p.total_tiles ? grid : p.total_tiles, K2D_THREADS, smem, st>>>(p);
     return cudaGetLastError();
 }
 
-template <int STEP, bool DEPTH>
-static cudaError_t launch_ws_t(const CascadeParams& p, cudaStream_t st) {
-    static int grid = 0;
-    const size_t smem = TileGeoW<STEP>::SMEM;
-    cudaError_t e = cudaFuncSetAttribute(k_ws<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    if (!grid) {
-        int dev = 0, sms = 0, per = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_ws<STEP, DEPTH>, WS_THREADS, smem);
-        grid = sms * (per > 0 ? per : 1);
-    }
-    k_ws<STEP, DEPTH><<<grid < p.total_tiles ? grid : p.total_tiles, WS_THREADS, smem, st>>>(p);
-    return cudaGetLastError();
-}
-
-cudaError_t launch_ws(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
+template <bool F1>
+static cudaError_t launch_deep1_f(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
     switch (step) {
-        case 1: return depth ? launch_ws_t<1, true>(p, st) : launch_ws_t<1, false>(p, st);
-        case 2: return depth ? launch_ws_t<2, true>(p, st) : launch_ws_t<2, false>(p, st);
-        case 3: return depth ? launch_ws_t<3, true>(p, st) : launch_ws_t<3, false>(p, st);
-        case 4: return depth ? launch_ws_t<4, true>(p, st) : launch_ws_t<4, false>(p, st);
+        case 1: return depth ? launch_deep1_t<1, true, F1>(p, st) : launch_deep1_t<1, false, F1>(p, st);
+        case 2: return depth ? launch_deep1_t<2, true, F1>(p, st) : launch_deep1_t<2, false, F1>(p, st);
+        case 3: return depth ? launch_deep1_t<3, true, F1>(p, st) : launch_deep1_t<3, false, F1>(p, st);
+        case 4: return depth ? launch_deep1_t<4, true, F1>(p, st) : launch_deep1_t<4, false, F1>(p, st);
         default: return cudaErrorInvalidValue;
     }
 }
 
-cudaError_t launch_deep1(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
+cudaError_t launch_deep1(const CascadeParams& p, bool depth, int step, bool f1, cudaStream_t st) {
+    return f1 ? launch_deep1_f<true>(p, depth, step, st) : launch_deep1_f<false>(p, depth, step, st);
+}
+
+template <int STEP, bool DEPTH>
+static cudaError_t launch_f1_t(const CascadeParams& p, cudaStream_t st) {
+    static int grid = 0;
+    const size_t smem = TileGeoF<STEP>::SMEM;
+    cudaError_t e = cudaFuncSetAttribute(k_f1<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    if (!grid) {
+        int dev = 0, sms = 0, per = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_f1<STEP, DEPTH>, k2_threads(STEP), smem);
+        grid = sms * (per > 0 ? per : 1);
+    }
+    k_f1<STEP, DEPTH><<<grid < p.total_tiles ? grid : p.total_tiles, k2_threads(STEP), smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_f1(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
     switch (step) {
-        case 1: return depth ? launch_deep1_t<1, true>(p, st) : launch_deep1_t<1, false>(p, st);
-        case 2: return depth ? launch_deep1_t<2, true>(p, st) : launch_deep1_t<2, false>(p, st);
-        case 3: return depth ? launch_deep1_t<3, true>(p, st) : launch_deep1_t<3, false>(p, st);
-        case 4: return depth ? launch_deep1_t<4, true>(p, st) : launch_deep1_t<4, false>(p, st);
+        case 1: return depth ? launch_f1_t<1, true>(p, st) : launch_f1_t<1, false>(p, st);
+        case 2: return depth ? launch_f1_t<2, true>(p, st) : launch_f1_t<2, false>(p, st);
+        case 3: return depth ? launch_f1_t<3, true>(p, st) : launch_f1_t<3, false>(p, st);
+        case 4: return depth ? launch_f1_t<4, true>(p, st) : launch_f1_t<4, false>(p, st);
         default: return cudaErrorInvalidValue;
     }
 }

@@ -3,14 +3,16 @@
 // Paper: "the scaling stage generates n resized images by subsampling the decompressed
 // frame ... tex2D linear interpolation"; "integral images are computed ... with a
 // combination of parallel prefix sum [17][18] and matrix transposition operations [19]"
-// (P:L368-384).  B200 design: no level image and no transpose
-// is materialised.  Each level is cut into tiles of 32 rows x 128 ii columns.  A tile CTA
-// resamples its pixels straight from the frame (exact integer bilinear, reading R2), runs
-// warp-shuffle row scans, stages the row prefixes in shared memory and runs a coalesced,
-// vectorised (uint4) column scan.  Every tile is independent: its row carries (pixels left of
-// the tile), column carries (pixels above) and corner (ii at its top-left) come from three
-// light kernels over per-tile marginal sums, so ii/sqii are written to HBM exactly once and all
-// tiles of all levels of all frames of a group run in parallel.
+// (P:L368-384).  B200 design: no transpose is materialised.
+// Each level is cut into tiles of 32 rows x 128 ii columns.  k_marg resamples a tile's pixels
+// from the frame (exact integer bilinear, reading R2), writes them to a level-image scratch
+// buffer (an HBM round trip of ~12 MB per 1080p frame) and its per-tile marginal sums;
+// k_carry / k_corner turn the marginals into row carries, column carries and tile corners;
+// k_tile re-reads the level image, runs warp-shuffle row scans, stages the row prefixes in
+// shared memory and runs a coalesced, vectorised (uint4) column scan, so ii/sqii are written to
+// HBM exactly once and all tiles of all levels of all frames of a group run in parallel.
+// K1 serves fd_integral, the soft-cascade path (k_soft) and the round-1 split K2 schedule; the
+// default detection path (f1) needs only k_level's level images (below).
 #include "fd_internal.h"
 
 namespace fdk {
@@ -467,6 +469,69 @@ __global__ void __launch_bounds__(K1_THREADS) k_tile(const uint8_t* __restrict__
     }
 }
 
+// ---------------------------------------------------------------- f1: level images
+// The group workspace of the f1 path holds only the level images: u8, level-major
+// out + L.u8_off + (g * H_k + y) * PB_k + x, each row zero-padded to PB_k (a 16-B multiple, for
+// the TMA boxes of k_f1).  Pixels are resampled from the frame (R2) and, when the cascade asks for
+// it, filtered (R3b) with exactly the arithmetic k_marg uses for K1.  One CTA per (frame, K1
+// tile of 32 rows x 128 columns); a lane writes 4 pixels as one aligned word.
+__global__ void __launch_bounds__(K1_THREADS) k_level(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
+                                                      uint8_t* __restrict__ out) {
+    __shared__ uint8_t raw[BAND + 2][CHUNK + 4];       // filtering stage: resampled rows with a 1-px halo
+    const int g = blockIdx.y;
+    const int k = find_level_k1(p, blockIdx.x);
+    const LevelDev& L = p.lv[k];
+    const int tl = blockIdx.x - L.k1t0;
+    const int b = tl / L.nchunks, c = tl % L.nchunks;
+    const int y0 = b * BAND, rows = min(BAND, L.H - y0);
+    const int x0 = c * CHUNK;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint8_t* frame = frames + (size_t)g * p.H * p.pitch;
+    const int x = x0 + 4 * lane;
+    ColSample cs[4];
+    if (L.r16 != 65536) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) cs[j] = col_sample(p.W, L.r16, min(x + j, L.W - 1));
+    }
+    uint8_t* o = out + L.u8_off + ((size_t)g * L.H + y0) * L.PB;
+    if (p.filter) {
+        for (int r = warp; r < rows + 2; r += K1_THREADS / 32) {
+            const int yy = min(max(y0 - 1 + r, 0), L.H - 1);
+            for (int q = lane; q < CHUNK + 2; q += 32) {
+                const int xx = min(max(x0 - 1 + q, 0), L.W - 1);
+                raw[r][q] = (uint8_t)level_pixel(frame, p.pitch, p.W, p.H, L.r16, xx, yy);
+            }
+        }
+        __syncthreads();
+    }
+#pragma unroll
+    for (int i = 0; i < BAND / 8; ++i) {
+        const int r = warp + 8 * i;
+        if (r < rows && x < L.PB) {
+            uint32_t pv[4];
+            if (p.filter) {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const int q = x + j - x0 + 1;
+                    uint32_t v = 0;
+                    if (x + j < L.W) {
+#pragma unroll
+                        for (int dy = 0; dy < 3; ++dy) {
+                            const uint32_t h = raw[r + dy][q - 1] + 2u * raw[r + dy][q] + raw[r + dy][q + 1];
+                            v += (dy == 1 ? 2u : 1u) * h;
+                        }
+                        v = (v + 8u) >> 4;
+                    }
+                    pv[j] = v;
+                }
+            } else {
+                tile_row_pixels(frame, p, L, y0 + r, x, cs, pv);
+            }
+            *reinterpret_cast<uint32_t*>(o + (size_t)r * L.PB + x) = pv[0] | (pv[1] << 8) | (pv[2] << 16) | (pv[3] << 24);
+        }
+    }
+}
+
 // ---------------------------------------------------------------- fd_build_pyramid
 __global__ void __launch_bounds__(256) k_pyramid(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
                                                  uint8_t* __restrict__ out, long long frame_stride) {
@@ -513,6 +578,12 @@ cudaError_t launch_k1_tiles_canonical(const uint8_t* img, const PlanDev& plan, i
     dim3 grid(plan.k1tiles_per_frame, n);
     k_tile<true><<<grid, K1_THREADS, 0, st>>>(img, plan, s, nullptr, ii, reinterpret_cast<unsigned long long*>(sqii),
                                               out_pitch);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_levels(const uint8_t* frames, const PlanDev& plan, int g_frames, uint8_t* out, cudaStream_t st) {
+    dim3 grid(plan.k1tiles_per_frame, g_frames);
+    k_level<<<grid, K1_THREADS, 0, st>>>(frames, plan, out);
     return cudaGetLastError();
 }
 

@@ -7,8 +7,9 @@
 // deepest window, a serial chain of up to ~1400 stumps.  k_cascade instead appends those
 // windows to a global queue and moves on to its next tile; this kernel finishes them, one warp
 // per window, with no block-level synchronisation at all:
-//   * the window's 25 x 25 ii region (plane 0 of the group workspace, still resident) is staged
-//     in the warp's shared memory once (25 coalesced row loads);
+//   * the window's 25 x 25 ii region is staged in the warp's shared memory once: 25 coalesced
+//     row loads of plane 0 of the group workspace, or -- on the f1 path, where no global integral
+//     exists -- a window-local integral built from the window's 24 x 24 level pixels;
 //   * lane j evaluates stump c0 + j of the current stage from SoA tail records (word w of
 //     stump j at trec[w * ns + j]: coalesced 128-B loads) whose corner offsets address the
 //     staged region directly;
@@ -28,29 +29,70 @@ struct IntC {
 };
 constexpr int TAIL_REGION = ((WIN + 1) * TAIL_RP + 31) & ~31;   // words per warp
 
+// Dynamic shared memory: the SoA records of stumps [j0, j0 + nsm) (the early deep stages, where
+// most tail windows are; word w of stump j at srec[w * nsm + j - j0]), then one 25 x 25 region per
+// warp.  Stages outside that range read the records from global memory.
+size_t tail_smem(int nsm) { return ((size_t)TAIL_REC_WORDS * nsm + (size_t)(TAIL_THREADS / 32) * TAIL_REGION) * 4; }
+
 template <bool DEPTH>
-__global__ void __launch_bounds__(TAIL_THREADS) k_tail(const __grid_constant__ TailParams p) {
-    __shared__ uint32_t region[TAIL_THREADS / 32][TAIL_REGION];
+__global__ void __launch_bounds__(TAIL_THREADS, 4) k_tail(const __grid_constant__ TailParams p) {
+    extern __shared__ uint32_t tsm[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    uint32_t* R = region[warp];
+    uint32_t* srec = tsm;
+    uint32_t* R = tsm + TAIL_REC_WORDS * p.nsm + warp * TAIL_REGION;
+    for (int i = threadIdx.x; i < TAIL_REC_WORDS * p.nsm; i += TAIL_THREADS) {
+        const int w = i / p.nsm, j = i - w * p.nsm;
+        srec[i] = __ldg(p.trec + (size_t)w * p.ns + p.j0 + j);
+    }
+    __syncthreads();
     const unsigned cnt = *p.count;
     const int n = (int)(cnt < (unsigned)p.cap ? cnt : (unsigned)p.cap);
     const int N = p.n_stages;
     for (int e = blockIdx.x * (TAIL_THREADS / 32) + warp; e < n; e += gridDim.x * (TAIL_THREADS / 32)) {
         const uint4 q = __ldg(p.q + e);
-        const int g = (int)(q.x >> 16), k = (int)((q.x >> 8) & 255), s = (int)(q.x & 255);
+        const int g = (int)q.w, k = (int)((q.x >> 8) & 255), s = (int)(q.x & 255);
         const int wyi = (int)(q.y >> 16), wxi = (int)(q.y & 0xffffu);
         const float nf = __int_as_float((int)q.z);
         const LevelDev L = p.lv[k];
-        const uint32_t* src = p.ws + L.ws_off + (long long)g * 2 * (L.H + 1) * L.P + (long long)(wyi * p.step) * L.P +
-                              wxi * p.step;
         __syncwarp();                         // previous window's region reads done
-        if (lane <= WIN) {           // 25 independent row loads in flight, then 25 stores
-            uint32_t v[WIN + 1];
+        if (p.lvl8) {
+            // f1: no global integral exists; the window's 25 x 25 ii is built from its 24 x 24
+            // level pixels (a window-local integral: rectangle sums are origin-independent, R4).
+            // Lane r < 24 scans pixel row r into R[r + 1][1..24]; then lane c adds down column c.
+            const uint8_t* src = p.lvl8 + L.u8_off + ((long long)g * L.H + (long long)wyi * p.step) * L.PB +
+                                 (long long)wxi * p.step;
+            if (lane < WIN) {
+                uint8_t px[WIN];
 #pragma unroll
-            for (int r = 0; r <= WIN; ++r) v[r] = __ldg(src + (long long)r * L.P + lane);
+                for (int c = 0; c < WIN; ++c) px[c] = __ldg(src + (long long)lane * L.PB + c);
+                uint32_t acc = 0;
+                R[(lane + 1) * TAIL_RP] = 0u;
 #pragma unroll
-            for (int r = 0; r <= WIN; ++r) R[r * TAIL_RP + lane] = v[r];
+                for (int c = 0; c < WIN; ++c) {
+                    acc += px[c];
+                    R[(lane + 1) * TAIL_RP + c + 1] = acc;
+                }
+            }
+            if (lane <= WIN) R[lane] = 0u;
+            __syncwarp();
+            if (lane < WIN) {
+                uint32_t acc = 0;
+#pragma unroll
+                for (int r = 1; r <= WIN; ++r) {
+                    acc += R[r * TAIL_RP + lane + 1];
+                    R[r * TAIL_RP + lane + 1] = acc;
+                }
+            }
+        } else {
+            const uint32_t* src = p.ws + L.ws_off + (long long)g * 2 * (L.H + 1) * L.P +
+                                  (long long)(wyi * p.step) * L.P + wxi * p.step;
+            if (lane <= WIN) {       // 25 independent row loads in flight, then 25 stores
+                uint32_t v[WIN + 1];
+#pragma unroll
+                for (int r = 0; r <= WIN; ++r) v[r] = __ldg(src + (long long)r * L.P + lane);
+#pragma unroll
+                for (int r = 0; r <= WIN; ++r) R[r * TAIL_RP + lane] = v[r];
+            }
         }
         __syncwarp();
         // leaf of stump c0 + lane of stage sd (0 beyond the stage); MC >= the stage's largest
@@ -59,16 +101,17 @@ __global__ void __launch_bounds__(TAIL_THREADS) k_tail(const __grid_constant__ T
         auto leaf_mc = [&](const StageDev& sd, int c0, auto mc_tag) -> float {
             constexpr int MC = decltype(mc_tag)::value;
             if (c0 + lane >= sd.n) return 0.0f;
-            const uint32_t* t = p.trec + sd.first + c0 + lane;
+            const bool shared = sd.first >= p.j0 && sd.first + sd.n <= p.j0 + p.nsm;   // stage-uniform
+            const uint32_t* t = shared ? srec + (sd.first - p.j0 + c0 + lane) : p.trec + sd.first + c0 + lane;
+            const size_t ws = shared ? (size_t)p.nsm : (size_t)p.ns;
             uint32_t f = 0;
 #pragma unroll
             for (int c = 0; c < MC; ++c) {
-                const uint32_t w = __ldg(t + (size_t)(4 + c) * p.ns);
+                const uint32_t w = t[(4 + c) * ws];
                 f += (uint32_t)((int)w >> 16) * R[w & 0xffffu];
             }
-            const float tt = __fmul_rn(__int_as_float((int)__ldg(t + (size_t)p.ns)), nf);
-            return (__int2float_rn((int)f) < tt) ? __int_as_float((int)__ldg(t + (size_t)2 * p.ns))
-                                                 : __int_as_float((int)__ldg(t + (size_t)3 * p.ns));
+            const float tt = __fmul_rn(__int_as_float((int)t[ws]), nf);
+            return (__int2float_rn((int)f) < tt) ? __int_as_float((int)t[2 * ws]) : __int_as_float((int)t[3 * ws]);
         };
         auto leaf_of = [&](const StageDev& sd, int c0) -> float {
             if (sd.mc <= 6) return leaf_mc(sd, c0, IntC<6>{});
@@ -134,17 +177,19 @@ __global__ void __launch_bounds__(TAIL_THREADS) k_tail(const __grid_constant__ T
 }
 
 cudaError_t launch_tail(const TailParams& p, bool depth, cudaStream_t st) {
-    static int grid = [] {
-        int dev = 0, sms = 148, per = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_tail<false>, TAIL_THREADS, 0);
-        return sms * (per > 0 ? per : 1);
-    }();
+    const size_t smem = tail_smem(p.nsm);
+    cudaError_t e = cudaFuncSetAttribute(depth ? k_tail<true> : k_tail<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)smem);
+    if (e != cudaSuccess) return e;
+    int dev = 0, sms = 148, per = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, depth ? k_tail<true> : k_tail<false>, TAIL_THREADS, smem);
+    const int grid = sms * (per > 0 ? per : 1);
     if (depth)
-        k_tail<true><<<grid, TAIL_THREADS, 0, st>>>(p);
+        k_tail<true><<<grid, TAIL_THREADS, smem, st>>>(p);
     else
-        k_tail<false><<<grid, TAIL_THREADS, 0, st>>>(p);
+        k_tail<false><<<grid, TAIL_THREADS, smem, st>>>(p);
     return cudaGetLastError();
 }
 

@@ -25,7 +25,7 @@ def test_library_exports_every_declared_symbol():
     assert len(syms) >= 12
     for s in syms:
         assert hasattr(L, s), s
-    assert L.fd_abi_version() == 2
+    assert L.fd_abi_version() == 3
 
 
 def test_detection_struct_layout_matches_oracle():

@@ -128,14 +128,23 @@ def test_depth_maps_generic_k2(monkeypatch):
 
 # K2 schedules (fd_api.cpp run_groups): every one computes the same depth maps and detections
 K2_SCHEDULES = {
-    "stage1_only": {"FD_S0": "1"},                          # k_stage1 stage 1, k_deep1 from stage 2
-    "no_tail": {"FD_TAIL": "0"},                            # k_deep1 finishes every window
-    "warp_specialised": {"FD_K2_WS": "1"},                  # k_ws
-    "warp_specialised_s0_1": {"FD_K2_WS": "1", "FD_WS_S0": "1"},
-    "fused": {"FD_K2_SPLIT": "0"},                          # k_cascade
-    "batched_deep": {"FD_K2_DEEP1": "0"},                   # k_stage1 + batched k_deep
-    "one_slot_pipeline": {"FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
-    "two_slot_pipeline": {"FD_GROUP_FRAMES": "1"},          # 3 frame groups over 2 slots/streams
+    "split_default": {},                                    # K1 -> k_stage1 -> k_deep1 -> k_tail
+    "split_s0_1": {"FD_S0": "1"},                           # k_stage1 stage 1 only
+    "split_no_tail": {"FD_TAIL": "0"},                      # k_deep1 finishes every window
+    "split_no_split_stump": {"FD_DEEP_SPLIT": "0"},         # deep stages without the split-stump mode
+    "split_s_tail_3": {"FD_S_TAIL": "3"},                   # every window alive at stage 3 through k_tail
+    "split_two_slot": {"FD_GROUP_FRAMES": "1"},             # 3 frame groups over 2 slots/streams
+    "split_one_slot": {"FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
+    "fused_k1": {"FD_K2_SPLIT": "0"},                       # K1 -> k_cascade -> k_tail
+    "f1": {"FD_F1": "1"},                                   # k_level -> k_f1 -> k_deep1<F1> -> k_tail
+    "f1_no_tail": {"FD_F1": "1", "FD_TAIL": "0"},
+    "f1_tail_early": {"FD_F1": "1", "FD_TAIL_N": "200"},    # most deep windows through k_tail (u8 rebuild)
+    "f1_small_groups": {"FD_F1": "1", "FD_GROUP_FRAMES": "1"},
+    "f1_one_slot": {"FD_F1": "1", "FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
+    "f1_fused": {"FD_F1": "1", "FD_F1_SPLIT": "0"},         # k_f1 runs every stage
+    "f1_fused_no_split_stump": {"FD_F1": "1", "FD_F1_SPLIT": "0", "FD_DEEP_SPLIT": "0"},
+    "f1_fused_s_tail_1": {"FD_F1": "1", "FD_F1_SPLIT": "0", "FD_S_TAIL": "1"},   # all stage-1 survivors to k_tail
+    "f1_tail_global_records": {"FD_F1": "1", "FD_TAIL_SMEM_STUMPS": "0", "FD_S_TAIL": "3"},
     "queue": {"FD_K2_QUEUE": "1"},                          # k_soft's schedule on a hard cascade
 }
 

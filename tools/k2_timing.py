@@ -30,7 +30,7 @@ print({k: round(v[1], 3) for k, v in fd.fd_profile_read().items() if v[0]})
 L.fd_debug_k2_timing(buf, 0)
 b = list(buf)
 if b[0]:
-    print(f"tiles {b[0]}  per tile cycles: tma-wait {b[1]/b[0]:.0f}  stage1 {b[2]/b[0]:.0f}")
+    print(f"tiles {b[0]}  per tile cycles: tma-wait {b[1]/b[0]:.0f}  build {b[85]/b[0]:.0f}  stage1 {b[2]/b[0]:.0f}")
 nbat = max(b[84], 1)
 print(f"group-mode decisions {b[95]}  undecided {b[94]}  exact recomputes {b[96]}")
 print(f"deep batches {b[84]}  tiles/batch {b[92]/nbat:.2f}  pool/batch {b[93]/nbat:.1f}")
