@@ -111,7 +111,7 @@ void make_plan_dev(const fd_plan& pl, int W, int H, int pitch, int step, int G, 
         L.cor_off = cor;
         L.lvl_off = lvl;
         L.win0 = win;
-        lvl += (long long)L.H * L.P;
+        lvl += (long long)L.H * L.PB;
         bands += L.nbands;
         k1t += L.nbands * L.nchunks;
         tiles += L.tiles_x * ((L.ny + ty - 1) / ty);
@@ -643,6 +643,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     PlanDev& PD = *w->plan;
     make_plan_dev(pl, W, H, pitch, step, G, &PD);
     PD.filter = c->filter;
+    PD.aligned4 = ((reinterpret_cast<uintptr_t>(d_frames) | (uintptr_t)pitch) & 3) == 0;
     // two pipeline slots on two streams when there is more than one group (FD_PIPE=0: one)
     const int nslots = (ngroups > 1 && env_int("FD_PIPE", 1) != 0) ? 2 : 1;
     K1Scratch k1s[2];
@@ -710,8 +711,8 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     // FD_S_TAIL: every window still alive at this stage is handed to k_tail (default: none, only
     // the FD_TAIL_N rule)
     P.s_tail = std::max(1, env_int("FD_S_TAIL", 255));
-    // deep stages with at most FD_DEEP_SPLIT windows (<= 64; 0 = off) run split-stump (k_f1)
-    P.split_max = std::max(0, env_int("FD_DEEP_SPLIT", 64));
+    // deep stages with at most FD_DEEP_SPLIT windows (<= 64; default 0 = off) run split-stump
+    P.split_max = std::max(0, env_int("FD_DEEP_SPLIT", 0));
     // k_stage1 runs stages [0, s0) (FD_S0 = 2, default, or 1); the fused kernels start their
     // deep phase at stage 1
     P.s0 = split ? (env_int("FD_S0", 2) >= 2 ? 2 : 1) : (f1_split ? 2 : 1);
@@ -973,6 +974,7 @@ fd_status fd_integral(const uint8_t* d_img, int n, int W, int H, int pitch, uint
     pl.h[0] = H;
     PlanDev p;
     make_plan_dev(pl, W, H, pitch, 1, 1, &p);
+    p.aligned4 = ((reinterpret_cast<uintptr_t>(d_img) | (uintptr_t)pitch) & 3) == 0;
     Workspace* w = nullptr;
     r = get_ws(st, &w);
     if (r != FD_OK) return r;

@@ -124,7 +124,11 @@ struct TileGeoF {
 #ifndef FD_K2D_CTAS
 #define FD_K2D_CTAS 8
 #endif
-constexpr int K2D_THREADS = 128;
+#ifndef FD_K2D_THREADS
+#define FD_K2D_THREADS 128                  // k_deep1 block size (the NVRTC program may override it)
+#endif
+constexpr int K2D_THREADS = FD_K2D_THREADS;
+constexpr int K2D_RED_MAX = 128;            // split-stump partial-sum space, for any k_deep1 block size
 template <int STEP, bool F1 = false>
 struct TileGeoD {
     static constexpr int PBUF = k2_pbuf(STEP);
@@ -133,7 +137,7 @@ struct TileGeoD {
     static constexpr size_t OFF_LOC = OFF_NF + (size_t)CP * 4;
     static constexpr size_t OFF_LIST = OFF_LOC + (size_t)CP * 2;
     static constexpr size_t OFF_RED = OFF_LIST + (size_t)2 * CP * 2;     // split-stump partial sums
-    static constexpr size_t OFF_U8 = (OFF_RED + (size_t)K2D_THREADS * 8 + 127) & ~(size_t)127;   // f1 pixels
+    static constexpr size_t OFF_U8 = (OFF_RED + (size_t)K2D_RED_MAX * 8 + 127) & ~(size_t)127;   // f1 pixels
     static constexpr size_t SMEM = F1 ? OFF_U8 + (size_t)TileGeoF<STEP>::UB : OFF_U8;
 };
 
@@ -151,7 +155,7 @@ struct LevelDev {
     long long col_off;      // u32 elements (per frame): column sums/carries [band][2][W]
     long long row_off;      // u32 elements (per frame): row sums/carries [band][chunk][2][BAND]
     long long cor_off;      // u64 elements (per frame): tile corners [band][chunk][2]
-    long long lvl_off;      // bytes (per frame): level image [H][P] written by K1a, read by K1b
+    long long lvl_off;      // bytes (per frame): level image [H][PB] written by K1a, read by K1b
     long long win0;         // first window index of the level within a frame
 };
 
@@ -171,6 +175,7 @@ struct PlanDev {
     long long u8_bytes;     // f1 group workspace bytes (level images of G frames)
     int G;                  // frames per group (tensor-map extent)
     int filter;             // K1: 1 = binomial 3x3 filtering stage after scaling (f2)
+    int aligned4;           // frames pointer and pitch are 4-byte aligned (word loads of identity levels)
     LevelDev lv[FD_MAX_LEVELS];
 };
 

@@ -170,6 +170,11 @@ static int env_or(const char* name, int dflt) {
     return e && *e ? std::atoi(e) : dflt;
 }
 
+// k_deep1 block size of the generated program (FD_K2D_THREADS: 64 or 128)
+static int jit_deep_threads() {
+    return env_or("FD_K2D_THREADS", FD_K2D_THREADS) <= 64 ? 64 : 128;
+}
+
 // resident CTAs per SM targeted by the fused kernel's launch bounds (FD_K2_CTAS, 2..6)
 static int jit_ctas() {
     const int c = env_or("FD_K2_CTAS", FD_K2_CTAS);
@@ -179,6 +184,7 @@ static int jit_ctas() {
 std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages) {
     const int k_end = jit_deep_end(st, n_stages);
     std::string src = "#define FD_K2D_CTAS " + std::to_string(env_or("FD_K2D_CTAS", FD_K2D_CTAS)) +
+                      "\n#define FD_K2D_THREADS " + std::to_string(jit_deep_threads()) +
                       "\n#define FD_F1_CTAS " + std::to_string(env_or("FD_F1_CTAS", FD_F1_CTAS)) +
                       "\n#define FD_K2_CTAS " + std::to_string(jit_ctas()) +
                       "\n#include \"fd_internal.h\"\n" + jit_stage1_source(rec_words, st[0].first, st[0].n) +
@@ -198,7 +204,7 @@ static std::string jit_name(int kind, bool depth) {
 
 static KindGeo jit_kind_geo(int kind) {
     KindGeo g;
-    g.threads = (kind == JIT_DEEP1 || kind == JIT_DEEP1_F1) ? K2D_THREADS : k2_threads(JIT_STEP);
+    g.threads = (kind == JIT_DEEP1 || kind == JIT_DEEP1_F1) ? jit_deep_threads() : k2_threads(JIT_STEP);
     if (kind == JIT_FUSED) g.smem = TileGeo<JIT_STEP>::SMEM;
     if (kind == JIT_STAGE1) g.smem = TileGeoA<JIT_STEP>::SMEM;
     if (kind == JIT_DEEP1) g.smem = TileGeoD<JIT_STEP, false>::SMEM;

@@ -584,7 +584,7 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
     uint16_t* sidx = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_SIDX);    //       and window index
     __shared__ __align__(8) uint64_t mbar[2];
     __shared__ int s_tile[2], s_frame[2], s_lvl[2], s_wx0[2], s_wy0[2];
-    __shared__ int s_c1, s_c2, s_off, s_prev, s_prev_off;
+    __shared__ int s_c1[2], s_c2[2], s_off, s_prev, s_prev_off;   // survivor counters per parity of the tile
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const StageDev& st0 = p.pstages[0];
     const ParamRec prec{p};
@@ -606,48 +606,62 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
             tma_load_4d(Q, p.tmaps + t.k, t.x, t.y, 1, t.g, &mbar[b]);
         }
     };
+    // this thread's windows (the same for every tile): WPT windows of column lx from row ly0
+    const int lx = lane + 32 * (warp % WARPS_X);
+    const int ly0 = (warp / WARPS_X) * WPT;
+    const int base = ly0 * STEP * TW + lx * STEP;
+    // variance normalisation (oracle c5) of this thread's windows of the tile in ii buffer bb + Q
+    auto variance = [&](int bb, float* nfo) {
+        const uint32_t* Tb = reinterpret_cast<const uint32_t*>(smem_raw) + bb * G::PBUF;
+#pragma unroll
+        for (int i = 0; i < WPT; ++i) {
+            const int bo = base + i * STEP * TW;
+            const uint32_t S = Tb[bo + WIN * TW + WIN] - Tb[bo + WIN] - Tb[bo + WIN * TW] + Tb[bo];
+            const uint32_t q = Q[bo + WIN * TW + WIN] - Q[bo + WIN] - Q[bo + WIN * TW] + Q[bo];
+            const long long v = 576LL * (long long)q - (long long)S * (long long)S;
+            nfo[i] = v > 0 ? __fsqrt_rn(__ll2float_rn(v)) : 1.0f;
+        }
+    };
     if (tid == 0) {
         mbar_init(&mbar[0], 1);
         mbar_init(&mbar[1], 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         s_prev = -1;
+        s_c1[0] = s_c1[1] = s_c2[0] = s_c2[1] = 0;
         claim(0);
     }
+    __syncthreads();
     uint32_t phases = 0;
+    float nf[WPT];
+    if (s_tile[0] < p.total_tiles) {              // the first tile's variance; later tiles' in the loop
+        mbar_wait(&mbar[0], 0u);
+        phases ^= 1u;
+        variance(0, nf);
+    }
     for (int it = 0;; ++it) {
         const int b = it & 1;
-        __syncthreads();                          // (A) previous tile done: list, counters, its ii buffer free
+        __syncthreads();                          // (A) previous tile done: list, counters, its ii buffer and
+                                                  //     (this tile's variance taken) the sqii buffer free
         const int tn = s_tile[b];
         if (tid == 0) {
-            if (s_prev >= 0) p.tile_rec[s_prev] = make_uint2((unsigned)s_prev_off, (unsigned)s_c2);
+            // the previous tile's record; its counters are reset for the tile after this one (a
+            // barrier separates that reset from their next use)
+            if (s_prev >= 0) p.tile_rec[s_prev] = make_uint2((unsigned)s_prev_off, (unsigned)s_c2[b ^ 1]);
             s_prev = -1;
-            s_c1 = 0;
-            s_c2 = 0;
+            s_c1[b ^ 1] = 0;
+            s_c2[b ^ 1] = 0;
         }
         if (tn >= p.total_tiles) break;
+        if (tid == 0) claim(b ^ 1);               // prefetch: next ii -> the other buffer, next sqii -> Q
         const WinOut<STEP, DEPTH> out{p, s_frame + b, s_lvl + b, s_wx0 + b, s_wy0 + b};
         const uint32_t* T = reinterpret_cast<const uint32_t*>(smem_raw) + b * G::PBUF;
-        mbar_wait(&mbar[b], (phases >> b) & 1u);
-        phases ^= 1u << b;
         const int k = s_lvl[b];
         const int nx = __ldg(&p.lv[k].nx), ny = __ldg(&p.lv[k].ny);
         const int wx0 = s_wx0[b], wy0 = s_wy0[b];
-        const int lx = lane + 32 * (warp % WARPS_X);
-        const int ly0 = (warp / WARPS_X) * WPT;
-        const int base = ly0 * STEP * TW + lx * STEP;
         const bool colok = wx0 + lx < nx;
-        float nf[WPT], sm[WPT];
+        float sm[WPT];
 #pragma unroll
-        for (int i = 0; i < WPT; ++i) {
-            const int bo = base + i * STEP * TW;
-            const uint32_t S = T[bo + WIN * TW + WIN] - T[bo + WIN] - T[bo + WIN * TW] + T[bo];
-            const uint32_t q = Q[bo + WIN * TW + WIN] - Q[bo + WIN] - Q[bo + WIN * TW] + Q[bo];
-            const long long v = 576LL * (long long)q - (long long)S * (long long)S;
-            nf[i] = v > 0 ? __fsqrt_rn(__ll2float_rn(v)) : 1.0f;
-            sm[i] = 0.0f;
-        }
-        __syncthreads();                          // (B) every sqii read done: prefetch the next tile
-        if (tid == 0) claim(b ^ 1);
+        for (int i = 0; i < WPT; ++i) sm[i] = 0.0f;
 #ifdef FD_JIT_STAGE1
         jit_stage1(T + base, nf, sm);
 #else
@@ -670,7 +684,7 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
             const unsigned m = __ballot_sync(0xffffffffu, pass);
             if (m) {
                 int pos = 0;
-                if (lane == 0) pos = atomicAdd(&s_c1, __popc(m));
+                if (lane == 0) pos = atomicAdd(&s_c1[b], __popc(m));
                 pos = __shfl_sync(0xffffffffu, pos, 0);
                 if (pass) {
                     const int at = pos + __popc(m & ((1u << lane) - 1u));
@@ -680,7 +694,7 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
             }
         }
         __syncthreads();                          // (C) stage-1 survivor list complete
-        const int c = s_c1;
+        const int c = s_c1[b];
         if (tid == 0) {
             // reserve c global entries for this tile's survivors (an upper bound after stage 2)
             s_off = c ? (int)atomicAdd(p.surv_count, (unsigned)c) : 0;
@@ -693,7 +707,7 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
         const int off = s_off;
         if (p.s0 < 2 || p.n_stages < 2) {
             for (int e = tid; e < c; e += THREADS) p.surv[off + e] = make_uint2(sidx[e], (unsigned)__float_as_int(snf[e]));
-            if (tid == 0) s_c2 = c;
+            if (tid == 0) s_c2[b] = c;
         } else {
             // stage 2 over the list, one lane per window; survivors straight to the global list
             const StageDev& sd = p.pstages[1];
@@ -723,13 +737,20 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
                 const unsigned m = __ballot_sync(0xffffffffu, pass);
                 if (m) {
                     int pos = 0;
-                    if (lane == 0) pos = atomicAdd(&s_c2, __popc(m));
+                    if (lane == 0) pos = atomicAdd(&s_c2[b], __popc(m));
                     pos = __shfl_sync(0xffffffffu, pos, 0);
                     if (pass)
                         p.surv[off + pos + __popc(m & ((1u << lane) - 1u))] =
                             make_uint2((unsigned)idx, (unsigned)__float_as_int(nfw));
                 }
             }
+        }
+        // the next tile's variance: its ii and sqii planes arrive during this tile's stages, and
+        // every thread takes its own windows' nf here -- the warps without stage-2 work first
+        if (s_tile[b ^ 1] < p.total_tiles) {
+            mbar_wait(&mbar[b ^ 1], (phases >> (b ^ 1)) & 1u);
+            phases ^= 1u << (b ^ 1);
+            variance(b ^ 1, nf);
         }
         if (tid == 0) {
             s_prev = tn;                          // tile_rec written after the next barrier (A)

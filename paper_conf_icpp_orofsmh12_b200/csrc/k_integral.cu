@@ -68,17 +68,29 @@ __device__ __forceinline__ uint32_t level_pixel(const uint8_t* frame, int pitch,
     return bilinear(r, col_sample(srcW, r16, x));
 }
 
-// The 4 pixels of row y at columns x0+4*lane .. +3 of a tile (0 beyond the level width).
+// The 4 level pixels of row y at columns x .. x+3 (0 at or beyond the level width).  Identity
+// level: one aligned 4-byte load when the frame allows it.  Bilinear levels: branch-free -- the
+// column taps cs[] are clamped into the frame (col_sample of min(x + j, W_k - 1)), every tap is
+// loaded and the pixels past the level width are masked afterwards.
 __device__ __forceinline__ void tile_row_pixels(const uint8_t* frame, const PlanDev& p, const LevelDev& L, int y, int x,
                                                 const ColSample* cs, uint32_t* pv) {
     if (L.r16 == 65536) {
         const uint8_t* row = frame + (size_t)y * p.pitch;
+        if (p.aligned4 && x + 4 <= p.pitch) {
+            const uint32_t w = __ldg(reinterpret_cast<const uint32_t*>(row + x));
 #pragma unroll
-        for (int j = 0; j < 4; ++j) pv[j] = x + j < L.W ? __ldg(row + x + j) : 0u;
-    } else {
-        const RowSample rs = row_sample(frame, p.pitch, p.H, L.r16, y);
+            for (int j = 0; j < 4; ++j) pv[j] = x + j < L.W ? (w >> (8 * j)) & 255u : 0u;
+        } else {
 #pragma unroll
-        for (int j = 0; j < 4; ++j) pv[j] = x + j < L.W ? bilinear(rs, cs[j]) : 0u;
+            for (int j = 0; j < 4; ++j) pv[j] = x + j < L.W ? (uint32_t)__ldg(row + x + j) : 0u;
+        }
+        return;
+    }
+    const RowSample rs = row_sample(frame, p.pitch, p.H, L.r16, y);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        const uint32_t v = bilinear(rs, cs[j]);
+        pv[j] = x + j < L.W ? v : 0u;
     }
 }
 
@@ -148,22 +160,20 @@ __global__ void __launch_bounds__(K1_THREADS) k_marg(const uint8_t* __restrict__
             } else {
                 tile_row_pixels(frame, p, L, y0 + r, x, cs, pv);
             }
-            if (x < L.P)       // level image row, 4 pixels per lane as one aligned word (0 past W)
-                *reinterpret_cast<uint32_t*>(lvl + (size_t)(y0 + r) * L.P + x) =
+            if (x < L.PB)      // level image row (pitch PB), 4 pixels per lane as one aligned word (0 past W)
+                *reinterpret_cast<uint32_t*>(lvl + (size_t)(y0 + r) * L.PB + x) =
                     pv[0] | (pv[1] << 8) | (pv[2] << 16) | (pv[3] << 24);
             uint32_t rs = 0, rq = 0;
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
+                const uint32_t q = pv[j] * pv[j];
                 rs += pv[j];
-                rq += pv[j] * pv[j];
+                rq += q;
                 cols[j] += pv[j];
-                colq[j] += pv[j] * pv[j];
+                colq[j] += q;
             }
-#pragma unroll
-            for (int o = 16; o > 0; o >>= 1) {
-                rs += __shfl_xor_sync(0xffffffffu, rs, o);
-                rq += __shfl_xor_sync(0xffffffffu, rq, o);
-            }
+            rs = __reduce_add_sync(0xffffffffu, rs);      // row sums of the tile (< 2^32: 128 * 255^2)
+            rq = __reduce_add_sync(0xffffffffu, rq);
             if (lane == 0) {
                 rowsum[r] = rs;
                 rowsum[BAND + r] = rq;
@@ -288,19 +298,24 @@ struct BandOut<true> {
     using QT = unsigned long long;
 };
 
+// Row phase: thread (r, sg) owns row r of the band and the 16 columns x0 + 16 sg .. of the chunk
+// (one 16-B load of the level image, pitch PB): exclusive prefixes of p and p^2 in registers, the
+// 8 segments of a row exchange exclusive offsets with 3 shuffles, plus the row carry (pixels left
+// of the chunk).  Column phase: thread per (column, plane) walks down the band adding the row
+// prefixes to the tile's top row ii[y0][X] and stores each ii / sqii entry once (a warp stores
+// 32 consecutive entries of a row: 128 or 256 B).
 template <bool CANON>
 __global__ void __launch_bounds__(K1_THREADS) k_tile(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
                                                      K1Scratch s, uint32_t* __restrict__ ws,
                                                      uint32_t* __restrict__ out_ii,
                                                      unsigned long long* __restrict__ out_sq, int out_pitch) {
     using QT = typename BandOut<CANON>::QT;
+    static_assert(K1_THREADS == 8 * BAND && CHUNK == 8 * 16, "row phase: 8 segments of 16 columns per row");
     __shared__ __align__(16) uint32_t rp_s[BAND][CHUNK];
-    __shared__ __align__(16) uint32_t rp_q[BAND][CHUNK];
-    __shared__ __align__(16) uint32_t seg_s[8][CHUNK];
-    __shared__ __align__(16) QT seg_q[8][CHUNK];
+    __shared__ __align__(16) uint32_t rp_q[BAND][CHUNK];   // row prefixes of p^2: < W * 255^2 < 2^32, exact
     __shared__ __align__(16) uint32_t top_s[CHUNK];
     __shared__ __align__(16) QT top_q[CHUNK];
-
+    (void)frames;
     const int g = blockIdx.y;
     const int k = find_level_k1(p, blockIdx.x);
     const LevelDev& L = p.lv[k];
@@ -308,61 +323,51 @@ __global__ void __launch_bounds__(K1_THREADS) k_tile(const uint8_t* __restrict__
     const int b = tl / L.nchunks, c = tl % L.nchunks;
     const int y0 = b * BAND, rows = min(BAND, L.H - y0);
     const int x0 = c * CHUNK;
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const uint8_t* frame = frames + (size_t)g * p.H * p.pitch;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const uint32_t* carry = s.col + (size_t)g * p.col_frame + L.col_off + (size_t)b * 2 * L.W;
     const uint32_t* rowc = s.row + (size_t)g * p.row_frame + L.row_off + (size_t)(b * L.nchunks + c) * 2 * BAND;
     const unsigned long long* cor = s.cor + (size_t)g * p.cor_frame + L.cor_off + (size_t)(b * L.nchunks + c) * 2;
-
-    const int P = CANON ? out_pitch : L.P;
-    uint32_t* o_ii;
-    QT* o_sq;
-    if constexpr (CANON) {
-        o_ii = out_ii + (size_t)g * (L.H + 1) * out_pitch;
-        o_sq = reinterpret_cast<QT*>(out_sq + (size_t)g * (L.H + 1) * out_pitch);
-    } else {
-        const size_t plane = (size_t)(L.H + 1) * L.P;
-        o_ii = ws + L.ws_off + (size_t)g * 2 * plane;
-        o_sq = reinterpret_cast<QT*>(o_ii + plane);
-    }
-
-    // ---- row phase: warp-shuffle exclusive scans of 4 rows per warp, plus the row carries;
-    // pixels come from the level image K1a wrote (one aligned 4-pixel word per lane)
-    const int x = x0 + 4 * lane;
     const uint8_t* lvl = s.lvl + (size_t)g * p.lvl_frame + L.lvl_off;
-    (void)frame;
+
+    // ---- row phase
+    {
+        const int r = tid >> 3, sg = tid & 7;
+        const int xs = x0 + 16 * sg;
+        uint4 w = make_uint4(0u, 0u, 0u, 0u);
+        if (r < rows && xs < L.PB) w = __ldg(reinterpret_cast<const uint4*>(lvl + (size_t)(y0 + r) * L.PB + xs));
+        const uint32_t wd[4] = {w.x, w.y, w.z, w.w};
+        uint32_t ps[16], pq[16];
+        uint32_t ts = 0, tq = 0;
 #pragma unroll
-    for (int i = 0; i < BAND / 8; ++i) {
-        const int r = warp + 8 * i;
-        if (r < rows) {
-            uint32_t pv[4];
-            const uint32_t wv = x < L.P ? __ldg(reinterpret_cast<const uint32_t*>(lvl + (size_t)(y0 + r) * L.P + x)) : 0u;
+        for (int i = 0; i < 16; ++i) {      // exclusive: ii column X sums the pixels x < X
+            const uint32_t v = (wd[i >> 2] >> (8 * (i & 3))) & 255u;
+            ps[i] = ts;
+            pq[i] = tq;
+            ts += v;
+            tq += v * v;
+        }
+        uint32_t is = ts, iq = tq;
 #pragma unroll
-            for (int j = 0; j < 4; ++j) pv[j] = (wv >> (8 * j)) & 255u;
-            uint32_t es[4], eq[4], ts = 0, tq = 0;
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                es[j] = ts;
-                eq[j] = tq;
-                ts += pv[j];
-                tq += pv[j] * pv[j];
+        for (int d = 1; d < 8; d <<= 1) {
+            const uint32_t a = __shfl_up_sync(0xffffffffu, is, d, 8);
+            const uint32_t q = __shfl_up_sync(0xffffffffu, iq, d, 8);
+            if (sg >= d) {
+                is += a;
+                iq += q;
             }
-            uint32_t is = ts, iq = tq;    // warp inclusive scan of lane totals
+        }
+        const uint32_t bs = (r < rows ? rowc[r] : 0u) + is - ts;
+        const uint32_t bq = (r < rows ? rowc[BAND + r] : 0u) + iq - tq;
 #pragma unroll
-            for (int d = 1; d < 32; d <<= 1) {
-                const uint32_t a = __shfl_up_sync(0xffffffffu, is, d);
-                const uint32_t q = __shfl_up_sync(0xffffffffu, iq, d);
-                if (lane >= d) {
-                    is += a;
-                    iq += q;
-                }
-            }
-            const uint32_t bs = rowc[r] + is - ts, bq = rowc[BAND + r] + iq - tq;
-            *reinterpret_cast<uint4*>(&rp_s[r][4 * lane]) = make_uint4(bs + es[0], bs + es[1], bs + es[2], bs + es[3]);
-            *reinterpret_cast<uint4*>(&rp_q[r][4 * lane]) = make_uint4(bq + eq[0], bq + eq[1], bq + eq[2], bq + eq[3]);
+        for (int i = 0; i < 16; i += 4) {
+            *reinterpret_cast<uint4*>(&rp_s[r][16 * sg + i]) =
+                make_uint4(bs + ps[i], bs + ps[i + 1], bs + ps[i + 2], bs + ps[i + 3]);
+            *reinterpret_cast<uint4*>(&rp_q[r][16 * sg + i]) =
+                make_uint4(bq + pq[i], bq + pq[i + 1], bq + pq[i + 2], bq + pq[i + 3]);
         }
     }
     if (warp == 0) {     // top row ii[y0][X] = corner + sum_{x0 <= x < X} carry[x]
+        const int x = x0 + 4 * lane;
         uint32_t cv[4];
         QT cq[4];
 #pragma unroll
@@ -400,71 +405,35 @@ __global__ void __launch_bounds__(K1_THREADS) k_tile(const uint8_t* __restrict__
     }
     __syncthreads();
 
-    // ---- column phase: thread (q4, sg) owns ii columns x0+4q4.. and rows 4sg..4sg+3
-    const int q4 = threadIdx.x & 31;
-    const int sg = threadIdx.x >> 5;
-    {
-        uint32_t ss[4] = {0, 0, 0, 0};
-        QT sq[4] = {0, 0, 0, 0};
-#pragma unroll
-        for (int rr = 0; rr < 4; ++rr) {
-            const int r = 4 * sg + rr;
-            if (r < rows) {
-                const uint4 a = *reinterpret_cast<const uint4*>(&rp_s[r][4 * q4]);
-                const uint4 q = *reinterpret_cast<const uint4*>(&rp_q[r][4 * q4]);
-                ss[0] += a.x; ss[1] += a.y; ss[2] += a.z; ss[3] += a.w;
-                sq[0] += q.x; sq[1] += q.y; sq[2] += q.z; sq[3] += q.w;
-            }
+    // ---- column phase: thread (plane, column)
+    const int col = tid & (CHUNK - 1), plane = tid / CHUNK;
+    const int X = x0 + col;
+    const int P = CANON ? out_pitch : L.P;
+    if (X >= P) return;
+    if (plane == 0) {
+        uint32_t* o = CANON ? out_ii + (size_t)g * (L.H + 1) * out_pitch
+                            : ws + L.ws_off + (size_t)g * 2 * (size_t)(L.H + 1) * L.P;
+        if (b == 0) o[X] = 0u;                    // ii row 0
+        uint32_t acc = top_s[col];
+        o += (size_t)(y0 + 1) * P + X;
+#pragma unroll 8
+        for (int r = 0; r < rows; ++r) {
+            acc += rp_s[r][col];
+            o[(size_t)r * P] = acc;
         }
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            seg_s[sg][4 * q4 + j] = ss[j];
-            seg_q[sg][4 * q4 + j] = sq[j];
-        }
-    }
-    __syncthreads();
-    uint32_t os[4];
-    QT oq[4];
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-        os[j] = top_s[4 * q4 + j];
-        oq[j] = top_q[4 * q4 + j];
-    }
-    for (int s2 = 0; s2 < sg; ++s2) {
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            os[j] += seg_s[s2][4 * q4 + j];
-            oq[j] += seg_q[s2][4 * q4 + j];
-        }
-    }
-    const int X = x0 + 4 * q4;
-    if (b == 0 && sg == 0 && X < P) {       // ii row 0 is zero
-        *reinterpret_cast<uint4*>(o_ii + X) = make_uint4(0, 0, 0, 0);
-        if constexpr (CANON) {
-            *reinterpret_cast<ulonglong2*>(o_sq + X) = make_ulonglong2(0, 0);
-            *reinterpret_cast<ulonglong2*>(o_sq + X + 2) = make_ulonglong2(0, 0);
-        } else {
-            *reinterpret_cast<uint4*>(o_sq + X) = make_uint4(0, 0, 0, 0);
-        }
-    }
-#pragma unroll
-    for (int rr = 0; rr < 4; ++rr) {
-        const int r = 4 * sg + rr;
-        if (r < rows) {
-            const uint4 a = *reinterpret_cast<const uint4*>(&rp_s[r][4 * q4]);
-            const uint4 q = *reinterpret_cast<const uint4*>(&rp_q[r][4 * q4]);
-            os[0] += a.x; os[1] += a.y; os[2] += a.z; os[3] += a.w;
-            oq[0] += q.x; oq[1] += q.y; oq[2] += q.z; oq[3] += q.w;
-            if (X < P) {
-                const size_t o = (size_t)(y0 + r + 1) * P + X;
-                *reinterpret_cast<uint4*>(o_ii + o) = make_uint4(os[0], os[1], os[2], os[3]);
-                if constexpr (CANON) {
-                    *reinterpret_cast<ulonglong2*>(o_sq + o) = make_ulonglong2(oq[0], oq[1]);
-                    *reinterpret_cast<ulonglong2*>(o_sq + o + 2) = make_ulonglong2(oq[2], oq[3]);
-                } else {
-                    *reinterpret_cast<uint4*>(o_sq + o) = make_uint4(oq[0], oq[1], oq[2], oq[3]);
-                }
-            }
+    } else {
+        QT* o;
+        if constexpr (CANON)
+            o = reinterpret_cast<QT*>(out_sq) + (size_t)g * (L.H + 1) * out_pitch;
+        else
+            o = reinterpret_cast<QT*>(ws + L.ws_off + (size_t)g * 2 * (size_t)(L.H + 1) * L.P + (size_t)(L.H + 1) * L.P);
+        if (b == 0) o[X] = (QT)0;
+        QT acc = top_q[col];
+        o += (size_t)(y0 + 1) * P + X;
+#pragma unroll 8
+        for (int r = 0; r < rows; ++r) {
+            acc += (QT)rp_q[r][col];
+            o[(size_t)r * P] = acc;
         }
     }
 }

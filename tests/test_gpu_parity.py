@@ -131,7 +131,8 @@ K2_SCHEDULES = {
     "split_default": {},                                    # K1 -> k_stage1 -> k_deep1 -> k_tail
     "split_s0_1": {"FD_S0": "1"},                           # k_stage1 stage 1 only
     "split_no_tail": {"FD_TAIL": "0"},                      # k_deep1 finishes every window
-    "split_no_split_stump": {"FD_DEEP_SPLIT": "0"},         # deep stages without the split-stump mode
+    "split_split_stump": {"FD_DEEP_SPLIT": "64"},           # deep stages <= 64 windows split-stump
+    "split_deep_2warps": {"FD_K2D_THREADS": "64"},          # two-warp k_deep1 blocks
     "split_s_tail_3": {"FD_S_TAIL": "3"},                   # every window alive at stage 3 through k_tail
     "split_two_slot": {"FD_GROUP_FRAMES": "1"},             # 3 frame groups over 2 slots/streams
     "split_one_slot": {"FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
@@ -142,7 +143,7 @@ K2_SCHEDULES = {
     "f1_small_groups": {"FD_F1": "1", "FD_GROUP_FRAMES": "1"},
     "f1_one_slot": {"FD_F1": "1", "FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
     "f1_fused": {"FD_F1": "1", "FD_F1_SPLIT": "0"},         # k_f1 runs every stage
-    "f1_fused_no_split_stump": {"FD_F1": "1", "FD_F1_SPLIT": "0", "FD_DEEP_SPLIT": "0"},
+    "f1_fused_split_stump": {"FD_F1": "1", "FD_F1_SPLIT": "0", "FD_DEEP_SPLIT": "64"},
     "f1_fused_s_tail_1": {"FD_F1": "1", "FD_F1_SPLIT": "0", "FD_S_TAIL": "1"},   # all stage-1 survivors to k_tail
     "f1_tail_global_records": {"FD_F1": "1", "FD_TAIL_SMEM_STUMPS": "0", "FD_S_TAIL": "3"},
     "queue": {"FD_K2_QUEUE": "1"},                          # k_soft's schedule on a hard cascade

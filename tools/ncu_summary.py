@@ -93,17 +93,20 @@ def main():
             if key in k:
                 lines.append(f"| {label} (`{key}`) | {k[key]} {units.get(key, '')} |")
         lines.append("")
-        dr = (num(k.get("dram__bytes_read.sum")) or 0) + (num(k.get("dram__bytes_write.sum")) or 0)
-        ub = units.get("dram__bytes_read.sum", "byte")
-        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(ub, 1)
-        # per-launch DRAM bytes of each K2 kernel family and of K1 (first capture of each kernel)
-        fam = ("k_stage1" if "k_stage1" in name else "k_deep" if ("k_deep" in name or "k_tail" in name)
-               else "k1" if any(t in name for t in ("k_marg", "k_carry", "k_corner", "k_tile")) else None)
-        if fam and name not in seen:
+        def scaled(key):
+            v = num(k.get(key)) or 0.0
+            return v * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}.get(units.get(key, "byte"), 1)
+        dr = scaled("dram__bytes_read.sum") + scaled("dram__bytes_write.sum")
+        l2 = scaled("lts__t_bytes.sum")
+        # per-launch DRAM / L2 bytes of each kernel (first capture of each), K1 summed as "k1"
+        short = name.split("<")[0].replace("void ", "").strip()
+        fam = "k1" if any(t in short for t in ("k_marg", "k_carry", "k_corner", "k_tile")) else short
+        if name not in seen:
             seen.add(name)
-            key = f"{fam}_dram_bytes_per_launch"
-            traffic[key] = traffic.get(key, 0.0) + dr * scale
-            traffic["frames_per_launch"] = a.frames_per_launch
+            t = traffic.setdefault(fam, {"dram_bytes_per_launch": 0.0, "l2_bytes_per_launch": 0.0,
+                                         "frames_per_launch": a.frames_per_launch})
+            t["dram_bytes_per_launch"] += dr
+            t["l2_bytes_per_launch"] += l2
     if a.launches:
         agg = launches(a.launches)
         tot = sum(v[1] for v in agg.values())
