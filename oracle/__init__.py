@@ -72,6 +72,16 @@ def _load():
             L.fdo_group.argtypes = [P, i64, dbl, i32, P, i64]
             L.fdo_s_eyes.restype = dbl
             L.fdo_s_eyes.argtypes = [dbl] * 8
+            L.fdo_half_bits.restype = C.c_int32
+            L.fdo_half_bits.argtypes = [f32]
+            L.fdo_half_value.restype = f32
+            L.fdo_half_value.argtypes = [C.c_uint16]
+            L.fdo_pack16.restype = i32
+            L.fdo_pack16.argtypes = [P, P]
+            L.fdo_unpack16.restype = i32
+            L.fdo_unpack16.argtypes = [P, i32, P]
+            L.fdo_cascade_words.restype = i64
+            L.fdo_cascade_words.argtypes = [P, P, i64]
             _lib = L
     return _lib
 
@@ -83,6 +93,7 @@ def _p(a: np.ndarray):
 class _CascadeC(C.Structure):
     _fields_ = [("win_w", C.c_int32), ("win_h", C.c_int32), ("n_stages", C.c_int32),
                 ("n_stumps", C.c_int32), ("filter", C.c_int32), ("soft", C.c_int32),
+                ("packed", C.c_int32), ("words", C.c_void_p), ("n_words", C.c_int64),
                 ("stages", C.c_void_p), ("stumps", C.c_void_p)]
 
 
@@ -271,6 +282,55 @@ def group(dets: np.ndarray, eyes_thresh: float = 0.5, min_neighbors: int = 1) ->
     out = np.zeros(max(cnt, 0), DET_DTYPE)
     if cnt > 0:
         L.fdo_group(_p(dets), len(dets), float(eyes_thresh), min_neighbors, _p(out), cnt)
+    return out
+
+
+class _RectC(C.Structure):
+    _fields_ = [("x", C.c_int32), ("y", C.c_int32), ("w", C.c_int32), ("h", C.c_int32), ("wt", C.c_int32)]
+
+
+class _StumpC(C.Structure):
+    _fields_ = [("nrect", C.c_int32), ("r", _RectC * 3), ("theta", C.c_float), ("left", C.c_float),
+                ("right", C.c_float)]
+
+
+def half_bits(v: float) -> int:
+    """f3 (R13): IEEE binary16 bits of v, or -1 if v is not exactly a finite binary16 value."""
+    return int(_load().fdo_half_bits(float(v)))
+
+
+def half_value(h: int) -> float:
+    return float(np.float32(_load().fdo_half_value(int(h))))
+
+
+def pack16(rects, theta, left, right):
+    """f3 (R13): a stump -> its compressed words (list of uint16), or None."""
+    s = _StumpC()
+    s.nrect = len(rects)
+    for i, (x, y, w, h, wt) in enumerate(rects):
+        s.r[i] = _RectC(x, y, w, h, wt)
+    s.theta, s.left, s.right = float(theta), float(left), float(right)
+    out = (C.c_uint16 * 9)()
+    n = _load().fdo_pack16(C.byref(s), out)
+    return None if n < 0 else [int(v) for v in out[:n]]
+
+
+def unpack16(words, nrect):
+    """f3: compressed words -> (rects, theta, left, right)."""
+    arr = (C.c_uint16 * len(words))(*words)
+    s = _StumpC()
+    _load().fdo_unpack16(arr, nrect, C.byref(s))
+    rects = [(s.r[i].x, s.r[i].y, s.r[i].w, s.r[i].h, s.r[i].wt) for i in range(nrect)]
+    return rects, float(np.float32(s.theta)), float(np.float32(s.left)), float(np.float32(s.right))
+
+
+def cascade_words(casc: "Cascade") -> np.ndarray:
+    """The compressed word stream of a 'compress packed16' cascade (empty otherwise)."""
+    L = _load()
+    n = L.fdo_cascade_words(casc._h, None, 0)
+    out = np.zeros(max(n, 0), np.uint16)
+    if n > 0:
+        L.fdo_cascade_words(casc._h, _p(out), n)
     return out
 
 

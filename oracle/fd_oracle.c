@@ -83,7 +83,84 @@ void fdo_cascade_free(fdo_cascade* c) {
     if (!c) return;
     free(c->stages);
     free(c->stumps);
+    free(c->words);
     free(c);
+}
+
+/* ------------------------------------------------------------------------------------ */
+/* f3: compressed feature records (reading R13)                              */
+/* ------------------------------------------------------------------------------------ */
+
+/* IEEE binary16 value of h: (-1)^s * 2^(e-15) * (1 + m/1024) for 1 <= e <= 30,
+ * (-1)^s * 2^-14 * (m/1024) for e = 0 (subnormals and zero); e = 31 is inf / NaN. */
+float fdo_half_value(uint16_t h) {
+    const int sgn = h >> 15, e = (h >> 10) & 31, m = h & 1023;
+    double v;
+    if (e == 31) v = m ? NAN : INFINITY;
+    else if (e == 0) v = ldexp((double)m, -24);
+    else v = ldexp(1024.0 + (double)m, e - 25);
+    return (float)(sgn ? -v : v);
+}
+
+/* binary16 bits of v if v is exactly a finite binary16 value, else -1: search the exponent whose
+ * grid contains v (plain definition, no conversion intrinsics) */
+int32_t fdo_half_bits(float v) {
+    if (!isfinite(v)) return -1;
+    const int sgn = signbit(v) ? 1 : 0;
+    const double a = fabs((double)v);
+    if (a == 0.0) return sgn << 15;
+    for (int e = 0; e <= 30; ++e) {
+        /* values of exponent field e: subnormal m * 2^-24 (e = 0), else (1024 + m) * 2^(e-25) */
+        const double scale = ldexp(1.0, e == 0 ? -24 : e - 25);
+        const double q = a / scale;                    /* exact: scale is a power of two */
+        const double lo = e == 0 ? 1.0 : 1024.0, hi = e == 0 ? 1023.0 : 2047.0;
+        if (q >= lo && q <= hi && q == floor(q)) return (sgn << 15) | (e << 10) | ((int)q - (e == 0 ? 0 : 1024));
+    }
+    return -1;
+}
+
+int fdo_pack16(const fdo_stump* s, uint16_t* out) {
+    int n = 0;
+    for (int r = 0; r < s->nrect; ++r) {
+        const fdo_rect* q = &s->r[r];
+        if (q->x < 0 || q->x > 31 || q->y < 0 || q->y > 31 || q->w < 0 || q->w > 31 || q->h < 0 || q->h > 31 ||
+            q->wt < -32 || q->wt > 31)
+            return -1;
+        out[n++] = (uint16_t)(q->x | (q->y << 5) | (q->w << 10));
+        out[n++] = (uint16_t)(q->h | ((q->wt & 63) << 5));
+    }
+    const int32_t t = fdo_half_bits(s->theta), l = fdo_half_bits(s->left), rr = fdo_half_bits(s->right);
+    if (t < 0 || l < 0 || rr < 0) return -1;
+    out[n++] = (uint16_t)t;
+    out[n++] = (uint16_t)l;
+    out[n++] = (uint16_t)rr;
+    return n;
+}
+
+int fdo_unpack16(const uint16_t* in, int nrect, fdo_stump* s) {
+    int n = 0;
+    memset(s, 0, sizeof *s);
+    s->nrect = nrect;
+    for (int r = 0; r < nrect; ++r) {
+        const uint16_t a = in[n++], b = in[n++];
+        s->r[r].x = a & 31;
+        s->r[r].y = (a >> 5) & 31;
+        s->r[r].w = (a >> 10) & 31;
+        s->r[r].h = b & 31;
+        const int wt = (b >> 5) & 63;
+        s->r[r].wt = wt >= 32 ? wt - 64 : wt;          /* 6-bit two's complement */
+    }
+    s->theta = fdo_half_value(in[n++]);
+    s->left = fdo_half_value(in[n++]);
+    s->right = fdo_half_value(in[n++]);
+    return n;
+}
+
+int64_t fdo_cascade_words(const fdo_cascade* c, uint16_t* out, int64_t cap) {
+    if (!c->packed) return 0;
+    if (out)
+        for (int64_t i = 0; i < c->n_words && i < cap; ++i) out[i] = c->words[i];
+    return c->n_words;
 }
 
 #define PERR(...) do { if (err && errlen > 0) snprintf(err, (size_t)errlen, __VA_ARGS__); goto fail; } while (0)
@@ -122,6 +199,14 @@ fdo_cascade* fdo_cascade_parse(const char* text, size_t len, char* err, int errl
     if (tok_word(&s, "soft")) {           /* optional: soft cascade (f4, reading R8b) */
         if (!at_end(s)) PERR("line %d: expected 'soft'", cur.line);
         c->soft = 1;
+        if (!next_line(&cur, line, sizeof line)) PERR("line %d: missing stages", cur.line);
+        s = line;
+    } else {
+        s = line;
+    }
+    if (tok_word(&s, "compress")) {       /* optional: compressed records (f3, reading R13) */
+        if (!tok_word(&s, "packed16") || !at_end(s)) PERR("line %d: expected 'compress packed16'", cur.line);
+        c->packed = 1;
         if (!next_line(&cur, line, sizeof line)) PERR("line %d: missing stages", cur.line);
         s = line;
     } else {
@@ -176,6 +261,18 @@ fdo_cascade* fdo_cascade_parse(const char* text, size_t len, char* err, int errl
         }
     }
     if (next_line(&cur, line, sizeof line)) PERR("line %d: trailing content", cur.line);
+    if (c->packed) {
+        /* encode every stump, then replace it by its decoded form: the cascade that is evaluated is
+           the one the compressed words describe */
+        c->words = (uint16_t*)malloc(sizeof(uint16_t) * (size_t)c->n_stumps * 9);
+        if (!c->words) PERR("out of memory");
+        for (int j = 0; j < c->n_stumps; ++j) {
+            const int n = fdo_pack16(&c->stumps[j], c->words + c->n_words);
+            if (n < 0) PERR("stump %d: not representable in packed16 (binary16 theta/left/right, fields)", j);
+            fdo_unpack16(c->words + c->n_words, c->stumps[j].nrect, &c->stumps[j]);
+            c->n_words += n;
+        }
+    }
     return c;
 fail:
     fdo_cascade_free(c);

@@ -30,6 +30,11 @@ typedef struct {
     int32_t filter;          /* 0: identity; 1: binomial 3x3 after scaling (.fdc 'filter binomial3') */
     int32_t soft;            /* 0: stage sums restart at 0 (R8); 1: soft cascade (.fdc 'soft'), the sum runs
                                 over all stumps and T_s is a rejection threshold on the running sum (R8b) */
+    int32_t packed;          /* 1: '.fdc compress packed16' (f3, reading R13): every stump is stored as two 16-bit
+                                words per rectangle + binary16 theta/left/right, and the stumps evaluated are
+                                the ones DECODED from those words */
+    uint16_t* words;         /* packed16: the compressed stream (per stump: 2 words per rect, theta, left, right) */
+    int64_t n_words;
     fdo_stage* stages;
     fdo_stump* stumps;
 } fdo_cascade;
@@ -45,6 +50,19 @@ typedef struct {
  * taps not given; reading R3b): 3x3 binomial [1 2 1]^T [1 2 1] / 16 with round-half-up
  * ((sum + 8) >> 4) and clamp-to-edge, in place on a W x H (pitch W) level image. */
 void fdo_filter_binomial(uint8_t* img, int W, int H);
+
+/* f3 ("reencoding and combining them into two 16-bit words using simple bitwise
+ * operations and masks"; reading R13).  Rectangle (x, y, w, h, wt): word 0 = x | y << 5 | w << 10,
+ * word 1 = h | (wt & 63) << 5 (wt as 6-bit two's complement).  theta, left, right: IEEE binary16.
+ * fdo_half_bits returns -1 if v is not exactly a finite binary16 value. */
+int32_t fdo_half_bits(float v);
+float fdo_half_value(uint16_t h);
+/* stump -> words (2 * nrect + 3); returns the word count, -1 if not representable */
+int fdo_pack16(const fdo_stump* s, uint16_t* out);
+/* words -> stump (nrect given); returns the words consumed */
+int fdo_unpack16(const uint16_t* in, int nrect, fdo_stump* s);
+/* the packed stream of a 'compress packed16' cascade (0 words otherwise); returns n_words */
+int64_t fdo_cascade_words(const fdo_cascade* c, uint16_t* out, int64_t cap);
 
 /* .fdc text -> cascade (NULL on error, message in err). */
 fdo_cascade* fdo_cascade_parse(const char* text, size_t len, char* err, int errlen);

@@ -542,3 +542,84 @@ def test_group_greedy_closest_pair_first():
     # a(0), b(9), c(18): S(a,b)=S(b,c)=0.45 -> (a,b) merge first (mean 4.5), then S(ab,c)=0.675 -> stop
     g = oracle.group(np.array([_det(0, 0, 0, 100), _det(0, 9, 0, 100), _det(0, 18, 0, 100)], D))
     assert sorted(g["aux"].tolist()) == [1, 2]
+
+
+# ---------------------------------------------------------------- f3: compressed records (R13)
+def test_packed16_hand_words():
+    """f3: the compressed words of two hand-encoded stumps (tests/golden/packed16.txt)
+    and their decoding back to the same stump."""
+    g = {r[0]: [int(v) for v in r[1:]] for r in _golden("packed16.txt")}
+    worked = ([(1, 1, 22, 22, -1), (1, 1, 11, 22, 2)], -0.5, 0.25, 0.75)
+    diag = ([(2, 3, 8, 8, -1), (2, 3, 4, 4, 2), (6, 7, 4, 4, 2)], 1.5, -1.0, 0.125)
+    for name, st in (("worked", worked), ("diagonal", diag)):
+        w = oracle.pack16(*st)
+        assert w == g[name], name
+        assert oracle.unpack16(w, len(st[0])) == (st[0], st[1], st[2], st[3])
+
+
+def test_binary16_codec_against_library():
+    """f3: the oracle's binary16 decoder (written from the IEEE 754 definition) equals numpy's
+    float16 for all 63488 finite encodings, and its encoder inverts it; values that are not
+    binary16 are refused."""
+    bits = np.arange(1 << 16, dtype=np.uint16)
+    finite = ((bits >> 10) & 31) != 31
+    ref = bits.view(np.float16).astype(np.float32)
+    for b in bits[finite][::7]:
+        v = oracle.half_value(int(b))
+        assert np.float32(v).view(np.uint32) == ref[b].view(np.uint32), hex(b)
+        h = oracle.half_bits(v)
+        assert h == int(b) or (v == 0.0 and h in (0, 0x8000)), hex(b)
+    for v, h in ((1.0, 0x3C00), (-2.0, 0xC000), (65504.0, 0x7BFF), (2.0 ** -24, 0x0001), (2.0 ** -14, 0x0400)):
+        assert oracle.half_bits(v) == h
+    for v in (0.1, 1.0 / 3.0, 65520.0, 2.0 ** -25, float("inf"), float(np.float32(1 + 2 ** -11))):
+        assert oracle.half_bits(v) == -1, v
+
+
+def test_packed_weights_and_fields():
+    """f3: 6-bit two's-complement weights cover the parser's range [-16, 16]; every field range
+    round-trips; a value outside binary16 makes the stump unpackable."""
+    for wt in (-16, -9, -3, -2, -1, 1, 2, 3, 9, 16):
+        rects = [(0, 0, 24, 24, wt), (23, 1, 1, 23, -wt)]
+        w = oracle.pack16(rects, 0.0, -0.0, 1.0)
+        assert oracle.unpack16(w, 2)[0] == rects
+    assert oracle.pack16([(1, 1, 2, 2, 1)], 0.1, 0.5, 0.5) is None
+
+
+def test_packed_cascade_round_trip_and_equivalence():
+    """f3 workload c6q (c6 with binary16 theta/leaves, 'compress packed16'): the word stream is the
+    concatenation of each stump's words, every stump decodes to the file's values, and the cascade
+    detects exactly what the same text WITHOUT the compress line detects (the decoded records are
+    the file's records)."""
+    path = os.path.join(ROOT, "cascades", "c6q.fdc")
+    text = open(path).read()
+    casc = oracle.Cascade(text)
+    words = oracle.cascade_words(casc)
+    stumps = []
+    for line in text.splitlines():
+        t = line.split()
+        if t and t[0] == "stump":
+            nr = int(t[1])
+            rects = [tuple(int(v) for v in t[2 + 5 * r: 7 + 5 * r]) for r in range(nr)]
+            vals = [float.fromhex(v) for v in t[2 + 5 * nr: 5 + 5 * nr]]
+            stumps.append((rects, *vals))
+    assert len(stumps) == casc.n_stumps == 2913
+    at = 0
+    for st in stumps:
+        w = oracle.pack16(*st)
+        assert w is not None and list(words[at:at + len(w)]) == w
+        assert oracle.unpack16(w, len(st[0])) == st
+        at += len(w)
+    assert at == len(words)
+    plain = oracle.Cascade(text.replace("compress packed16\n", ""))
+    assert len(oracle.cascade_words(plain)) == 0
+    W, H, s = 320, 240, 1.25
+    lv = oracle.plan(W, H, 24, s, 1)
+    fr, _ = fdgen.frames(6, 3, 2, W, H, lv, faces="fixed", face_param=3, max_face_level=8)
+    a, _ = oracle.detect(casc, fr, 24, s, 1, nthreads=4)
+    b, _ = oracle.detect(plain, fr, 24, s, 1, nthreads=4)
+    assert np.array_equal(a, b)
+    # a cascade whose values are not binary16 cannot be compressed
+    c1 = open(os.path.join(ROOT, "cascades", "c1.fdc")).read().replace("window 24 24\n", "window 24 24\ncompress packed16\n")
+    with pytest.raises(ValueError):
+        oracle.Cascade(c1)
+
