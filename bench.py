@@ -55,9 +55,10 @@ def parse_args():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=2, help="frames timed on the CPU oracle")
-    ap.add_argument("--cascade", default="c3", choices=["c3", "c6", "c3s"],
+    ap.add_argument("--cascade", default="c3", choices=["c3", "c6", "c6q", "c3s"],
                     help="c3: the paper-shaped 1446-stump cascade (c4 workload, default); c6: the "
-                         "OpenCV-shaped 2913-stump cascade (SURVEY 8(f) f3 workload); c3s: c3 as a soft "
+                         "OpenCV-shaped 2913-stump cascade (SURVEY 8(f) f3 workload); c6q: c6 with compressed "
+                         "records (f3, 'compress packed16'); c3s: c3 as a soft "
                          "cascade (SURVEY 8(f) f4, reading R8b, k_soft)")
     return ap.parse_args()
 
@@ -212,6 +213,8 @@ def make_frames(rank: int, n: int, plan):
 
 CASCADES = {"c3": ("c4", "25-stage 1446-stump cascade (cascades/c3.fdc)"),
             "c6": ("c6", "OpenCV-shaped 25-stage 2913-stump cascade (cascades/c6.fdc)"),
+            "c6q": ("c6q", "c6 with compressed records: two 16-bit words per rectangle, binary16 theta/leaves "
+                           "(cascades/c6q.fdc, 'compress packed16')"),
             "c3s": ("c4-soft", "25-stage 1446-stump soft cascade (cascades/c3s.fdc, running-sum thresholds)")}
 
 

@@ -172,6 +172,8 @@ struct fd_cascade_s {
     int device = 0;
     int filter = 0;                         // filtering stage after scaling: 0 none, 1 binomial 3x3
     int soft = 0;                           // 1: soft cascade (f4, reading R8b), stage sums carried over
+    int compressed = 0;                     // 1: 'compress packed16' (f3, reading R13)
+    std::vector<uint32_t> pk16;             // f3: FD_PK_WORDS u32 per stump (rects: two 16-bit words each)
     std::vector<HStump> stumps;
     std::vector<HStage> stages;
     std::mutex mu;
@@ -197,6 +199,51 @@ struct fd_cascade_s {
 using Packed = fd_cascade_s::Packed;
 
 namespace {
+
+// f3 ("reencoding and combining them into two 16-bit words using simple bitwise
+// operations and masks"; reading R13).  binary16 from a float by its bits: exact only if the float's
+// exponent is in binary16 range and the dropped fraction bits are zero.  -1 if not representable.
+int half_bits_of(float v) {
+    uint32_t u;
+    std::memcpy(&u, &v, 4);
+    const uint32_t sgn = (u >> 16) & 0x8000u, e = (u >> 23) & 255u, m = u & 0x7fffffu;
+    if (e == 255u) return -1;                           // inf / nan
+    if (e == 0u) return m == 0u ? (int)sgn : -1;        // +-0 (fp32 subnormals are below binary16)
+    const int ue = (int)e - 127;                        // unbiased exponent
+    if (ue > 15) return -1;
+    if (ue >= -14) {                                    // normal binary16: 10 fraction bits
+        if (m & 0x1fffu) return -1;
+        return (int)(sgn | (uint32_t)(ue + 15) << 10 | (m >> 13));
+    }
+    // subnormal binary16: value = q * 2^-24 with q = (2^23 + m) * 2^(ue - 23 + 24)
+    const int sh = -14 - ue;                            // 1 .. (extra right shift beyond 13)
+    if (sh > 10) return -1;
+    const uint32_t full = 0x800000u | m;
+    if (full & ((1u << (13 + sh)) - 1u)) return -1;
+    return (int)(sgn | (full >> (13 + sh)));
+}
+float half_to_float(uint32_t h) {                        // exact widening
+    const uint32_t sgn = (h & 0x8000u) << 16, e = (h >> 10) & 31u, m = h & 1023u;
+    uint32_t u;
+    if (e == 0u) {
+        if (m == 0u) {
+            u = sgn;
+        } else {                                        // subnormal: normalise
+            int ee = -1;
+            uint32_t mm = m;
+            do {
+                ++ee;
+                mm <<= 1;
+            } while (!(mm & 1024u));
+            u = sgn | (uint32_t)(127 - 15 - ee) << 23 | (mm & 1023u) << 13;
+        }
+    } else {
+        u = sgn | (e - 15u + 127u) << 23 | m << 13;
+    }
+    float v;
+    std::memcpy(&v, &u, 4);
+    return v;
+}
 
 fd_status parse_cascade(const char* text, size_t len, fd_cascade_s* c) {
     std::vector<Line> lines;
@@ -253,6 +300,11 @@ fd_status parse_cascade(const char* text, size_t len, fd_cascade_s* c) {
         c->soft = 1;
         L = need("stages");
     }
+    if (L && !L->tok.empty() && L->tok[0] == "compress") {    // optional compressed records (f3, R13)
+        if (L->tok.size() != 2 || L->tok[1] != "packed16") return fail(FD_EFORMAT, "line %d: expected 'compress packed16'", L->no);
+        c->compressed = 1;
+        L = need("stages");
+    }
     long ns = 0;
     if (!L || L->tok.size() != 2 || L->tok[0] != "stages" || !parse_int(L->tok[1], &ns) || ns < 1 || ns > 250)
         return fail(FD_EFORMAT, "line %d: expected 'stages N' with 1 <= N <= 250", L ? L->no : 0);
@@ -293,6 +345,33 @@ fd_status parse_cascade(const char* text, size_t len, fd_cascade_s* c) {
         }
     }
     if (li != lines.size()) return fail(FD_EFORMAT, "line %d: trailing content", lines[li].no);
+    if (c->compressed) {
+        // encode each stump into its compressed record, then evaluate what the record says
+        c->pk16.assign(c->stumps.size() * FD_PK_WORDS, 0u);
+        for (size_t j = 0; j < c->stumps.size(); ++j) {
+            HStump& sp = c->stumps[j];
+            uint32_t* R = &c->pk16[j * FD_PK_WORDS];
+            for (int r = 0; r < sp.nrect; ++r) {
+                const int x = sp.r[r][0], y = sp.r[r][1], w = sp.r[r][2], h = sp.r[r][3], wt = sp.r[r][4];
+                if (wt < -32 || wt > 31) return fail(FD_EFORMAT, "stump %zu: weight %d outside the packed16 range", j, wt);
+                const uint32_t lo = (uint32_t)(x | y << 5 | w << 10), hi = (uint32_t)(h | (wt & 63) << 5);
+                R[r] = lo | hi << 16;
+                sp.r[r][0] = (int)(R[r] & 31u);
+                sp.r[r][1] = (int)((R[r] >> 5) & 31u);
+                sp.r[r][2] = (int)((R[r] >> 10) & 31u);
+                sp.r[r][3] = (int)((R[r] >> 16) & 31u);
+                sp.r[r][4] = (int)(R[r] << 5) >> 26;
+            }
+            const int th = half_bits_of(sp.theta), lf = half_bits_of(sp.left), rt = half_bits_of(sp.right);
+            if (th < 0 || lf < 0 || rt < 0)
+                return fail(FD_EFORMAT, "stump %zu: theta/left/right not exactly binary16 (packed16)", j);
+            R[3] = (uint32_t)th | (uint32_t)lf << 16;
+            R[4] = (uint32_t)rt | (uint32_t)sp.nrect << 16;
+            sp.theta = half_to_float(R[3] & 0xffffu);
+            sp.left = half_to_float(R[3] >> 16);
+            sp.right = half_to_float(R[4] & 0xffffu);
+        }
+    }
     return FD_OK;
 }
 
@@ -750,7 +829,8 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         if (!c->jit_tried) {
             c->jit_tried = true;
             std::string err;
-            c->jit = jit_k2_build(pk->h_rec.data(), pk->h_st.data(), (int)pk->h_st.size(), &err);
+            c->jit = jit_k2_build(pk->h_rec.data(), pk->h_st.data(), (int)pk->h_st.size(),
+                                  c->compressed ? &c->pk16 : nullptr, &err);
             if (!c->jit) return fail(FD_ECUDA, "K2 specialisation: %s", err.c_str());
         }
         jit = c->jit;
@@ -918,7 +998,8 @@ fd_status fd_debug_jit_compile(const char* text, size_t len, size_t* cubin_bytes
     std::vector<char> cubin;
     std::vector<std::string> lowered;
     std::string err;
-    if (!jit_k2_compile(jit_program(pk.h_rec.data(), pk.h_st.data(), (int)pk.h_st.size()), false, &cubin, &lowered, &err))
+    if (!jit_k2_compile(jit_program(pk.h_rec.data(), pk.h_st.data(), (int)pk.h_st.size(), c->compressed ? &c->pk16 : nullptr),
+                        false, &cubin, &lowered, &err))
         return fail(FD_ECUDA, "%s", err.c_str());
     if (cubin_bytes) *cubin_bytes = cubin.size();
     return FD_OK;

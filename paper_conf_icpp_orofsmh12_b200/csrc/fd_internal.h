@@ -36,6 +36,7 @@ constexpr int BAND = 32;             // K1 band height (rows)
 constexpr int CHUNK = 128;           // K1 chunk width (ii columns): 32 lanes x 4
 constexpr int K1_THREADS = 256;
 constexpr int REC_WORDS = 16;        // packed stump record: 16 u32 (64 B)
+#define FD_PK_WORDS 5                // f3 compressed record (R13): 3 rects (two 16-bit words each), theta|left, right|nrect
 constexpr int MAX_CORNERS = 12;
 constexpr int MAX_STEP = 4;
 

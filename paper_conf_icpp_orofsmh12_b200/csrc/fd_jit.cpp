@@ -38,6 +38,7 @@ struct KindGeo {
 };
 struct JitK2 {
     std::string key;                              // generated program (NVRTC source)
+    std::vector<uint32_t> pk16;                   // f3 records for the module's __constant__ fd_pk
     KindGeo geo[JIT_KINDS];
     cudaKernel_t kern[2][JIT_KINDS] = {};         // [depth][kind], compiled on first use (g_jit_mu)
     int grid[2][JIT_KINDS] = {};
@@ -181,9 +182,18 @@ static int jit_ctas() {
     return c < 2 ? 2 : (c > 6 ? 6 : c);
 }
 
-std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages) {
+std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages, const std::vector<uint32_t>* pk16) {
     const int k_end = jit_deep_end(st, n_stages);
-    std::string src = "#define FD_K2D_CTAS " + std::to_string(env_or("FD_K2D_CTAS", FD_K2D_CTAS)) +
+    std::string pre;
+    if (pk16 && !pk16->empty()) {
+        // the records are data of this program (its own __constant__ bank); a digest of them in the
+        // source keeps cascades with equal generated code from sharing a loaded module
+        unsigned long long h = 1469598103934665603ull;
+        for (uint32_t w : *pk16) h = (h ^ w) * 1099511628211ull;
+        pre = "// packed16 records digest " + std::to_string(h) + "\n#define FD_PACKED_WORDS " +
+              std::to_string(pk16->size()) + "\n";
+    }
+    std::string src = pre + "#define FD_K2D_CTAS " + std::to_string(env_or("FD_K2D_CTAS", FD_K2D_CTAS)) +
                       "\n#define FD_K2D_THREADS " + std::to_string(jit_deep_threads()) +
                       "\n#define FD_F1_CTAS " + std::to_string(env_or("FD_F1_CTAS", FD_F1_CTAS)) +
                       "\n#define FD_K2_CTAS " + std::to_string(jit_ctas()) +
@@ -227,6 +237,8 @@ bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cu
         names[k] = jit_name(k, depth);
         nvrtcAddNameExpression(prog, names[k].c_str());
     }
+    const bool packed = source.find("#define FD_PACKED_WORDS") != std::string::npos;
+    if (packed) nvrtcAddNameExpression(prog, "&fdk::fd_pk");
     const bool verbose = std::getenv("FD_JIT_VERBOSE") && std::getenv("FD_JIT_VERBOSE")[0] == '1';
     const char* opts[] = {"-arch=sm_100a", "-std=c++17", "--fmad=false", "-lineinfo", "-default-device",
                           "--ptxas-options=-v"};
@@ -245,20 +257,27 @@ bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cu
     nvrtcGetCUBINSize(prog, &cb);
     cubin->resize(cb);
     nvrtcGetCUBIN(prog, cubin->data());
-    lowered->assign(JIT_KINDS, std::string());
+    lowered->assign(JIT_KINDS + 1, std::string());
     for (int k = 0; k < JIT_KINDS; ++k) {
         const char* lw = nullptr;
         nvrtcGetLoweredName(prog, names[k].c_str(), &lw);
         (*lowered)[k] = lw ? lw : "";
     }
+    if (packed) {                                 // [JIT_KINDS]: the constant bank of the f3 records
+        const char* lw = nullptr;
+        nvrtcGetLoweredName(prog, "&fdk::fd_pk", &lw);
+        (*lowered)[JIT_KINDS] = lw ? lw : "";
+    }
     nvrtcDestroyProgram(&prog);
     return true;
 }
 
-JitK2* jit_k2_build(const uint32_t* rec_words, const StageDev* st, int n_stages, std::string* err) {
+JitK2* jit_k2_build(const uint32_t* rec_words, const StageDev* st, int n_stages, const std::vector<uint32_t>* pk16,
+                    std::string* err) {
     (void)err;
     std::unique_ptr<JitK2> J(new JitK2());
-    J->key = jit_program(rec_words, st, n_stages);
+    J->key = jit_program(rec_words, st, n_stages, pk16);
+    if (pk16) J->pk16 = *pk16;
     for (int k = 0; k < JIT_KINDS; ++k) J->geo[k] = jit_kind_geo(k);
     return J.release();
 }
@@ -294,6 +313,15 @@ cudaError_t jit_k2_launch(JitK2* J, const CascadeParams& p, bool depth, int kind
                     return cudaErrorInvalidSource;
                 }
                 cudaError_t e = cudaLibraryLoadData(&L.lib, cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0);
+                if (e == cudaSuccess && !J->pk16.empty()) {      // f3: fill the module's constant bank once
+                    void* dp = nullptr;
+                    size_t bytes = 0;
+                    e = cudaLibraryGetGlobal(&dp, &bytes, L.lib, lowered[JIT_KINDS].c_str());
+                    if (e == cudaSuccess && bytes == J->pk16.size() * 4)
+                        e = cudaMemcpy(dp, J->pk16.data(), bytes, cudaMemcpyHostToDevice);
+                    else if (e == cudaSuccess)
+                        e = cudaErrorInvalidValue;
+                }
                 int dev = 0, sms = 0;
                 if (e == cudaSuccess) e = cudaGetDevice(&dev);
                 if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);

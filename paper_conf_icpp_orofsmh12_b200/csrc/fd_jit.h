@@ -17,12 +17,16 @@ std::string jit_stage1_source(const uint32_t* rec_words, int first, int n);
 // generated deep stages [1, k_end) (lane-per-window code with immediate corner offsets)
 std::string jit_deep_source(const uint32_t* rec_words, const StageDev* st, int k_end);
 // the whole NVRTC program for a cascade (generated stages + k_cascade.cu)
-std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages);
+// pk16: f3 compressed records (FD_PK_WORDS u32 per stump) held in the program's __constant__ bank
+// and read by the lane-per-window deep stages, or null
+std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages,
+                        const std::vector<uint32_t>* pk16 = nullptr);
 // NVRTC compile only (no device needed): cubin + lowered names of the JIT_KINDS kernels
 bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cubin, std::vector<std::string>* lowered,
                     std::string* err);
 // specialisation handle for one cascade (code generated now, compiled and loaded on first launch)
-JitK2* jit_k2_build(const uint32_t* rec_words, const StageDev* st, int n_stages, std::string* err);
+JitK2* jit_k2_build(const uint32_t* rec_words, const StageDev* st, int n_stages, const std::vector<uint32_t>* pk16,
+                    std::string* err);
 // launch (compiling on first use; cudaErrorInvalidSource + *err when NVRTC fails)
 cudaError_t jit_k2_launch(JitK2* j, const CascadeParams& p, bool depth, int kind, cudaStream_t st, std::string* err);
 void jit_k2_free(JitK2* j);

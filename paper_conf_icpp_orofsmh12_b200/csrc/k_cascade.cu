@@ -44,6 +44,54 @@ extern "C" int fd_debug_k2_timing(unsigned long long* out, int reset) {
 #define FD_JIT_DEEP 0        // run-time specialised kernel: deep stages [1, FD_JIT_DEEP) are generated code
 #endif
 
+#ifdef FD_PACKED_WORDS
+// f3 (reading R13): the cascade's compressed records, resident in this program's
+// constant bank (58 KB for the 2913-stump c6q) and read warp-uniformly (constant-cache broadcast,
+// the paper's reason for compressing them).  Record j: words 0-2 = rectangles (x | y<<5 | w<<10 in
+// the low 16 bits, h | wt<<5 in the high 16 bits, wt 6-bit two's complement; an absent rectangle
+// is all zeros), word 3 = theta | left << 16, word 4 = right | nrect << 16 (binary16 values).
+__constant__ uint32_t fd_pk[FD_PACKED_WORDS];
+
+// binary16 -> binary32, exact (finite values only: the parser refuses the others): a normal value
+// re-biases its exponent (15 -> 127); a subnormal m * 2^-24 is an exact fp32 product
+__device__ __forceinline__ float half_bits_to_float(uint32_t h) {
+    const uint32_t sgn = (h & 0x8000u) << 16, e = (h >> 10) & 31u, m = h & 1023u;
+    if (e) return __uint_as_float(sgn | ((e + 112u) << 23) | (m << 13));
+    const float v = __fmul_rn(__uint2float_rn(m), 0x1p-24f);
+    return sgn ? -v : v;
+}
+
+// One stage for one window from the compressed records: f = sum_r wt_r * (A - B - C + D) (mod 2^32,
+// equal to the corner-compiled sum), leaf = ((float)f < theta*nf) ? left : right, fp32 sum in
+// stump order (oracle c6-c8).
+template <int STEP>
+__device__ __forceinline__ float eval_stage_packed(const uint32_t* __restrict__ T, int b, float nf, int first, int n) {
+    constexpr int TW = tile_w(STEP);
+    float sum = 0.0f;
+    for (int j = first; j < first + n; ++j) {
+        const uint32_t* r = fd_pk + FD_PK_WORDS * j;
+        const uint32_t w3 = r[3], w4 = r[4];
+        const int nr = (int)(w4 >> 16);
+        uint32_t f = 0;
+#pragma unroll
+        for (int q = 0; q < 3; ++q) {
+            if (q < nr) {
+                const uint32_t w = r[q];
+                const int x = (int)(w & 31u), y = (int)((w >> 5) & 31u), ww = (int)((w >> 10) & 31u);
+                const int h = (int)((w >> 16) & 31u), wt = (int)(w << 5) >> 26;
+                const uint32_t* a = T + b + y * TW + x;
+                const uint32_t R = a[0] - a[ww] - a[h * TW] + a[h * TW + ww];
+                f += (uint32_t)wt * R;
+            }
+        }
+        const float th = half_bits_to_float(w3 & 0xffffu), lf = half_bits_to_float(w3 >> 16);
+        const float rt = half_bits_to_float(w4 & 0xffffu);
+        sum = __fadd_rn(sum, (__int2float_rn((int)f) < __fmul_rn(th, nf)) ? lf : rt);
+    }
+    return sum;
+}
+#endif
+
 // Output of a window of ii slot sl (batch tile table in shared memory).
 template <int STEP, bool DEPTH>
 struct WinOut {
@@ -315,8 +363,12 @@ __device__ __forceinline__ void deep_phase(const CascadeParams& p, int s0, const
                     sum = jit_deep(s, slots + b, nfw);
                 else
 #endif
+#ifdef FD_PACKED_WORDS
+                    sum = eval_stage_packed<STEP>(slots, b, nfw, sd.first, sd.n);   // f3: constant-bank records
+#else
                     sum = in_param ? eval_stage(slots, b, nfw, prec, sd.first, sd.n, sd.mc)
                                    : eval_stage(slots, b, nfw, grec, sd.first, sd.n, sd.mc);
+#endif
             }
             const bool pass = act && (sum >= sd.T);
             if (act && !pass) reject(sl, idx, s, sum);

@@ -209,6 +209,60 @@ def test_c6_workload_1080p():
     assert sc.cpu().tolist() == [int((od >= k).sum()) for k in range(gc.n_stages + 1)]
 
 
+def _to_packed16(text):
+    """Input generation (f3): a cascade text with theta/left/right rounded to binary16 and the
+    'compress packed16' line (the oracle re-checks representability when it parses it)."""
+    out = []
+    for line in text.splitlines():
+        t = line.split()
+        if t and t[0] == "window":
+            out += [line, "compress packed16"]
+            continue
+        if t and t[0] == "stump":
+            b = 2 + 5 * int(t[1])
+            t[b:b + 3] = [float(np.float32(np.float16(float.fromhex(v) if "x" in v else float(v)))).hex() for v in t[b:b + 3]]
+            line = " ".join(t)
+        out.append(line)
+    return "\n".join(out) + "\n"
+
+
+@pytest.mark.parametrize("jit", ["1", "0"])
+def test_c6q_compressed_1080p(jit, monkeypatch):
+    """f3 (R13): the compressed 2913-stump workload c6q -- the JIT program evaluates the
+    deep lane-per-window stages from the compressed records in its constant bank, the generic
+    kernels from the decoded corner records; both bit-exact with the oracle (which evaluates the
+    decoded records): depth maps, detections and stage counters at 1080p."""
+    monkeypatch.setenv("FD_JIT", jit)
+    W, H, s = 1920, 1080, 1.1
+    lv = oracle.plan(W, H, 24, s, 1)
+    fr, _ = fdgen.frames(4, 200, 2, W, H, lv, faces="poisson", face_param=4, max_face_level=30)
+    text = open(os.path.join(ROOT, "cascades", "c6q.fdc")).read()
+    pair = (fd.Cascade(text), oracle.Cascade(text))
+    compare_depth(pair, fr[:1], s)
+    gc, oc = pair
+    sc = torch.zeros(gc.n_stages + 1, dtype=torch.int64, device="cuda")
+    got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1, capacity=1 << 20, stage_counts=sc))
+    ref, _ = oracle.detect(oc, fr, 24, s, 1, nthreads=os.cpu_count())
+    assert np.array_equal(got, ref)
+    od, _, _ = oracle.detect_depth(oc, fr, 24, s, 1, nthreads=os.cpu_count())
+    assert sc.cpu().tolist() == [int((od >= k).sum()) for k in range(gc.n_stages + 1)]
+
+
+@pytest.mark.parametrize("cfg", [1, 2])
+def test_packed16_small_configs(cfg):
+    """f3 on the c1/c2 cascades rounded to binary16 (incl. 3-rect stumps and steps): depth maps
+    bit-exact; a non-binary16 cascade is refused by the library as by the oracle."""
+    W, H, s, _ = CFG[cfg]
+    text = _to_packed16(open(os.path.join(ROOT, "cascades", f"c{cfg}.fdc")).read())
+    pair = (fd.Cascade(text), oracle.Cascade(text))
+    fr, _ = gen(cfg, 50, 2)
+    compare_depth(pair, fr, s)
+    compare_depth(pair, fr, s, step=2)
+    bad = open(os.path.join(ROOT, "cascades", f"c{cfg}.fdc")).read().replace("window 24 24\n", "window 24 24\ncompress packed16\n")
+    with pytest.raises(fd.FDError):
+        fd.Cascade(bad)
+
+
 @pytest.mark.parametrize("cfg,n,step", [(1, 3, 1), (2, 2, 2), (3, 1, 1)])
 def test_depth_histogram(cfg, n, step):
     """f4: fd_depth_histogram (Fig. 7 analytics) equals the oracle's histogram of the oracle
