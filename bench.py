@@ -270,10 +270,22 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
+    # one process per GPU; FD_DIST_BACKEND=gloo lets ranks share a device (the 2-rank dry run of
+    # this branch on a 1-GPU box, tests/test_dist.py); the detection lists then travel via the host
+    backend = os.environ.get("FD_DIST_BACKEND", "nccl")
+    dev_index = local % max(torch.cuda.device_count(), 1)
+    torch.cuda.set_device(dev_index)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev_index))
+        else:
+            dist.init_process_group(backend)
+    dev = torch.device("cuda", dev_index)
+
+    def allreduce_max(x: float) -> float:
+        t = torch.tensor([x], dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
     F = args.frames
     plan = fd.fd_pyramid_plan(CFG["W"], CFG["H"], CFG["min_size"], CFG["scale"], CFG["step"])
     frames_np, _faces = make_frames(rank, F, plan)
@@ -304,7 +316,7 @@ def run_ours(args):
     torch.cuda.synchronize()
     # ---- the timed region: no counters, no per-kernel events (launch counting only)
     fd.fd_profile_reset(time_kernels=False)
-    clk = ClockSampler(local)
+    clk = ClockSampler(dev_index)
     clk.start()
     barrier()
     torch.cuda.synchronize()
@@ -321,9 +333,7 @@ def run_ours(args):
     launches = fd.fd_profile_read()
     nraw, ngrp = int(dets.shape[0]), int(grp.shape[0])
     if world > 1:
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+        ms = allreduce_max(ms)
     frames_total = F * world * args.steps
     value = frames_total / (ms / 1000.0)
 
@@ -451,9 +461,7 @@ def run_ours(args):
                                              capacity=cap)
         dt = time.perf_counter() - t0
         if world > 1:
-            t = torch.tensor([dt], dtype=torch.float64, device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            dt = float(t.item())
+            dt = allreduce_max(dt)
         out["e2e"] = {"value": F * world * ne / dt, "unit": "frames/s",
                       "h2d_bytes_per_step": int(h_frames.numel()), "d2h_bytes_per_step": int(len(g) * 40),
                       "api": "fd_detect_group_host (pinned host frames -> grouped detections on host)"}

@@ -32,8 +32,12 @@ def globalize(dets: torch.Tensor, frame_offset: int) -> torch.Tensor:
 
 def gather_detections(dets: torch.Tensor, group=None) -> torch.Tensor:
     """All-gather variable-length [n_r, 10] int32 detection tensors; returns the concatenation
-    in rank order on every rank.  Two collectives: counts, then padded payloads."""
+    in rank order on every rank.  Two collectives: counts, then padded payloads.  With a backend
+    that cannot move device tensors (gloo) the payload goes through host memory and the result
+    comes back to the caller's device."""
     world = dist.get_world_size(group)
+    if dets.is_cuda and dist.get_backend(group) != "nccl":
+        return gather_detections(dets.cpu(), group).to(dets.device)
     dev = dets.device
     cnt = torch.tensor([dets.shape[0]], dtype=torch.int64, device=dev)
     counts = [torch.zeros_like(cnt) for _ in range(world)]
