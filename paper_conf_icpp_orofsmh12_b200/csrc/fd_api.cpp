@@ -723,6 +723,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     make_plan_dev(pl, W, H, pitch, step, G, &PD);
     PD.filter = c->filter;
     PD.aligned4 = ((reinterpret_cast<uintptr_t>(d_frames) | (uintptr_t)pitch) & 3) == 0;
+    PD.aligned16 = ((reinterpret_cast<uintptr_t>(d_frames) | (uintptr_t)pitch) & 15) == 0;
     // two pipeline slots on two streams when there is more than one group (FD_PIPE=0: one)
     const int nslots = (ngroups > 1 && env_int("FD_PIPE", 1) != 0) ? 2 : 1;
     K1Scratch k1s[2];
@@ -1056,6 +1057,7 @@ fd_status fd_integral(const uint8_t* d_img, int n, int W, int H, int pitch, uint
     PlanDev p;
     make_plan_dev(pl, W, H, pitch, 1, 1, &p);
     p.aligned4 = ((reinterpret_cast<uintptr_t>(d_img) | (uintptr_t)pitch) & 3) == 0;
+    p.aligned16 = ((reinterpret_cast<uintptr_t>(d_img) | (uintptr_t)pitch) & 15) == 0;
     Workspace* w = nullptr;
     r = get_ws(st, &w);
     if (r != FD_OK) return r;

@@ -177,6 +177,7 @@ struct PlanDev {
     int G;                  // frames per group (tensor-map extent)
     int filter;             // K1: 1 = binomial 3x3 filtering stage after scaling (f2)
     int aligned4;           // frames pointer and pitch are 4-byte aligned (word loads of identity levels)
+    int aligned16;          // ... 16-byte aligned (staged resampling, k_integral.cu stage_source)
     LevelDev lv[FD_MAX_LEVELS];
 };
 

@@ -17,6 +17,10 @@
 
 namespace fdk {
 
+#ifndef FD_K1_MINB
+#define FD_K1_MINB 1        // min resident CTAs per SM for k_marg / k_tile (6 measured: no gain, k_marg spills)
+#endif
+
 // ---------------------------------------------------------------- scaling (reading R2)
 struct RowSample {
     const uint8_t* r0;
@@ -94,6 +98,67 @@ __device__ __forceinline__ void tile_row_pixels(const uint8_t* frame, const Plan
     }
 }
 
+// Staged resampling (reading R2 unchanged, only where the taps come from): for levels with
+// f <= 2.25 the source rows and columns that the 32 x 128 output pixels of a K1 tile sample are
+// copied to shared memory with 16-byte loads, and the bilinear taps are read there with 32-bit
+// addresses.  For such f every coordinate product fits 32 bits: (2 * 3840 + 1) * 2.25 * 2^16 < 2^31.
+constexpr int STAGE_R16_MAX = 147456;              // 2.25 * 2^16
+constexpr int SRC_ROWS = 74, SRC_PITCH = 336;      // >= 31 * 2.25 + 3 rows; >= 127 * 2.25 + 3 + 15 + 1 columns
+
+struct SrcStage {
+    int ys0, xa;                                   // first staged source row / (16-aligned) column
+};
+
+__device__ __forceinline__ int src_coord(int v, int r16, int lim, int* frac) {
+    const int sv = ((2 * v + 1) * r16 - 65536) >> 1;
+    *frac = (sv >> 8) & 255;
+    const int v0 = sv >> 16;
+    return v0 < lim - 1 ? v0 : lim - 1;
+}
+
+// Copies the tile's source region to S (all threads; ends with a barrier).  The column right of
+// the last frame column is a copy of it, so the tap x0 + 1 is the clamped x1 everywhere.
+__device__ __forceinline__ SrcStage stage_source(const uint8_t* __restrict__ frame, const PlanDev& p, const LevelDev& L,
+                                                 int y0, int rows, int x0, uint8_t* S) {
+    int fr;
+    SrcStage st;
+    st.ys0 = src_coord(y0, L.r16, p.H, &fr);
+    const int ys1 = min(p.H - 1, src_coord(y0 + rows - 1, L.r16, p.H, &fr) + 1);
+    const int xs0 = src_coord(x0, L.r16, p.W, &fr);
+    const int xs1 = min(p.W - 1, src_coord(min(x0 + CHUNK, L.W) - 1, L.r16, p.W, &fr) + 1);
+    st.xa = xs0 & ~15;
+    const int nch = (xs1 - st.xa) / 16 + 1, nr = ys1 - st.ys0 + 1;
+    for (int i = threadIdx.x; i < nr * nch; i += K1_THREADS) {
+        const int r = i / nch, c = i - r * nch;
+        *reinterpret_cast<uint4*>(S + r * SRC_PITCH + 16 * c) =
+            __ldg(reinterpret_cast<const uint4*>(frame + (size_t)(st.ys0 + r) * p.pitch + st.xa + 16 * c));
+    }
+    __syncthreads();
+    if (xs1 == p.W - 1)
+        for (int r = threadIdx.x; r < nr; r += K1_THREADS) S[r * SRC_PITCH + p.W - st.xa] = S[r * SRC_PITCH + p.W - 1 - st.xa];
+    __syncthreads();
+    return st;
+}
+
+// The 4 level pixels of row y at columns x .. x+3 from the staged source (o[j]: staged column of
+// x0(x + j), ax[j] its weight), 0 at or beyond the level width.
+__device__ __forceinline__ void staged_row_pixels(const uint8_t* __restrict__ S, const PlanDev& p, const LevelDev& L,
+                                                  const SrcStage& st, int y, int x, const int* o, const int* ax,
+                                                  uint32_t* pv) {
+    int ay;
+    const int y0s = src_coord(y, L.r16, p.H, &ay);
+    const int y1s = y0s + 1 < p.H ? y0s + 1 : p.H - 1;
+    const uint8_t* r0 = S + (y0s - st.ys0) * SRC_PITCH;
+    const uint8_t* r1 = S + (y1s - st.ys0) * SRC_PITCH;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        const int h0 = (int)r0[o[j]] * (256 - ax[j]) + (int)r0[o[j] + 1] * ax[j];
+        const int h1 = (int)r1[o[j]] * (256 - ax[j]) + (int)r1[o[j] + 1] * ax[j];
+        const uint32_t v = (uint32_t)((h0 * (256 - ay) + h1 * ay + 32768) >> 16);
+        pv[j] = x + j < L.W ? v : 0u;
+    }
+}
+
 __device__ __forceinline__ int find_level_k1(const PlanDev& p, int t) {
     int k = 0;
     while (k + 1 < p.n_levels && p.lv[k + 1].k1t0 <= t) ++k;
@@ -103,7 +168,7 @@ __device__ __forceinline__ int find_level_k1(const PlanDev& p, int t) {
 // ---------------------------------------------------------------- K1a: per-tile marginals
 // colsum[band][plane][x] = sum over the tile's rows of p (plane 0) / p^2 (plane 1)
 // rowsum[band][chunk][plane][r] = sum over the tile's columns
-__global__ void __launch_bounds__(K1_THREADS) k_marg(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
+__global__ void __launch_bounds__(K1_THREADS, FD_K1_MINB) k_marg(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
                                                      K1Scratch s) {
     __shared__ uint32_t red_s[8][CHUNK], red_q[8][CHUNK];
     __shared__ uint8_t raw[BAND + 2][CHUNK + 4];       // filtering stage: resampled rows with a 1-px halo
@@ -117,6 +182,8 @@ __global__ void __launch_bounds__(K1_THREADS) k_marg(const uint8_t* __restrict__
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint8_t* frame = frames + (size_t)g * p.H * p.pitch;
     const int x = x0 + 4 * lane;
+    // (staged resampling, as in k_level, measured slower here: 14.5 vs 13.5 ms per 512 frames --
+    // the extra 25 KB of shared memory costs this short-lived, latency-bound kernel occupancy)
     ColSample cs[4];
     if (L.r16 != 65536) {
 #pragma unroll
@@ -305,7 +372,7 @@ struct BandOut<true> {
 // prefixes to the tile's top row ii[y0][X] and stores each ii / sqii entry once (a warp stores
 // 32 consecutive entries of a row: 128 or 256 B).
 template <bool CANON>
-__global__ void __launch_bounds__(K1_THREADS) k_tile(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
+__global__ void __launch_bounds__(K1_THREADS, FD_K1_MINB) k_tile(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
                                                      K1Scratch s, uint32_t* __restrict__ ws,
                                                      uint32_t* __restrict__ out_ii,
                                                      unsigned long long* __restrict__ out_sq, int out_pitch) {
@@ -447,6 +514,7 @@ __global__ void __launch_bounds__(K1_THREADS) k_tile(const uint8_t* __restrict__
 __global__ void __launch_bounds__(K1_THREADS) k_level(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
                                                       uint8_t* __restrict__ out) {
     __shared__ uint8_t raw[BAND + 2][CHUNK + 4];       // filtering stage: resampled rows with a 1-px halo
+    __shared__ __align__(16) uint8_t src[SRC_ROWS * SRC_PITCH];   // staged source region
     const int g = blockIdx.y;
     const int k = find_level_k1(p, blockIdx.x);
     const LevelDev& L = p.lv[k];
@@ -457,8 +525,15 @@ __global__ void __launch_bounds__(K1_THREADS) k_level(const uint8_t* __restrict_
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint8_t* frame = frames + (size_t)g * p.H * p.pitch;
     const int x = x0 + 4 * lane;
+    const bool staged = !p.filter && p.aligned16 && L.r16 != 65536 && L.r16 <= STAGE_R16_MAX;
     ColSample cs[4];
-    if (L.r16 != 65536) {
+    int so[4], sax[4];
+    SrcStage sst{0, 0};
+    if (staged) {
+        sst = stage_source(frame, p, L, y0, rows, x0, src);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) so[j] = src_coord(min(x + j, L.W - 1), L.r16, p.W, &sax[j]) - sst.xa;
+    } else if (L.r16 != 65536) {
 #pragma unroll
         for (int j = 0; j < 4; ++j) cs[j] = col_sample(p.W, L.r16, min(x + j, L.W - 1));
     }
@@ -493,6 +568,8 @@ __global__ void __launch_bounds__(K1_THREADS) k_level(const uint8_t* __restrict_
                     }
                     pv[j] = v;
                 }
+            } else if (staged) {
+                staged_row_pixels(src, p, L, sst, y0 + r, x, so, sax, pv);
             } else {
                 tile_row_pixels(frame, p, L, y0 + r, x, cs, pv);
             }
