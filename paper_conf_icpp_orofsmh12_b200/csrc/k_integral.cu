@@ -17,9 +17,7 @@
 
 namespace fdk {
 
-#ifndef FD_K1_MINB
-#define FD_K1_MINB 1        // min resident CTAs per SM for k_marg / k_tile (6 measured: no gain, k_marg spills)
-#endif
+// (k_marg / k_tile compiled for 6 resident CTAs per SM -- 40 registers -- measured no faster)
 
 // ---------------------------------------------------------------- scaling (reading R2)
 struct RowSample {
@@ -168,7 +166,7 @@ __device__ __forceinline__ int find_level_k1(const PlanDev& p, int t) {
 // ---------------------------------------------------------------- K1a: per-tile marginals
 // colsum[band][plane][x] = sum over the tile's rows of p (plane 0) / p^2 (plane 1)
 // rowsum[band][chunk][plane][r] = sum over the tile's columns
-__global__ void __launch_bounds__(K1_THREADS, FD_K1_MINB) k_marg(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
+__global__ void __launch_bounds__(K1_THREADS) k_marg(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
                                                      K1Scratch s) {
     __shared__ uint32_t red_s[8][CHUNK], red_q[8][CHUNK];
     __shared__ uint8_t raw[BAND + 2][CHUNK + 4];       // filtering stage: resampled rows with a 1-px halo
@@ -372,7 +370,7 @@ struct BandOut<true> {
 // prefixes to the tile's top row ii[y0][X] and stores each ii / sqii entry once (a warp stores
 // 32 consecutive entries of a row: 128 or 256 B).
 template <bool CANON>
-__global__ void __launch_bounds__(K1_THREADS, FD_K1_MINB) k_tile(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
+__global__ void __launch_bounds__(K1_THREADS) k_tile(const uint8_t* __restrict__ frames, const __grid_constant__ PlanDev p,
                                                      K1Scratch s, uint32_t* __restrict__ ws,
                                                      uint32_t* __restrict__ out_ii,
                                                      unsigned long long* __restrict__ out_sq, int out_pitch) {
