@@ -35,6 +35,7 @@ namespace fdk {
 struct KindGeo {
     int threads = 0;
     size_t smem = 0;
+    int grid_per_sm = 0;                          // persistent grid: CTAs per SM (0 = occupancy)
 };
 struct JitK2 {
     std::string key;                              // generated program (NVRTC source)
@@ -220,6 +221,10 @@ static KindGeo jit_kind_geo(int kind) {
     if (kind == JIT_DEEP1) g.smem = TileGeoD<JIT_STEP, false>::SMEM;
     if (kind == JIT_DEEP1_F1) g.smem = TileGeoD<JIT_STEP, true>::SMEM;
     if (kind == JIT_F1) g.smem = TileGeoF<JIT_STEP>::SMEM;
+    // FD_S1_GRID / FD_DEEP_GRID: cap the persistent grids of k_stage1 / k_deep1 at that many CTAs
+    // per SM, so the other pipeline slot's kernels can co-reside
+    if (kind == JIT_STAGE1) g.grid_per_sm = env_or("FD_S1_GRID", 0);
+    if (kind == JIT_DEEP1 || kind == JIT_DEEP1_F1) g.grid_per_sm = env_or("FD_DEEP_GRID", 0);
     return g;
 }
 
@@ -335,6 +340,7 @@ cudaError_t jit_k2_launch(JitK2* J, const CascadeParams& p, bool depth, int kind
                     if (e == cudaSuccess)
                         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, reinterpret_cast<const void*>(L.kern[k]),
                                                                           g.threads, g.smem);
+                    if (g.grid_per_sm > 0 && g.grid_per_sm < per) per = g.grid_per_sm;
                     L.grid[k] = sms * (per > 0 ? per : 1);
                 }
                 if (e != cudaSuccess) {
