@@ -6,7 +6,7 @@
  * Problem statement: "determine the presence of faces in arbitrary images, along with their
  * locations and dimensions" (abstract).  The pipeline is Fig. 1:
  * scaling -> (filtering) -> integral images -> cascade evaluation -> detections.
- * Readings where the paper is silent are listed in DESIGN.md ("Readings", R1..R12).
+ * Readings where the paper is silent are listed in DESIGN.md ("Readings", R1..R13).
  *
  * Conventions common to every entry point
  *   - Every function returns fd_status; FD_OK == 0.  On failure a thread-local message is
@@ -79,8 +79,13 @@ typedef struct {
 } fd_plan;
 
 /* Parse a cascade in .fdc text (format in DESIGN.md "Cascade format": FDC 1 / window 24 24 /
- * optional "filter none|binomial3" / optional "soft" / stages N / per stage "stage n T" / per
- * stump "stump r (x y w h wt)*r theta left right").  "filter binomial3" switches on the filtering
+ * optional "filter none|binomial3" / optional "soft" / optional "compress packed16" / stages N /
+ * per stage "stage n T" / per stump "stump r (x y w h wt)*r theta left right").
+ * "compress packed16" ("reencoding and combining them into two 16-bit
+ * words using simple bitwise operations and masks"; reading R13): every rectangle is stored as two
+ * 16-bit words (x | y<<5 | w<<10, h | (wt & 63)<<5) and theta/left/right as IEEE binary16; the
+ * values in the text must be exactly representable (else FD_EFORMAT) and the stumps evaluated are
+ * the ones decoded from the words.  "filter binomial3" switches on the filtering
  * stage between scaling and the integral images (reading R3b) for
  * fd_detect / fd_detect_depth with this cascade; fd_build_pyramid and fd_integral are unfiltered.
  * "soft" makes it a soft cascade (the paper's future work, ref [32]; SURVEY 8(f)
@@ -124,7 +129,10 @@ fd_status fd_integral(const uint8_t* d_img, int n, int W, int H, int pitch, uint
  * capacity = elements of d_out.  *n_out = number of detections (host).  If
  * *n_out > capacity returns FD_ECAPACITY and d_out is unspecified.
  * Synchronises `stream` once (to read the count); the records in d_out are complete when
- * `stream` next completes. */
+ * `stream` next completes.
+ * Schedules (identical results): default K1 (global ii/sqii) -> k_stage1 ->
+ * k_deep1 -> k_tail; environment FD_F1=1 selects SURVEY 8(f) f1 (k_level -> k_f1 with tile-local
+ * integrals in shared memory -> k_deep1<F1> -> k_tail; no global integral image). */
 fd_status fd_detect(fd_cascade c, const uint8_t* d_frames, int n, int W, int H, int pitch,
                     int min_size, double scale_factor, int step, fd_detection* d_out,
                     int64_t capacity, int64_t* n_out, void* stream);

@@ -75,6 +75,7 @@ def main():
     ap.add_argument("--launches")
     ap.add_argument("--frames-per-launch", type=int, default=16)
     ap.add_argument("--tag", default="r1")
+    ap.add_argument("--l2", help="ncu --metrics lts__t_bytes.sum,... --csv log: per-kernel L2 bytes (first launch)")
     a = ap.parse_args()
     kernels, units = raw(a.full)
     lines = [f"# ncu summary ({a.tag})", "",
@@ -107,6 +108,32 @@ def main():
                                          "frames_per_launch": a.frames_per_launch})
             t["dram_bytes_per_launch"] += dr
             t["l2_bytes_per_launch"] += l2
+    if a.l2:
+        rows = list(csv.reader(open(a.l2)))
+        for i, r in enumerate(rows):
+            if "Kernel Name" in r:
+                hdr, data = r, rows[i + 1:]
+                break
+        idx = {h: j for j, h in enumerate(hdr)}
+        first = {}
+        for r in data:
+            if len(r) < len(hdr):
+                continue
+            name = r[idx["Kernel Name"]].split("(")[0].replace("void ", "").split("<")[0].replace("fdk::", "").strip()
+            fam = "k1" if any(t in name for t in ("k_marg", "k_tile")) else name
+            key = (name, r[idx["ID"]])
+            first.setdefault(name, r[idx["ID"]])
+            if first[name] != r[idx["ID"]]:
+                continue
+            scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(r[idx["Metric Unit"]], 1)
+            if r[idx["Metric Name"]] == "lts__t_bytes.sum" and fam in traffic:
+                traffic[fam]["l2_bytes_per_launch"] += (num(r[idx["Metric Value"]]) or 0.0) * scale
+        lines += ["## L2 traffic (`ncu --metrics lts__t_bytes.sum`, first launch of each kernel, bytes)", "",
+                  "| kernel | L2 bytes per launch | DRAM bytes per launch |", "|---|---|---|"]
+        for fam, t in traffic.items():
+            if isinstance(t, dict):
+                lines.append(f"| {fam} | {t['l2_bytes_per_launch']:.3e} | {t['dram_bytes_per_launch']:.3e} |")
+        lines.append("")
     if a.launches:
         agg = launches(a.launches)
         tot = sum(v[1] for v in agg.values())
