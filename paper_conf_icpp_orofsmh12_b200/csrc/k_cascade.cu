@@ -625,12 +625,20 @@ __global__ void __launch_bounds__(k2_threads(STEP), FD_K2_CTAS) k_cascade(const 
 //   * stage 2 (p.s0 == 2) runs over that list one lane per window; the survivors of the last
 //     stage run here -- window index and nf -- go to a global list at an offset reserved per tile
 //     (tile_rec[tile] = (offset, count)) for k_deep1.
+__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* a) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(a) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_u32(unsigned* a, unsigned v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(a), "r"(v) : "memory");
+}
+
 template <int STEP, bool DEPTH>
-__global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_constant__ CascadeParams p) {
+__device__ __forceinline__ void stage1_tiles(const CascadeParams& p, uint8_t* smem_raw) {
     using G = TileGeoA<STEP>;
     constexpr int TW = tile_w(STEP), TX = k2_tx(STEP), TY = k2_ty(STEP), WPT = k2_wpt(STEP);
     constexpr int WARPS_X = TX / 32, PLANE = tile_w(STEP) * tile_h(STEP), THREADS = k2_threads(STEP);
-    extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint32_t* Q = reinterpret_cast<uint32_t*>(smem_raw + G::OFF_Q);           // sqii plane (mod 2^32)
     float* snf = reinterpret_cast<float*>(smem_raw + G::OFF_SNF);             // [NW] stage-1 survivors: nf
     uint16_t* sidx = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_SIDX);    //       and window index
@@ -698,7 +706,13 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
         if (tid == 0) {
             // the previous tile's record; its counters are reset for the tile after this one (a
             // barrier separates that reset from their next use)
-            if (s_prev >= 0) p.tile_rec[s_prev] = make_uint2((unsigned)s_prev_off, (unsigned)s_c2[b ^ 1]);
+            if (s_prev >= 0) {
+                p.tile_rec[s_prev] = make_uint2((unsigned)s_prev_off, (unsigned)s_c2[b ^ 1]);
+                if (p.tile_ready) {               // k_k2r: publish the tile to the deep CTAs
+                    __threadfence();
+                    st_release_u32(p.tile_ready + s_prev, 1u);
+                }
+            }
             s_prev = -1;
             s_c1[b ^ 1] = 0;
             s_c2[b ^ 1] = 0;
@@ -811,6 +825,12 @@ __global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_con
     }
 }
 
+template <int STEP, bool DEPTH>
+__global__ void __launch_bounds__(k2_threads(STEP), 3) k_stage1(const __grid_constant__ CascadeParams p) {
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    stage1_tiles<STEP, DEPTH>(p, smem_raw);
+}
+
 // ======================================================================== f1: fused K2
 // the tile's integral images are built in shared memory from its level pixels,
 // so no ii / sqii plane ever makes an HBM round trip (the paper's integral kernels take "20% of
@@ -907,11 +927,13 @@ __device__ __forceinline__ void build_tile_integral(const uint8_t* __restrict__ 
 // tile with stage-1 survivors, TMAs its ii plane and runs deep_phase over the survivors (in
 // chunks of CP); with ~25 KB of shared memory and 4 warps per CTA, FD_K2D_CTAS tiles are in
 // flight per SM, so the latency-bound stage chains of different tiles overlap.
-template <int STEP, bool DEPTH, bool F1 = false>
-__global__ void __launch_bounds__(K2D_THREADS, FD_K2D_CTAS) k_deep1(const __grid_constant__ CascadeParams p) {
+// The deep stages of tiles claimed in order from p.deep_counter, by THREADS threads starting at
+// TID0 synchronising on barrier BAR (0: the whole CTA); WAIT: spin until the tile is published
+// (k_k2r, where stage-1 CTAs of the same launch produce the tiles).
+template <int STEP, bool DEPTH, bool F1, int THREADS, int TID0, int BAR, bool WAIT>
+__device__ __forceinline__ void deep_tiles(const CascadeParams& p, uint8_t* smem_raw) {
     using G = TileGeoD<STEP, F1>;
     constexpr int CP = G::CP, PLANE = tile_w(STEP) * tile_h(STEP);
-    extern __shared__ __align__(1024) uint8_t smem_raw[];
     uint32_t* slot = reinterpret_cast<uint32_t*>(smem_raw);
     float* pnf = reinterpret_cast<float*>(smem_raw + G::OFF_NF);
     uint16_t* ploc = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LOC);
@@ -921,7 +943,7 @@ __global__ void __launch_bounds__(K2D_THREADS, FD_K2D_CTAS) k_deep1(const __grid
     __shared__ int s_frame[1], s_lvl[1], s_wx0[1], s_wy0[1];
     __shared__ int s_cnt[3];
     __shared__ int s_tpos, s_tile, s_off, s_n;
-    const int tid = threadIdx.x;
+    const int tid = (int)threadIdx.x - TID0;
     const WinOut<STEP, DEPTH> out{p, s_frame, s_lvl, s_wx0, s_wy0};
     if (tid == 0) {
         mbar_init(&mbar, 1);
@@ -929,13 +951,15 @@ __global__ void __launch_bounds__(K2D_THREADS, FD_K2D_CTAS) k_deep1(const __grid
     }
     uint32_t phase = 0;
     for (;;) {
-        __syncthreads();
+        phase_sync<BAR, THREADS>();
         if (tid == 0) {
             int tn;
             uint2 tr = make_uint2(0u, 0u);
             do {
                 tn = (int)atomicAdd(p.deep_counter, 1u);
                 if (tn >= p.total_tiles) break;
+                if constexpr (WAIT)
+                    while (!ld_acquire_u32(p.tile_ready + tn)) __nanosleep(256);
                 tr = p.tile_rec[tn];
             } while (tr.y == 0u);
             s_tile = tn;
@@ -957,13 +981,13 @@ __global__ void __launch_bounds__(K2D_THREADS, FD_K2D_CTAS) k_deep1(const __grid
                 s_n = (int)tr.y;
             }
         }
-        __syncthreads();
+        phase_sync<BAR, THREADS>();
         if (s_tile >= p.total_tiles) break;
         const int off = s_off, n = s_n;
         for (int c0 = 0; c0 < n; c0 += CP) {
             const int m = min(CP, n - c0);
-            if (c0) __syncthreads();              // previous chunk's deep phase done with the pool
-            for (int e = tid; e < m; e += K2D_THREADS) {
+            if (c0) phase_sync<BAR, THREADS>();   // previous chunk's deep phase done with the pool
+            for (int e = tid; e < m; e += THREADS) {
                 const uint2 v = p.surv[off + c0 + e];
                 ploc[e] = (uint16_t)v.x;
                 pnf[e] = __int_as_float((int)v.y);
@@ -977,12 +1001,44 @@ __global__ void __launch_bounds__(K2D_THREADS, FD_K2D_CTAS) k_deep1(const __grid
             if (c0 == 0) {
                 mbar_wait(&mbar, phase);
                 phase ^= 1;
-                if constexpr (F1) build_tile_integral<STEP, K2D_THREADS, false>(U, slot, nullptr);
+                if constexpr (F1) build_tile_integral<STEP, THREADS, false>(U, slot, nullptr);
             }
-            __syncthreads();
-            deep_phase<STEP, DEPTH, CP, K2D_THREADS>(p, p.s0, slot, pnf, ploc, lists, s_cnt, s_tpos, out,
-                                                     reinterpret_cast<float2*>(smem_raw + G::OFF_RED));
+            phase_sync<BAR, THREADS>();
+            deep_phase<STEP, DEPTH, CP, THREADS, TID0, BAR>(p, p.s0, slot, pnf, ploc, lists, s_cnt, s_tpos, out,
+                                                           reinterpret_cast<float2*>(smem_raw + G::OFF_RED));
         }
+    }
+}
+
+template <int STEP, bool DEPTH, bool F1 = false>
+__global__ void __launch_bounds__(K2D_THREADS, FD_K2D_CTAS) k_deep1(const __grid_constant__ CascadeParams p) {
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    deep_tiles<STEP, DEPTH, F1, K2D_THREADS, 0, 0, false>(p, smem_raw);
+}
+
+// k_k2r: k_stage1 and k_deep1 as CTA roles of ONE persistent launch.  Every role_div-th CTA is a
+// deep CTA whose two 4-warp halves (named barriers 1 and 2) each consume tiles in the order the
+// stage-1 CTAs publish them (tile_ready, release/acquire), while those tiles' ii planes are still
+// L2-resident, and whose latency-bound stage chains overlap the stage-1 CTAs' dense work on the
+// same SMs.  Deadlock-free: stage-1 CTAs never wait on deep CTAs, and CTAs dispatch in blockIdx
+// order, so stage-1 CTAs are resident before any deep CTA can wait for them.
+constexpr size_t k2r_half_bytes(int step) {
+    return (step == 1 ? TileGeoD<1>::SMEM : step == 2 ? TileGeoD<2>::SMEM : step == 3 ? TileGeoD<3>::SMEM
+                                                                                          : TileGeoD<4>::SMEM) +
+           1023 & ~(size_t)1023;
+}
+template <int STEP, bool DEPTH>
+__global__ void __launch_bounds__(k2_threads(STEP), 3) k_k2r(const __grid_constant__ CascadeParams p) {
+    extern __shared__ __align__(1024) uint8_t smem_raw[];
+    static_assert(K2D_THREADS == 128 && k2_threads(STEP) == 256, "two 4-warp deep halves per deep CTA");
+    static_assert(2 * k2r_half_bytes(STEP) <= TileGeoA<STEP>::SMEM, "deep halves fit the stage-1 layout");
+    if ((int)(blockIdx.x % (unsigned)p.role_div) == p.role_div - 1) {
+        if (threadIdx.x < 128)
+            deep_tiles<STEP, DEPTH, false, 128, 0, 1, true>(p, smem_raw);
+        else
+            deep_tiles<STEP, DEPTH, false, 128, 128, 2, true>(p, smem_raw + k2r_half_bytes(STEP));
+    } else {
+        stage1_tiles<STEP, DEPTH>(p, smem_raw);
     }
 }
 
