@@ -605,7 +605,7 @@ struct DevBuf {
 // between two such slots on two streams, so K1 of group g+1 overlaps the latency-bound deep
 // stages and tail of group g (different resources: HBM vs issue/latency).
 struct PipeSlot {
-    DevBuf ws, colbuf, rowbuf, corbuf, lvlbuf, tmaps, tailq, surv, tilerec, ready;
+    DevBuf ws, colbuf, rowbuf, corbuf, lvlbuf, tmaps, tailq, surv, tilerec;
     // K1 scratch for g frames of plan p
     cudaError_t k1_scratch(const PlanDev& p, int g, K1Scratch* s) {
         cudaError_t e = colbuf.ensure((size_t)g * p.col_frame * 4 + 16);
@@ -627,26 +627,11 @@ struct Workspace {
     PipeSlot slot[2];              // pipeline slots (slot 0 also serves fd_integral / fd_build_pyramid)
     cudaStream_t side = nullptr;   // stream of slot 1, forked from / joined to the caller's stream
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
-    // FD_K1_PRIO: K1 of each slot on its own highest-priority stream, ordered by events against
-    // the slot's K2 stream (so K1 blocks are dispatched first whenever K2 blocks retire)
-    cudaStream_t hp[2] = {nullptr, nullptr};
-    cudaEvent_t ev_k1[2] = {nullptr, nullptr}, ev_k2[2] = {nullptr, nullptr};
     cudaError_t ensure_side() {
         if (side) return cudaSuccess;
         cudaError_t e = cudaStreamCreateWithFlags(&side, cudaStreamNonBlocking);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_fork, cudaEventDisableTiming);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_join, cudaEventDisableTiming);
-        return e;
-    }
-    cudaError_t ensure_hp() {
-        if (hp[0]) return cudaSuccess;
-        int lo = 0, hi = 0;
-        cudaError_t e = cudaDeviceGetStreamPriorityRange(&lo, &hi);
-        for (int b = 0; b < 2 && e == cudaSuccess; ++b) {
-            e = cudaStreamCreateWithPriority(&hp[b], cudaStreamNonBlocking, hi);
-            if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_k1[b], cudaEventDisableTiming);
-            if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ev_k2[b], cudaEventDisableTiming);
-        }
         return e;
     }
     cudaError_t k1_scratch(const PlanDev& p, int g, K1Scratch* s) { return slot[0].k1_scratch(p, g, s); }
@@ -661,11 +646,6 @@ struct Workspace {
         if (ev_fork) cudaEventDestroy(ev_fork);
         if (ev_join) cudaEventDestroy(ev_join);
         if (side) cudaStreamDestroy(side);
-        for (int b = 0; b < 2; ++b) {
-            if (ev_k1[b]) cudaEventDestroy(ev_k1[b]);
-            if (ev_k2[b]) cudaEventDestroy(ev_k2[b]);
-            if (hp[b]) cudaStreamDestroy(hp[b]);
-        }
     }
 };
 
@@ -722,9 +702,6 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     const bool f1_split = f1 && env_int("FD_F1_SPLIT", 1) != 0;
     const bool split = !queue && !f1 && env_int("FD_K2_SPLIT", 1) != 0;
     const bool surv = split || f1_split;
-    // FD_K2R=1: k_stage1 and k_deep1 as CTA roles of one persistent launch (k_k2r; step 1, JIT),
-    // every FD_K2R_DIV-th CTA a deep CTA
-    const bool k2r = split && step == 1 && env_int("FD_K2R", 0) != 0 && env_int("FD_JIT", 1) != 0;
     // tail queue (k_tail): FD_TAIL=0 keeps every window inside K2; FD_TAIL_N = windows left in a
     // batch at which it hands them over; FD_TAIL_CAP = queue entries (16 B each) per group
     const bool use_tail = !queue && env_int("FD_TAIL", 1) != 0;
@@ -757,7 +734,6 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
             CK(sl.surv.ensure((size_t)G * (size_t)PD.win_per_frame * 8 + 16));
             CK(sl.tilerec.ensure((size_t)G * PD.tiles_per_frame * 8 + 16));
         }
-        if (k2r) CK(sl.ready.ensure((size_t)G * PD.tiles_per_frame * 4 + 16));
         if (f1) {
             CK(sl.ws.ensure((size_t)PD.u8_bytes + 16));
             s = encode_maps8(PD, sl.ws.as<uint8_t>(), step, maps.data());
@@ -869,8 +845,6 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         sts[1] = w->side;
     }
     const int grid = cascade_grid(depth, step);
-    const bool k1prio = env_int("FD_K1_PRIO", 0) != 0;
-    if (k1prio) CK(w->ensure_hp());
     for (int gi = 0; gi < ngroups; ++gi) {
         // group gi runs on slot gi % nslots; the slot's stream orders it after group gi - nslots,
         // the previous user of the slot's buffers
@@ -879,12 +853,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         const cudaStream_t gs = sts[b];
         const int f0 = gi * G, gf = (n - f0) < G ? (n - f0) : G;
         const uint8_t* fr = d_frames + (size_t)f0 * H * pitch;
-        cudaStream_t ks = gs;                     // K1's stream
-        if (k1prio) {                             // after the slot's previous K2, on the priority stream
-            ks = w->hp[b];
-            CK(cudaEventRecord(w->ev_k2[b], gs));
-            CK(cudaStreamWaitEvent(ks, w->ev_k2[b], 0));
-        }
+        const cudaStream_t ks = gs;               // K1's stream
         if (f1) {
             LAUNCH(FD_K_LEVEL, ks, launch_levels(fr, PD, gf, sl.ws.as<uint8_t>(), ks));
         } else {
@@ -894,10 +863,6 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
                 CK(launch_k1_carry(PD, gf, k1s[b], ks));
             }
             LAUNCH(FD_K_BAND, ks, launch_k1_tiles(fr, PD, gf, k1s[b], sl.ws.as<uint32_t>(), ks));
-        }
-        if (k1prio) {                             // this group's K2 after its K1
-            CK(cudaEventRecord(w->ev_k1[b], ks));
-            CK(cudaStreamWaitEvent(gs, w->ev_k1[b], 0));
         }
         P.tmaps = sl.tmaps.as<CUtensorMap>();
         P.tail_q = use_tail ? sl.tailq.as<uint4>() : nullptr;
@@ -910,9 +875,6 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         P.deep_counter = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + 3 * ngroups + gi;
         P.surv = surv ? sl.surv.as<uint2>() : nullptr;
         P.tile_rec = surv ? sl.tilerec.as<uint2>() : nullptr;
-        P.tile_ready = k2r ? sl.ready.as<unsigned int>() : nullptr;
-        P.role_div = std::max(2, env_int("FD_K2R_DIV", 3));
-        if (k2r) CK(cudaMemsetAsync(sl.ready.p, 0, (size_t)P.total_tiles * 4, gs));
         const int gr = grid < P.total_tiles ? grid : P.total_tiles;
         if (queue) {
             LAUNCH(FD_K_CASCADE, gs, launch_soft(P, depth, step, soft, gs));
@@ -921,9 +883,9 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
             cudaError_t e;
             {
                 ProfScope ps(FD_K_CASCADE, gs);
-                e = jit_k2_launch(jit, P, depth, k2r ? JIT_K2R : (f1 ? JIT_F1 : (split ? JIT_STAGE1 : JIT_FUSED)), gs, &err);
+                e = jit_k2_launch(jit, P, depth, f1 ? JIT_F1 : (split ? JIT_STAGE1 : JIT_FUSED), gs, &err);
             }
-            if (e == cudaSuccess && surv && !k2r) {
+            if (e == cudaSuccess && surv) {
                 ProfScope ps(FD_K_DEEP, gs);
                 e = jit_k2_launch(jit, P, depth, f1 ? JIT_DEEP1_F1 : JIT_DEEP1, gs, &err);
             }

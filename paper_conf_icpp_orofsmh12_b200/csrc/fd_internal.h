@@ -224,8 +224,6 @@ struct alignas(16) CascadeParams {
     int s_tail;                             // windows still alive at stage s_tail go to the tail queue
     int split_max;                          // deep stages with <= split_max windows use the split-stump mode
     int f1;                                 // 1: tmaps are u8 level-image maps (k_f1, k_deep1 rebuilds ii)
-    unsigned int* tile_ready;               // k_k2r: per tile, 1 once its survivors are published (else null)
-    int role_div;                           // k_k2r: every role_div-th CTA is a deep CTA
     uint2* surv;                            // split K2: stage-1 survivors (window index, nf bits)
     uint2* tile_rec;                        // split K2: per tile (offset into surv, count)
     unsigned int* surv_count;

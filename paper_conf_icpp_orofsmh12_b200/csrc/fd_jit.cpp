@@ -211,7 +211,6 @@ static std::string jit_name(int kind, bool depth) {
     if (kind == JIT_STAGE1) return "fdk::k_stage1<1, " + d + ">";
     if (kind == JIT_DEEP1) return "fdk::k_deep1<1, " + d + ", false>";
     if (kind == JIT_DEEP1_F1) return "fdk::k_deep1<1, " + d + ", true>";
-    if (kind == JIT_K2R) return "fdk::k_k2r<1, " + d + ">";
     return "fdk::k_f1<1, " + d + ">";
 }
 
@@ -219,7 +218,7 @@ static KindGeo jit_kind_geo(int kind) {
     KindGeo g;
     g.threads = (kind == JIT_DEEP1 || kind == JIT_DEEP1_F1) ? jit_deep_threads() : k2_threads(JIT_STEP);
     if (kind == JIT_FUSED) g.smem = TileGeo<JIT_STEP>::SMEM;
-    if (kind == JIT_STAGE1 || kind == JIT_K2R) g.smem = TileGeoA<JIT_STEP>::SMEM;
+    if (kind == JIT_STAGE1) g.smem = TileGeoA<JIT_STEP>::SMEM;
     if (kind == JIT_DEEP1) g.smem = TileGeoD<JIT_STEP, false>::SMEM;
     if (kind == JIT_DEEP1_F1) g.smem = TileGeoD<JIT_STEP, true>::SMEM;
     if (kind == JIT_F1) g.smem = TileGeoF<JIT_STEP>::SMEM;
@@ -342,7 +341,7 @@ cudaError_t jit_k2_launch(JitK2* J, const CascadeParams& p, bool depth, int kind
                     if (e == cudaSuccess)
                         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, reinterpret_cast<const void*>(L.kern[k]),
                                                                           g.threads, g.smem);
-                    if (g.grid_per_sm > 0 && g.grid_per_sm < per) per = g.grid_per_sm;   // (< 0: see launch)
+                    if (g.grid_per_sm > 0 && g.grid_per_sm < per) per = g.grid_per_sm;
                     L.grid[k] = sms * (per > 0 ? per : 1);
                 }
                 if (e != cudaSuccess) {
@@ -359,11 +358,7 @@ cudaError_t jit_k2_launch(JitK2* J, const CascadeParams& p, bool depth, int kind
         kern = J->kern[d][kind];
         kgrid = J->grid[d][kind];
     }
-    // k_k2r keeps its whole grid: its deep CTAs own no tiles of their own.  A negative grid cap
-    // (FD_S1_GRID / FD_DEEP_GRID = -m) launches total_tiles / m CTAs: more CTAs than fit, so the
-    // block scheduler can interleave the other slot's kernels as CTAs retire
-    int grid = (kind == JIT_K2R || kgrid < p.total_tiles) ? kgrid : p.total_tiles;
-    if (J->geo[kind].grid_per_sm < 0) grid = std::max(1, p.total_tiles / -J->geo[kind].grid_per_sm);
+    const int grid = kgrid < p.total_tiles ? kgrid : p.total_tiles;
     void* args[] = {const_cast<CascadeParams*>(&p)};
     return cudaLaunchKernel(reinterpret_cast<const void*>(kern), dim3(grid), dim3(J->geo[kind].threads), args,
                             J->geo[kind].smem, st);

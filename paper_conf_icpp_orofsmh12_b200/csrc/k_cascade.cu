@@ -625,15 +625,6 @@ __global__ void __launch_bounds__(k2_threads(STEP), FD_K2_CTAS) k_cascade(const 
 //   * stage 2 (p.s0 == 2) runs over that list one lane per window; the survivors of the last
 //     stage run here -- window index and nf -- go to a global list at an offset reserved per tile
 //     (tile_rec[tile] = (offset, count)) for k_deep1.
-__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* a) {
-    unsigned v;
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(a) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_release_u32(unsigned* a, unsigned v) {
-    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(a), "r"(v) : "memory");
-}
-
 template <int STEP, bool DEPTH>
 __device__ __forceinline__ void stage1_tiles(const CascadeParams& p, uint8_t* smem_raw) {
     using G = TileGeoA<STEP>;
@@ -706,13 +697,7 @@ __device__ __forceinline__ void stage1_tiles(const CascadeParams& p, uint8_t* sm
         if (tid == 0) {
             // the previous tile's record; its counters are reset for the tile after this one (a
             // barrier separates that reset from their next use)
-            if (s_prev >= 0) {
-                p.tile_rec[s_prev] = make_uint2((unsigned)s_prev_off, (unsigned)s_c2[b ^ 1]);
-                if (p.tile_ready) {               // k_k2r: publish the tile to the deep CTAs
-                    __threadfence();
-                    st_release_u32(p.tile_ready + s_prev, 1u);
-                }
-            }
+            if (s_prev >= 0) p.tile_rec[s_prev] = make_uint2((unsigned)s_prev_off, (unsigned)s_c2[b ^ 1]);
             s_prev = -1;
             s_c1[b ^ 1] = 0;
             s_c2[b ^ 1] = 0;
@@ -928,9 +913,8 @@ __device__ __forceinline__ void build_tile_integral(const uint8_t* __restrict__ 
 // chunks of CP); with ~25 KB of shared memory and 4 warps per CTA, FD_K2D_CTAS tiles are in
 // flight per SM, so the latency-bound stage chains of different tiles overlap.
 // The deep stages of tiles claimed in order from p.deep_counter, by THREADS threads starting at
-// TID0 synchronising on barrier BAR (0: the whole CTA); WAIT: spin until the tile is published
-// (k_k2r, where stage-1 CTAs of the same launch produce the tiles).
-template <int STEP, bool DEPTH, bool F1, int THREADS, int TID0, int BAR, bool WAIT>
+// TID0 synchronising on barrier BAR (0: the whole CTA).
+template <int STEP, bool DEPTH, bool F1, int THREADS, int TID0, int BAR>
 __device__ __forceinline__ void deep_tiles(const CascadeParams& p, uint8_t* smem_raw) {
     using G = TileGeoD<STEP, F1>;
     constexpr int CP = G::CP, PLANE = tile_w(STEP) * tile_h(STEP);
@@ -958,8 +942,6 @@ __device__ __forceinline__ void deep_tiles(const CascadeParams& p, uint8_t* smem
             do {
                 tn = (int)atomicAdd(p.deep_counter, 1u);
                 if (tn >= p.total_tiles) break;
-                if constexpr (WAIT)
-                    while (!ld_acquire_u32(p.tile_ready + tn)) __nanosleep(256);
                 tr = p.tile_rec[tn];
             } while (tr.y == 0u);
             s_tile = tn;
@@ -1013,34 +995,9 @@ __device__ __forceinline__ void deep_tiles(const CascadeParams& p, uint8_t* smem
 template <int STEP, bool DEPTH, bool F1 = false>
 __global__ void __launch_bounds__(K2D_THREADS, FD_K2D_CTAS) k_deep1(const __grid_constant__ CascadeParams p) {
     extern __shared__ __align__(1024) uint8_t smem_raw[];
-    deep_tiles<STEP, DEPTH, F1, K2D_THREADS, 0, 0, false>(p, smem_raw);
+    deep_tiles<STEP, DEPTH, F1, K2D_THREADS, 0, 0>(p, smem_raw);
 }
 
-// k_k2r: k_stage1 and k_deep1 as CTA roles of ONE persistent launch.  Every role_div-th CTA is a
-// deep CTA whose two 4-warp halves (named barriers 1 and 2) each consume tiles in the order the
-// stage-1 CTAs publish them (tile_ready, release/acquire), while those tiles' ii planes are still
-// L2-resident, and whose latency-bound stage chains overlap the stage-1 CTAs' dense work on the
-// same SMs.  Deadlock-free: stage-1 CTAs never wait on deep CTAs, and CTAs dispatch in blockIdx
-// order, so stage-1 CTAs are resident before any deep CTA can wait for them.
-constexpr size_t k2r_half_bytes(int step) {
-    return (step == 1 ? TileGeoD<1>::SMEM : step == 2 ? TileGeoD<2>::SMEM : step == 3 ? TileGeoD<3>::SMEM
-                                                                                          : TileGeoD<4>::SMEM) +
-           1023 & ~(size_t)1023;
-}
-template <int STEP, bool DEPTH>
-__global__ void __launch_bounds__(k2_threads(STEP), 3) k_k2r(const __grid_constant__ CascadeParams p) {
-    extern __shared__ __align__(1024) uint8_t smem_raw[];
-    static_assert(K2D_THREADS == 128 && k2_threads(STEP) == 256, "two 4-warp deep halves per deep CTA");
-    static_assert(2 * k2r_half_bytes(STEP) <= TileGeoA<STEP>::SMEM, "deep halves fit the stage-1 layout");
-    if ((int)(blockIdx.x % (unsigned)p.role_div) == p.role_div - 1) {
-        if (threadIdx.x < 128)
-            deep_tiles<STEP, DEPTH, false, 128, 0, 1, true>(p, smem_raw);
-        else
-            deep_tiles<STEP, DEPTH, false, 128, 128, 2, true>(p, smem_raw + k2r_half_bytes(STEP));
-    } else {
-        stage1_tiles<STEP, DEPTH>(p, smem_raw);
-    }
-}
 
 // k_f1: persistent over every (frame, level, tile) of a frame group, like k_cascade, with the
 // tile's planes built in shared memory (above) instead of TMA'd from a global integral:

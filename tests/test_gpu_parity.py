@@ -137,9 +137,6 @@ K2_SCHEDULES = {
     "split_two_slot": {"FD_GROUP_FRAMES": "1"},             # 3 frame groups over 2 slots/streams
     "split_one_slot": {"FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
     "fused_k1": {"FD_K2_SPLIT": "0"},                       # K1 -> k_cascade -> k_tail
-    "k2r": {"FD_K2R": "1"},                                 # k_stage1 + k_deep1 as CTA roles of one launch
-    "k2r_div2": {"FD_K2R": "1", "FD_K2R_DIV": "2"},
-    "k2r_two_slot": {"FD_K2R": "1", "FD_GROUP_FRAMES": "1"},
     "f1": {"FD_F1": "1"},                                   # k_level -> k_f1 -> k_deep1<F1> -> k_tail
     "f1_no_tail": {"FD_F1": "1", "FD_TAIL": "0"},
     "f1_tail_early": {"FD_F1": "1", "FD_TAIL_N": "200"},    # most deep windows through k_tail (u8 rebuild)
