@@ -63,18 +63,10 @@ struct TileGeo {
     static constexpr int CP = NW;                                       // pool capacity (a whole tile)
     static constexpr int QBUF = ((PBUF > NW * 10 / 4 ? PBUF : NW * 10 / 4) + 31) & ~31;
     static constexpr size_t OFF_Q = (size_t)PBUF * 4;
-#ifdef FD_POOL_SEPARATE
-    static constexpr size_t OFF_NF = OFF_Q + (size_t)QBUF * 4;
-#else
     static constexpr size_t OFF_NF = OFF_Q;                             // pool in the sqii buffer
-#endif
     static constexpr size_t OFF_LOC = OFF_NF + (size_t)NW * 4;
     static constexpr size_t OFF_LIST = OFF_LOC + (size_t)NW * 2;
-#ifdef FD_POOL_SEPARATE
-    static constexpr size_t OFF_RED = OFF_LIST + (size_t)NW * 4;
-#else
     static constexpr size_t OFF_RED = OFF_Q + (size_t)QBUF * 4;
-#endif
     static constexpr size_t SMEM = OFF_RED + (size_t)k2_threads(STEP) * 8;   // + split-stump partial sums
 };
 #ifndef FD_K2_CTAS

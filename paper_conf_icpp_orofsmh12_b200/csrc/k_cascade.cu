@@ -20,6 +20,10 @@
 //     (one stump per lane) and the leaves are added in stump order;
 //   * fp32 arithmetic matches the oracle bit for bit: __fmul_rn/__fadd_rn (no FMA
 //     contraction), __int2float_rn, __ll2float_rn, IEEE __fsqrt_rn.
+// Kernels: k_stage1 + k_deep1 (default schedule, split at stage 2), k_cascade (fused, all stages
+// in one CTA), k_f1 (+ k_deep1<F1>: SURVEY 8(f) f1, tile-local integrals built in shared memory).
+// This file is also compiled at run time by NVRTC with the cascade's specialised stages
+// (fd_jit.cpp: FD_JIT_STAGE1, FD_JIT_DEEP, FD_PACKED_WORDS).
 #include "k_common.cuh"
 
 namespace fdk {

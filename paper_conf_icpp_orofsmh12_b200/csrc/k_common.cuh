@@ -1,4 +1,4 @@
-// k_common.cuh -- device helpers shared by the K2 cascade kernels (k_cascade.cu, k_cascade_ws.cu):
+// k_common.cuh -- device helpers shared by the K2 cascade kernels (k_cascade.cu, k_tail.cu, k_soft.cu):
 // mbarrier / TMA wrappers, stump-record accessors and the exact stump / stage evaluators
 // (oracle c7/c8: (float)f < theta*nf ? left : right, fp32 stage sums in stump order, no FMA).
 #pragma once
