@@ -605,7 +605,7 @@ struct DevBuf {
 // between two such slots on two streams, so K1 of group g+1 overlaps the latency-bound deep
 // stages and tail of group g (different resources: HBM vs issue/latency).
 struct PipeSlot {
-    DevBuf ws, colbuf, rowbuf, corbuf, lvlbuf, tmaps, tailq, surv, tilerec;
+    DevBuf ws, colbuf, rowbuf, corbuf, lvlbuf, tmaps, tailq, surv, tilerec, tlist;
     // K1 scratch for g frames of plan p
     cudaError_t k1_scratch(const PlanDev& p, int g, K1Scratch* s) {
         cudaError_t e = colbuf.ensure((size_t)g * p.col_frame * 4 + 16);
@@ -702,9 +702,12 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     const bool f1_split = f1 && env_int("FD_F1_SPLIT", 1) != 0;
     const bool split = !queue && !f1 && env_int("FD_K2_SPLIT", 1) != 0;
     const bool surv = split || f1_split;
+    // split K2 deep stages: k_deep1 (CTA per tile, stage-synchronous) + k_tail, or FD_DEEPQ=1:
+    // k_deepq (warp-autonomous batches over a per-SM tile pool, no tail hand-off)
+    const bool deepq = split && env_int("FD_DEEPQ", 0) != 0;
     // tail queue (k_tail): FD_TAIL=0 keeps every window inside K2; FD_TAIL_N = windows left in a
     // batch at which it hands them over; FD_TAIL_CAP = queue entries (16 B each) per group
-    const bool use_tail = !queue && env_int("FD_TAIL", 1) != 0;
+    const bool use_tail = !queue && !deepq && env_int("FD_TAIL", 1) != 0;
     const int tail_cap = use_tail ? std::max(1024, env_int("FD_TAIL_CAP", 1 << 22)) : 0;
     // frames per group: one K2 launch per group.  f1: the group's level images (12.5 MB per 1080p
     // frame) should stay L2-resident between k_level and k_f1 (FD_F1_GROUP_MB, default 64 MB);
@@ -734,6 +737,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
             CK(sl.surv.ensure((size_t)G * (size_t)PD.win_per_frame * 8 + 16));
             CK(sl.tilerec.ensure((size_t)G * PD.tiles_per_frame * 8 + 16));
         }
+        if (deepq) CK(sl.tlist.ensure((size_t)G * PD.tiles_per_frame * 16 + 16));
         if (f1) {
             CK(sl.ws.ensure((size_t)PD.u8_bytes + 16));
             s = encode_maps8(PD, sl.ws.as<uint8_t>(), step, maps.data());
@@ -751,9 +755,9 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
                            cudaMemcpyHostToDevice, st));
     }
     // ctl: [0] detection count, [256 B..] per-group K2 tile counters, then per-group tail counts,
-    // survivor counts and k_deep1 tile counters
-    CK(w->ctl.ensure(256 + (size_t)ngroups * 16));
-    CK(cudaMemsetAsync(w->ctl.p, 0, 256 + (size_t)ngroups * 16, st));
+    // survivor counts, deep-kernel tile counters and tile-list counts
+    CK(w->ctl.ensure(256 + (size_t)ngroups * 20));
+    CK(cudaMemsetAsync(w->ctl.p, 0, 256 + (size_t)ngroups * 20, st));
     if (!depth) {
         const size_t cap = (size_t)(det_cap > 0 ? det_cap : 1);
         CK(w->keys.ensure(cap * 8));
@@ -873,6 +877,8 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         P.tail_count = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + ngroups + gi;
         P.surv_count = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + 2 * ngroups + gi;
         P.deep_counter = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + 3 * ngroups + gi;
+        P.tile_list_count = reinterpret_cast<unsigned int*>(w->ctl.as<char>() + 256) + 4 * ngroups + gi;
+        P.tile_list = deepq ? sl.tlist.as<uint4>() : nullptr;
         P.surv = surv ? sl.surv.as<uint2>() : nullptr;
         P.tile_rec = surv ? sl.tilerec.as<uint2>() : nullptr;
         const int gr = grid < P.total_tiles ? grid : P.total_tiles;
@@ -887,7 +893,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
             }
             if (e == cudaSuccess && surv) {
                 ProfScope ps(FD_K_DEEP, gs);
-                e = jit_k2_launch(jit, P, depth, f1 ? JIT_DEEP1_F1 : JIT_DEEP1, gs, &err);
+                e = jit_k2_launch(jit, P, depth, f1 ? JIT_DEEP1_F1 : (deepq ? JIT_DEEPQ : JIT_DEEP1), gs, &err);
             }
             if (e != cudaSuccess)
                 return fail(FD_ECUDA, "specialised K2: %s", err.empty() ? cudaGetErrorString(e) : err.c_str());
@@ -896,7 +902,10 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
             if (f1_split) LAUNCH(FD_K_DEEP, gs, launch_deep1(P, depth, step, true, gs));
         } else if (split) {
             LAUNCH(FD_K_CASCADE, gs, launch_stage1(P, depth, step, gs));
-            LAUNCH(FD_K_DEEP, gs, launch_deep1(P, depth, step, false, gs));
+            if (deepq)
+                LAUNCH(FD_K_DEEP, gs, launch_deepq(P, depth, step, gs));
+            else
+                LAUNCH(FD_K_DEEP, gs, launch_deep1(P, depth, step, false, gs));
         } else {
             LAUNCH(FD_K_CASCADE, gs, launch_cascade(P, depth, step, gr, gs));
         }

@@ -134,6 +134,39 @@ struct TileGeoD {
     static constexpr size_t SMEM = F1 ? OFF_U8 + (size_t)TileGeoF<STEP>::UB : OFF_U8;
 };
 
+// k_deepq (K2b, k_deepq.cuh): one persistent CTA per SM; tile slots (ii planes via TMA) as many as
+// fit next to the per-stage window rings (DQ_QC entries + sequence words for stages
+// s0+1 .. s0+DQ_NQ) and a 32-entry staging row per warp
+#ifndef FD_DQ_WARPS
+#define FD_DQ_WARPS 16
+#endif
+#ifndef FD_DQ_SLOTS
+#define FD_DQ_SLOTS 10
+#endif
+constexpr int DQ_THREADS = FD_DQ_WARPS * 32;
+constexpr int DQ_NQ = 24;
+constexpr int DQ_QC = 64;                   // power of two
+constexpr size_t DQ_SMEM_MAX = 225 * 1024;  // dynamic shared memory budget (static: < 2 KB)
+__host__ __device__ constexpr size_t dq_fixed(int warps) { return (size_t)DQ_NQ * DQ_QC * 12 + (size_t)warps * 32 * 8; }
+__host__ __device__ constexpr int dq_slots(int step, int slots, int warps) {
+    return slots < (int)((DQ_SMEM_MAX - dq_fixed(warps)) / ((size_t)k2_pbuf(step) * 4))
+               ? slots
+               : (int)((DQ_SMEM_MAX - dq_fixed(warps)) / ((size_t)k2_pbuf(step) * 4));
+}
+__host__ __device__ constexpr size_t dq_smem(int step, int slots, int warps) {
+    return (size_t)dq_slots(step, slots, warps) * k2_pbuf(step) * 4 + dq_fixed(warps);
+}
+template <int STEP>
+struct TileGeoQ {
+    static constexpr int NS = dq_slots(STEP, FD_DQ_SLOTS, FD_DQ_WARPS);   // tile slots
+    static constexpr int PBUF = k2_pbuf(STEP);
+    static constexpr size_t OFF_Q = (size_t)NS * PBUF * 4;                 // uint2 [DQ_NQ][DQ_QC] entries
+    static constexpr size_t OFF_SEQ = OFF_Q + (size_t)DQ_NQ * DQ_QC * 8;    // int [DQ_NQ][DQ_QC] cell sequence
+    static constexpr size_t OFF_STG = OFF_SEQ + (size_t)DQ_NQ * DQ_QC * 4;  // uint2 [warps][32]
+    static constexpr size_t SMEM = OFF_STG + (size_t)FD_DQ_WARPS * 32 * 8;
+    static_assert(NS >= 1 && NS <= 32 && SMEM == dq_smem(STEP, FD_DQ_SLOTS, FD_DQ_WARPS), "k_deepq layout");
+};
+
 struct LevelDev {
     int W, H, P;            // level size, ii pitch (elements)
     int PB;                 // f1: u8 level-image pitch (bytes, 16-B multiple >= P)
@@ -220,6 +253,8 @@ struct alignas(16) CascadeParams {
     uint2* tile_rec;                        // split K2: per tile (offset into surv, count)
     unsigned int* surv_count;
     unsigned int* deep_counter;             // k_deep tile claims
+    uint4* tile_list;                       // split K2: tiles with stage-s0 survivors {tile, offset, count, 0} (k_deepq)
+    unsigned int* tile_list_count;
     StageDev pstages[PSTAGE_MAX];
     uint4 prec[PREC_MAX * (REC_WORDS / 4)];
 };
@@ -287,6 +322,7 @@ cudaError_t launch_tail(const TailParams& p, bool depth_mode, cudaStream_t st);
 // split K2: k_stage1 then k_deep (precompiled kernels; step 1 normally runs the NVRTC ones)
 cudaError_t launch_stage1(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
 cudaError_t launch_deep1(const CascadeParams& p, bool depth_mode, int step, bool f1, cudaStream_t st);
+cudaError_t launch_deepq(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);   // k_deepq.cuh
 cudaError_t launch_soft(const CascadeParams& p, bool depth_mode, int step, bool soft, cudaStream_t st);  // k_soft.cu (R8b)
 cudaError_t launch_depth_hist(const uint8_t* depth, int n, long long win_per_frame, const long long* d_win0,
                               int n_levels, int n_stages, long long* hist, int max_span, cudaStream_t st);

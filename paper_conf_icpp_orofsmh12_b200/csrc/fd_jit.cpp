@@ -178,6 +178,16 @@ static int jit_deep_threads() {
     return env_or("FD_K2D_THREADS", FD_K2D_THREADS) <= 64 ? 64 : 128;
 }
 
+// k_deepq geometry of the generated program (FD_DQ_SLOTS tile slots, FD_DQ_WARPS warps)
+static int jit_dq_slots() {
+    const int v = env_or("FD_DQ_SLOTS", FD_DQ_SLOTS);
+    return v < 1 ? 1 : (v > 32 ? 32 : v);
+}
+static int jit_dq_warps() {
+    const int v = env_or("FD_DQ_WARPS", FD_DQ_WARPS);
+    return v < 1 ? 1 : (v > 32 ? 32 : v);
+}
+
 // resident CTAs per SM targeted by the fused kernel's launch bounds (FD_K2_CTAS, 2..6)
 static int jit_ctas() {
     const int c = env_or("FD_K2_CTAS", FD_K2_CTAS);
@@ -199,6 +209,8 @@ std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_sta
                       "\n#define FD_K2D_THREADS " + std::to_string(jit_deep_threads()) +
                       "\n#define FD_F1_CTAS " + std::to_string(env_or("FD_F1_CTAS", FD_F1_CTAS)) +
                       "\n#define FD_K2_CTAS " + std::to_string(jit_ctas()) +
+                      "\n#define FD_DQ_SLOTS " + std::to_string(jit_dq_slots()) +
+                      "\n#define FD_DQ_WARPS " + std::to_string(jit_dq_warps()) +
                       "\n#include \"fd_internal.h\"\n" + jit_stage1_source(rec_words, st[0].first, st[0].n) +
                       "#define FD_JIT_STAGE1 1\n";
     if (k_end > 1) src += jit_deep_source(rec_words, st, k_end) + "#define FD_JIT_DEEP " + std::to_string(k_end) + "\n";
@@ -211,6 +223,7 @@ static std::string jit_name(int kind, bool depth) {
     if (kind == JIT_STAGE1) return "fdk::k_stage1<1, " + d + ">";
     if (kind == JIT_DEEP1) return "fdk::k_deep1<1, " + d + ", false>";
     if (kind == JIT_DEEP1_F1) return "fdk::k_deep1<1, " + d + ", true>";
+    if (kind == JIT_DEEPQ) return "fdk::k_deepq<1, " + d + ">";
     return "fdk::k_f1<1, " + d + ">";
 }
 
@@ -222,6 +235,10 @@ static KindGeo jit_kind_geo(int kind) {
     if (kind == JIT_DEEP1) g.smem = TileGeoD<JIT_STEP, false>::SMEM;
     if (kind == JIT_DEEP1_F1) g.smem = TileGeoD<JIT_STEP, true>::SMEM;
     if (kind == JIT_F1) g.smem = TileGeoF<JIT_STEP>::SMEM;
+    if (kind == JIT_DEEPQ) {
+        g.threads = jit_dq_warps() * 32;
+        g.smem = dq_smem(JIT_STEP, jit_dq_slots(), jit_dq_warps());
+    }
     // FD_S1_GRID / FD_DEEP_GRID: cap the persistent grids of k_stage1 / k_deep1 at that many CTAs
     // per SM, so the other pipeline slot's kernels can co-reside
     if (kind == JIT_STAGE1) g.grid_per_sm = env_or("FD_S1_GRID", 0);
@@ -231,10 +248,11 @@ static KindGeo jit_kind_geo(int kind) {
 
 bool jit_k2_compile(const std::string& source, bool depth, std::vector<char>* cubin, std::vector<std::string>* lowered,
                     std::string* err) {
-    const char* hdr_src[] = {jit_src_fd_h, jit_src_fd_internal_h, jit_src_k_common_cuh, jit_src_k_cascade_cu};
-    const char* hdr_names[] = {"fd.h", "fd_internal.h", "k_common.cuh", "k_cascade.cu"};
+    const char* hdr_src[] = {jit_src_fd_h, jit_src_fd_internal_h, jit_src_k_common_cuh, jit_src_k_cascade_cu,
+                             jit_src_k_deepq_cuh};
+    const char* hdr_names[] = {"fd.h", "fd_internal.h", "k_common.cuh", "k_cascade.cu", "k_deepq.cuh"};
     nvrtcProgram prog = nullptr;
-    if (nvrtcCreateProgram(&prog, source.c_str(), "k_cascade_jit.cu", 4, hdr_src, hdr_names) != NVRTC_SUCCESS) {
+    if (nvrtcCreateProgram(&prog, source.c_str(), "k_cascade_jit.cu", 5, hdr_src, hdr_names) != NVRTC_SUCCESS) {
         *err = "nvrtcCreateProgram failed";
         return false;
     }

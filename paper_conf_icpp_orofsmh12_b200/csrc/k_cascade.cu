@@ -701,7 +701,12 @@ __device__ __forceinline__ void stage1_tiles(const CascadeParams& p, uint8_t* sm
         if (tid == 0) {
             // the previous tile's record; its counters are reset for the tile after this one (a
             // barrier separates that reset from their next use)
-            if (s_prev >= 0) p.tile_rec[s_prev] = make_uint2((unsigned)s_prev_off, (unsigned)s_c2[b ^ 1]);
+            if (s_prev >= 0) {
+                p.tile_rec[s_prev] = make_uint2((unsigned)s_prev_off, (unsigned)s_c2[b ^ 1]);
+                if (p.tile_list && s_c2[b ^ 1] > 0)      // k_deepq's compact list of tiles with work
+                    p.tile_list[atomicAdd(p.tile_list_count, 1u)] =
+                        make_uint4((unsigned)s_prev, (unsigned)s_prev_off, (unsigned)s_c2[b ^ 1], 0u);
+            }
             s_prev = -1;
             s_c1[b ^ 1] = 0;
             s_c2[b ^ 1] = 0;
@@ -1187,7 +1192,15 @@ __global__ void __launch_bounds__(k2_threads(STEP), FD_F1_CTAS) k_f1(const __gri
     }
 }
 
+}  // namespace fdk
+#include "k_deepq.cuh"
+namespace fdk {
+
 #ifndef __CUDACC_RTC__
+// ------------------------------------------------------------------ host launchers
+// build.py compiles this file once per window step (-DFD_KC_STEP=1..4, in parallel): each object
+// instantiates only its own step's kernels (StepLaunch<FD_KC_STEP>), and the step-1 object also
+// holds the dispatchers over the step.  Without FD_KC_STEP every step is instantiated here.
 template <int STEP, bool DEPTH>
 static cudaError_t launch_one(const CascadeParams& p, int grid, cudaStream_t st) {
     const size_t smem = TileGeo<STEP>::SMEM;
@@ -1209,40 +1222,6 @@ static int grid_step() {
 }
 
 template <int STEP, bool DEPTH>
-static cudaError_t launch_step(const CascadeParams& p, int grid, cudaStream_t st) {
-    return launch_one<STEP, DEPTH>(p, grid, st);
-}
-
-size_t cascade_smem(int step) {
-    switch (step) {
-        case 1: return TileGeo<1>::SMEM;
-        case 2: return TileGeo<2>::SMEM;
-        case 3: return TileGeo<3>::SMEM;
-        default: return TileGeo<4>::SMEM;
-    }
-}
-
-int cascade_grid(bool depth, int step) {
-    switch (step) {
-        case 1: return depth ? grid_step<1, true>() : grid_step<1, false>();
-        case 2: return depth ? grid_step<2, true>() : grid_step<2, false>();
-        case 3: return depth ? grid_step<3, true>() : grid_step<3, false>();
-        default: return depth ? grid_step<4, true>() : grid_step<4, false>();
-    }
-}
-
-cudaError_t launch_cascade(const CascadeParams& p, bool depth, int step, int grid, cudaStream_t st) {
-    switch (step) {
-        case 1: return depth ? launch_step<1, true>(p, grid, st) : launch_step<1, false>(p, grid, st);
-        case 2: return depth ? launch_step<2, true>(p, grid, st) : launch_step<2, false>(p, grid, st);
-        case 3: return depth ? launch_step<3, true>(p, grid, st) : launch_step<3, false>(p, grid, st);
-        case 4: return depth ? launch_step<4, true>(p, grid, st) : launch_step<4, false>(p, grid, st);
-        default: return cudaErrorInvalidValue;
-    }
-}
-
-
-template <int STEP, bool DEPTH>
 static cudaError_t launch_stage1_t(const CascadeParams& p, cudaStream_t st) {
     static int grid = 0;
     const size_t smem = TileGeoA<STEP>::SMEM;
@@ -1259,15 +1238,6 @@ static cudaError_t launch_stage1_t(const CascadeParams& p, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-cudaError_t launch_stage1(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
-    switch (step) {
-        case 1: return depth ? launch_stage1_t<1, true>(p, st) : launch_stage1_t<1, false>(p, st);
-        case 2: return depth ? launch_stage1_t<2, true>(p, st) : launch_stage1_t<2, false>(p, st);
-        case 3: return depth ? launch_stage1_t<3, true>(p, st) : launch_stage1_t<3, false>(p, st);
-        case 4: return depth ? launch_stage1_t<4, true>(p, st) : launch_stage1_t<4, false>(p, st);
-        default: return cudaErrorInvalidValue;
-    }
-}
 
 template <int STEP, bool DEPTH, bool F1>
 static cudaError_t launch_deep1_t(const CascadeParams& p, cudaStream_t st) {
@@ -1286,20 +1256,23 @@ static cudaError_t launch_deep1_t(const CascadeParams& p, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-template <bool F1>
-static cudaError_t launch_deep1_f(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
-    switch (step) {
-        case 1: return depth ? launch_deep1_t<1, true, F1>(p, st) : launch_deep1_t<1, false, F1>(p, st);
-        case 2: return depth ? launch_deep1_t<2, true, F1>(p, st) : launch_deep1_t<2, false, F1>(p, st);
-        case 3: return depth ? launch_deep1_t<3, true, F1>(p, st) : launch_deep1_t<3, false, F1>(p, st);
-        case 4: return depth ? launch_deep1_t<4, true, F1>(p, st) : launch_deep1_t<4, false, F1>(p, st);
-        default: return cudaErrorInvalidValue;
+template <int STEP, bool DEPTH>
+static cudaError_t launch_deepq_t(const CascadeParams& p, cudaStream_t st) {
+    static int grid = 0;
+    const size_t smem = TileGeoQ<STEP>::SMEM;
+    cudaError_t e = cudaFuncSetAttribute(k_deepq<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    if (!grid) {
+        int dev = 0, sms = 0, per = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_deepq<STEP, DEPTH>, DQ_THREADS, smem);
+        grid = sms * (per > 0 ? per : 1);
     }
+    k_deepq<STEP, DEPTH><<<grid, DQ_THREADS, smem, st>>>(p);
+    return cudaGetLastError();
 }
 
-cudaError_t launch_deep1(const CascadeParams& p, bool depth, int step, bool f1, cudaStream_t st) {
-    return f1 ? launch_deep1_f<true>(p, depth, step, st) : launch_deep1_f<false>(p, depth, step, st);
-}
 
 template <int STEP, bool DEPTH>
 static cudaError_t launch_f1_t(const CascadeParams& p, cudaStream_t st) {
@@ -1318,15 +1291,80 @@ static cudaError_t launch_f1_t(const CascadeParams& p, cudaStream_t st) {
     return cudaGetLastError();
 }
 
-cudaError_t launch_f1(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
+
+template <int STEP>
+struct StepLaunch {
+    static cudaError_t cascade(const CascadeParams& p, bool d, int grid, cudaStream_t st) {
+        return d ? launch_one<STEP, true>(p, grid, st) : launch_one<STEP, false>(p, grid, st);
+    }
+    static int grid(bool d) { return d ? grid_step<STEP, true>() : grid_step<STEP, false>(); }
+    static cudaError_t stage1(const CascadeParams& p, bool d, cudaStream_t st) {
+        return d ? launch_stage1_t<STEP, true>(p, st) : launch_stage1_t<STEP, false>(p, st);
+    }
+    static cudaError_t deep1(const CascadeParams& p, bool d, bool f1, cudaStream_t st) {
+        if (f1) return d ? launch_deep1_t<STEP, true, true>(p, st) : launch_deep1_t<STEP, false, true>(p, st);
+        return d ? launch_deep1_t<STEP, true, false>(p, st) : launch_deep1_t<STEP, false, false>(p, st);
+    }
+    static cudaError_t deepq(const CascadeParams& p, bool d, cudaStream_t st) {
+        return d ? launch_deepq_t<STEP, true>(p, st) : launch_deepq_t<STEP, false>(p, st);
+    }
+    static cudaError_t f1(const CascadeParams& p, bool d, cudaStream_t st) {
+        return d ? launch_f1_t<STEP, true>(p, st) : launch_f1_t<STEP, false>(p, st);
+    }
+};
+
+#ifdef FD_KC_STEP
+template struct StepLaunch<FD_KC_STEP>;
+#endif
+
+#if !defined(FD_KC_STEP) || FD_KC_STEP == 1
+#ifdef FD_KC_STEP
+extern template struct StepLaunch<2>;
+extern template struct StepLaunch<3>;
+extern template struct StepLaunch<4>;
+#endif
+#define FD_STEP_SWITCH(step, call)                   \
+    switch (step) {                                   \
+        case 1: return StepLaunch<1>::call;           \
+        case 2: return StepLaunch<2>::call;           \
+        case 3: return StepLaunch<3>::call;           \
+        case 4: return StepLaunch<4>::call;           \
+        default: return cudaErrorInvalidValue;        \
+    }
+
+size_t cascade_smem(int step) {
     switch (step) {
-        case 1: return depth ? launch_f1_t<1, true>(p, st) : launch_f1_t<1, false>(p, st);
-        case 2: return depth ? launch_f1_t<2, true>(p, st) : launch_f1_t<2, false>(p, st);
-        case 3: return depth ? launch_f1_t<3, true>(p, st) : launch_f1_t<3, false>(p, st);
-        case 4: return depth ? launch_f1_t<4, true>(p, st) : launch_f1_t<4, false>(p, st);
-        default: return cudaErrorInvalidValue;
+        case 1: return TileGeo<1>::SMEM;
+        case 2: return TileGeo<2>::SMEM;
+        case 3: return TileGeo<3>::SMEM;
+        default: return TileGeo<4>::SMEM;
     }
 }
+int cascade_grid(bool depth, int step) {
+    switch (step) {
+        case 1: return StepLaunch<1>::grid(depth);
+        case 2: return StepLaunch<2>::grid(depth);
+        case 3: return StepLaunch<3>::grid(depth);
+        default: return StepLaunch<4>::grid(depth);
+    }
+}
+cudaError_t launch_cascade(const CascadeParams& p, bool depth, int step, int grid, cudaStream_t st) {
+    FD_STEP_SWITCH(step, cascade(p, depth, grid, st))
+}
+cudaError_t launch_stage1(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
+    FD_STEP_SWITCH(step, stage1(p, depth, st))
+}
+cudaError_t launch_deep1(const CascadeParams& p, bool depth, int step, bool f1, cudaStream_t st) {
+    FD_STEP_SWITCH(step, deep1(p, depth, f1, st))
+}
+cudaError_t launch_deepq(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
+    FD_STEP_SWITCH(step, deepq(p, depth, st))
+}
+cudaError_t launch_f1(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
+    FD_STEP_SWITCH(step, f1(p, depth, st))
+}
+#undef FD_STEP_SWITCH
+#endif
 
 #endif  // !__CUDACC_RTC__
 

@@ -130,12 +130,16 @@ def test_depth_maps_generic_k2(monkeypatch):
 K2_SCHEDULES = {
     "split_default": {},                                    # K1 -> k_stage1 -> k_deep1 -> k_tail
     "split_s0_1": {"FD_S0": "1"},                           # k_stage1 stage 1 only
-    "split_no_tail": {"FD_TAIL": "0"},                      # k_deep1 finishes every window
-    "split_split_stump": {"FD_DEEP_SPLIT": "64"},           # deep stages <= 64 windows split-stump
-    "split_deep_2warps": {"FD_K2D_THREADS": "64"},          # two-warp k_deep1 blocks
-    "split_s_tail_3": {"FD_S_TAIL": "3"},                   # every window alive at stage 3 through k_tail
     "split_two_slot": {"FD_GROUP_FRAMES": "1"},             # 3 frame groups over 2 slots/streams
     "split_one_slot": {"FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
+    "deepq": {"FD_DEEPQ": "1"},                             # K1 -> k_stage1 -> k_deepq
+    "deepq_s0_1": {"FD_DEEPQ": "1", "FD_S0": "1"},
+    "deepq_two_slot": {"FD_DEEPQ": "1", "FD_GROUP_FRAMES": "1"},
+    "deepq_2_slots": {"FD_DEEPQ": "1", "FD_DQ_SLOTS": "2", "FD_DQ_WARPS": "4"},   # slot reuse / pinning pressure (JIT only)
+    "deep1_no_tail": {"FD_DEEPQ": "0", "FD_TAIL": "0"},     # k_deep1 finishes every window
+    "deep1_split_stump": {"FD_DEEPQ": "0", "FD_DEEP_SPLIT": "64"},   # deep stages <= 64 windows split-stump
+    "deep1_2warps": {"FD_DEEPQ": "0", "FD_K2D_THREADS": "64"},       # two-warp k_deep1 blocks
+    "deep1_s_tail_3": {"FD_DEEPQ": "0", "FD_S_TAIL": "3"},  # every window alive at stage 3 through k_tail
     "fused_k1": {"FD_K2_SPLIT": "0"},                       # K1 -> k_cascade -> k_tail
     "f1": {"FD_F1": "1"},                                   # k_level -> k_f1 -> k_deep1<F1> -> k_tail
     "f1_no_tail": {"FD_F1": "1", "FD_TAIL": "0"},
@@ -150,15 +154,22 @@ K2_SCHEDULES = {
 }
 
 
+# variables read when a cascade's specialised program is generated (once per fd.Cascade)
+JIT_GEOMETRY_ENV = {"FD_DQ_SLOTS", "FD_DQ_WARPS", "FD_K2D_THREADS", "FD_K2D_CTAS", "FD_K2_CTAS", "FD_F1_CTAS"}
+
+
 @pytest.mark.parametrize("jit", ["1", "0"])
 @pytest.mark.parametrize("name", sorted(K2_SCHEDULES))
 def test_k2_schedules(name, jit, monkeypatch):
     for k, v in K2_SCHEDULES[name].items():
         monkeypatch.setenv(k, v)
     monkeypatch.setenv("FD_JIT", jit)
+    pair = cascades(2)
+    if jit == "1" and JIT_GEOMETRY_ENV & set(K2_SCHEDULES[name]):
+        pair = (fd.Cascade(open(os.path.join(ROOT, "cascades", "c2.fdc")).read()), pair[1])
     fr, _ = gen(2, 5, 3)
-    compare_depth(cascades(2), fr, 1.2)
-    gc, oc = cascades(2)
+    compare_depth(pair, fr, 1.2)
+    gc, oc = pair
     got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, 1.2, 1, capacity=1 << 20))
     ref, _ = oracle.detect(oc, fr, 24, 1.2, 1, nthreads=os.cpu_count())
     assert np.array_equal(got, ref)
@@ -448,6 +459,25 @@ def test_all_pass_and_all_reject():
     d, sc = fd.fd_detect_depth(allrej, torch.from_numpy(fr).cuda(), 24, s, 1)
     assert (d.cpu().numpy() == 0).all() and (sc.cpu().numpy() == 0.5).all()
     assert len(fd.fd_detect(allrej, torch.from_numpy(fr).cuda(), 24, s, 1)) == 0
+
+
+@pytest.mark.parametrize("env", [{}, {"FD_DEEPQ": "1"}, {"FD_DEEPQ": "1", "FD_JIT": "0"},
+                                 {"FD_DEEPQ": "1", "FD_DQ_SLOTS": "2", "FD_DQ_WARPS": "4"}])
+def test_all_pass_deep(env, monkeypatch):
+    """Every window survives every stage of a 7-stage cascade: k_deepq's queues overflow (2048
+    windows per tile), batches stay full through every deep stage, slots are reused only after
+    all of their windows are emitted.  Detections and depth maps equal the oracle's."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    st = ([(1, 1, 10, 10, -1), (1, 1, 5, 10, 2)], 0.1, 0.5, 0.25)
+    text = _casc_text([("-1e30", [st] * (1 + i % 3)) for i in range(7)])
+    W, H, s = 301, 203, 1.2
+    fr = np.stack([fdgen.background(2, 80 + i, W, H) for i in range(3)])
+    tot = sum(p[3] for p in oracle.plan(W, H, 24, s, 1))
+    got = fd.to_numpy(fd.fd_detect(fd.Cascade(text), torch.from_numpy(fr).cuda(), 24, s, 1, capacity=3 * tot))
+    ref, _ = oracle.detect(oracle.Cascade(text), fr, 24, s, 1, nthreads=os.cpu_count())
+    assert len(got) == 3 * tot and np.array_equal(got, ref)
+    compare_depth((fd.Cascade(text), oracle.Cascade(text)), fr, s)
 
 
 def test_worked_example_single_stump():
