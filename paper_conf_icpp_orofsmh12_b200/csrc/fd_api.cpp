@@ -705,9 +705,12 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     // split K2 deep stages: k_deep1 (CTA per tile, stage-synchronous) + k_tail, or FD_DEEPQ=1:
     // k_deepq (warp-autonomous batches over a per-SM tile pool, no tail hand-off)
     const bool deepq = split && env_int("FD_DEEPQ", 0) != 0;
+    // k_deepq hands every window that enters stage FD_DQ_TAIL to k_tail (long chains would hold
+    // their tile's slot); 255 = never
+    const int dq_tail = std::max(1, env_int("FD_DQ_TAIL", 7));
     // tail queue (k_tail): FD_TAIL=0 keeps every window inside K2; FD_TAIL_N = windows left in a
     // batch at which it hands them over; FD_TAIL_CAP = queue entries (16 B each) per group
-    const bool use_tail = !queue && !deepq && env_int("FD_TAIL", 1) != 0;
+    const bool use_tail = !queue && env_int("FD_TAIL", 1) != 0 && (!deepq || dq_tail < (int)c->stages.size());
     const int tail_cap = use_tail ? std::max(1024, env_int("FD_TAIL_CAP", 1 << 22)) : 0;
     // frames per group: one K2 launch per group.  f1: the group's level images (12.5 MB per 1080p
     // frame) should stay L2-resident between k_level and k_f1 (FD_F1_GROUP_MB, default 64 MB);
@@ -794,7 +797,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     P.tail_n = std::max(1, env_int("FD_TAIL_N", 8));
     // FD_S_TAIL: every window still alive at this stage is handed to k_tail (default: none, only
     // the FD_TAIL_N rule)
-    P.s_tail = std::max(1, env_int("FD_S_TAIL", 255));
+    P.s_tail = deepq ? dq_tail : std::max(1, env_int("FD_S_TAIL", 255));
     // deep stages with at most FD_DEEP_SPLIT windows (<= 64; default 0 = off) run split-stump
     P.split_max = std::max(0, env_int("FD_DEEP_SPLIT", 0));
     // k_stage1 runs stages [0, s0) (FD_S0 = 2, default, or 1); the fused kernels start their
@@ -811,7 +814,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     // stage 1 on, FD_TAIL_SMEM_STUMPS budget, default 256 stumps = 16 KB)
     {
         const int budget = std::max(0, env_int("FD_TAIL_SMEM_STUMPS", 256));
-        const int s1 = c->stages.size() > 1 ? 1 : 0;
+        const int s1 = std::min((int)c->stages.size() - 1, deepq ? dq_tail : 1);
         TP.j0 = c->stages[s1].first;
         int k = s1, m = 0;
         while (k < (int)c->stages.size() && m + c->stages[k].n <= budget) m += c->stages[k++].n;

@@ -134,9 +134,9 @@ struct TileGeoD {
     static constexpr size_t SMEM = F1 ? OFF_U8 + (size_t)TileGeoF<STEP>::UB : OFF_U8;
 };
 
-// k_deepq (K2b, k_deepq.cuh): one persistent CTA per SM; tile slots (ii planes via TMA) as many as
-// fit next to the per-stage window rings (DQ_QC entries + sequence words for stages
-// s0+1 .. s0+DQ_NQ) and a 32-entry staging row per warp
+// k_deepq (K2b, k_deepq.cuh): one persistent CTA per SM; as many tile slots as fit -- each the
+// tile's ii plane (TMA) and its first DQ_CAPF stage-s0 survivors -- and a 32-entry staging row
+// per warp
 #ifndef FD_DQ_WARPS
 #define FD_DQ_WARPS 16
 #endif
@@ -144,25 +144,23 @@ struct TileGeoD {
 #define FD_DQ_SLOTS 10
 #endif
 constexpr int DQ_THREADS = FD_DQ_WARPS * 32;
-constexpr int DQ_NQ = 24;
-constexpr int DQ_QC = 64;                   // power of two
-constexpr size_t DQ_SMEM_MAX = 225 * 1024;  // dynamic shared memory budget (static: < 2 KB)
-__host__ __device__ constexpr size_t dq_fixed(int warps) { return (size_t)DQ_NQ * DQ_QC * 12 + (size_t)warps * 32 * 8; }
+constexpr int DQ_CAPF = 224;                // survivors per slot kept in shared memory (the rest read from HBM)
+constexpr size_t DQ_SMEM_MAX = 225 * 1024;  // dynamic shared memory budget (static: < 1 KB)
+__host__ __device__ constexpr size_t dq_slot_bytes(int step) { return (size_t)k2_pbuf(step) * 4 + (size_t)DQ_CAPF * 8; }
 __host__ __device__ constexpr int dq_slots(int step, int slots, int warps) {
-    return slots < (int)((DQ_SMEM_MAX - dq_fixed(warps)) / ((size_t)k2_pbuf(step) * 4))
+    return slots < (int)((DQ_SMEM_MAX - (size_t)warps * 256) / dq_slot_bytes(step))
                ? slots
-               : (int)((DQ_SMEM_MAX - dq_fixed(warps)) / ((size_t)k2_pbuf(step) * 4));
+               : (int)((DQ_SMEM_MAX - (size_t)warps * 256) / dq_slot_bytes(step));
 }
 __host__ __device__ constexpr size_t dq_smem(int step, int slots, int warps) {
-    return (size_t)dq_slots(step, slots, warps) * k2_pbuf(step) * 4 + dq_fixed(warps);
+    return (size_t)dq_slots(step, slots, warps) * dq_slot_bytes(step) + (size_t)warps * 256;
 }
 template <int STEP>
 struct TileGeoQ {
     static constexpr int NS = dq_slots(STEP, FD_DQ_SLOTS, FD_DQ_WARPS);   // tile slots
     static constexpr int PBUF = k2_pbuf(STEP);
-    static constexpr size_t OFF_Q = (size_t)NS * PBUF * 4;                 // uint2 [DQ_NQ][DQ_QC] entries
-    static constexpr size_t OFF_SEQ = OFF_Q + (size_t)DQ_NQ * DQ_QC * 8;    // int [DQ_NQ][DQ_QC] cell sequence
-    static constexpr size_t OFF_STG = OFF_SEQ + (size_t)DQ_NQ * DQ_QC * 4;  // uint2 [warps][32]
+    static constexpr size_t OFF_F = (size_t)NS * PBUF * 4;                 // uint2 [NS][DQ_CAPF] survivors
+    static constexpr size_t OFF_STG = OFF_F + (size_t)NS * DQ_CAPF * 8;     // uint2 [warps][32]
     static constexpr size_t SMEM = OFF_STG + (size_t)FD_DQ_WARPS * 32 * 8;
     static_assert(NS >= 1 && NS <= 32 && SMEM == dq_smem(STEP, FD_DQ_SLOTS, FD_DQ_WARPS), "k_deepq layout");
 };

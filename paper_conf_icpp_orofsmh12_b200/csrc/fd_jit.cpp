@@ -127,11 +127,11 @@ std::string jit_stage1_source(const uint32_t* rec_words, int first, int n) {
     return o.str();
 }
 
-std::string jit_deep_source(const uint32_t* rec_words, const StageDev* st, int k_end) {
+std::string jit_deep_source(const uint32_t* rec_words, const StageDev* st, int k_end, const char* name) {
     constexpr int TW = tile_w(JIT_STEP);
     std::ostringstream o;
     o << "namespace fdk {\n"
-      << "__device__ __forceinline__ float jit_deep(int s, const uint32_t* __restrict__ T, float nf) {\n"
+      << "__device__ __forceinline__ float " << name << "(int s, const uint32_t* __restrict__ T, float nf) {\n"
       << "  float sum = 0.0f;\n  switch (s) {\n";
     for (int s = 1; s < k_end; ++s) {
         o << "  case " << s << ":\n";
@@ -160,9 +160,8 @@ std::string jit_deep_source(const uint32_t* rec_words, const StageDev* st, int k
     return o.str();
 }
 
-int jit_deep_end(const StageDev* st, int n_stages) {
-    int budget = 60;                                   // generated deep stumps (code size bound)
-    if (const char* e = std::getenv("FD_JIT_DEEP_STUMPS")) budget = std::atoi(e);
+int jit_deep_end(const StageDev* st, int n_stages, const char* env, int budget) {
+    if (const char* e = std::getenv(env)) budget = std::atoi(e);   // generated deep stumps (code size bound)
     int k = 1;
     while (k < n_stages && st[k].n <= budget) budget -= st[k++].n;
     return k;
@@ -195,7 +194,11 @@ static int jit_ctas() {
 }
 
 std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages, const std::vector<uint32_t>* pk16) {
-    const int k_end = jit_deep_end(st, n_stages);
+    // k_deep1 runs its specialised stages one lane per window even when few windows are left, so
+    // it gets the first ~60 stumps; k_deepq's warps each run their own stage, so only the code of
+    // its busiest stage (s0 = 2) is generated -- more straight-line code thrashes the I-caches
+    const int k_end = jit_deep_end(st, n_stages, "FD_JIT_DEEP_STUMPS", 60);
+    const int k_endq = jit_deep_end(st, n_stages, "FD_JIT_DEEPQ_STUMPS", n_stages > 2 ? st[1].n + st[2].n : 0);
     std::string pre;
     if (pk16 && !pk16->empty()) {
         // the records are data of this program (its own __constant__ bank); a digest of them in the
@@ -211,9 +214,13 @@ std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_sta
                       "\n#define FD_K2_CTAS " + std::to_string(jit_ctas()) +
                       "\n#define FD_DQ_SLOTS " + std::to_string(jit_dq_slots()) +
                       "\n#define FD_DQ_WARPS " + std::to_string(jit_dq_warps()) +
+                      "\n#define FD_DQ_GROUP " + std::to_string(env_or("FD_DQ_GROUP", 16)) +
                       "\n#include \"fd_internal.h\"\n" + jit_stage1_source(rec_words, st[0].first, st[0].n) +
                       "#define FD_JIT_STAGE1 1\n";
-    if (k_end > 1) src += jit_deep_source(rec_words, st, k_end) + "#define FD_JIT_DEEP " + std::to_string(k_end) + "\n";
+    // (two functions: one switch over every generated stage bloats k_deep1's code)
+    if (k_end > 1) src += jit_deep_source(rec_words, st, k_end, "jit_deep") + "#define FD_JIT_DEEP " + std::to_string(k_end) + "\n";
+    if (k_endq > 1)
+        src += jit_deep_source(rec_words, st, k_endq, "jit_deepq") + "#define FD_JIT_DEEPQ " + std::to_string(k_endq) + "\n";
     return src + "#include \"k_cascade.cu\"\n";
 }
 

@@ -15,7 +15,7 @@ enum { JIT_FUSED = 0, JIT_STAGE1 = 1, JIT_DEEP1 = 2, JIT_F1 = 3, JIT_DEEP1_F1 = 
 // records, REC_WORDS u32 per stump)
 std::string jit_stage1_source(const uint32_t* rec_words, int first, int n);
 // generated deep stages [1, k_end) (lane-per-window code with immediate corner offsets)
-std::string jit_deep_source(const uint32_t* rec_words, const StageDev* st, int k_end);
+std::string jit_deep_source(const uint32_t* rec_words, const StageDev* st, int k_end, const char* name);
 // the whole NVRTC program for a cascade (generated stages + k_cascade.cu)
 // pk16: f3 compressed records (FD_PK_WORDS u32 per stump) held in the program's __constant__ bank
 // and read by the lane-per-window deep stages, or null

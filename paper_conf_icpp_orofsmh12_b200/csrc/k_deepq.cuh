@@ -5,52 +5,95 @@
 // windows are rejected (the divergence problem; Fig. 7's rejection profile,
 // P:L1311-1325).  k_stage1 leaves ~1.7% of the windows alive after stage 2, ~70 per tile that has
 // any.  Here one persistent CTA per SM keeps NS tiles' ii planes in shared memory (TMA, one
-// mbarrier per slot) and every warp works on its own batch of up to 32 windows, one lane per
-// window, all at the same stage s so the stump records stay warp-uniform (parameter bank):
-//   * after a stage the warp compacts its survivors (ballot + rank), tops them up from the ring of
-//     stage s+1, and keeps going while the batch is at least DQ_KEEP windows; a thinner batch is
-//     parked in that ring when fuller work exists -- a ring holding >= 32 windows (deepest
-//     first), fresh windows of a loaded tile, or a new tile (claimed into a free slot); with
-//     nothing fuller it continues, and an idle warp takes the deepest non-empty ring;
-//   * no CTA barrier and no lock after the start: the rings are multi-producer multi-consumer
-//     (head / tail reserved with CAS, a sequence word per cell publishes and frees it), fresh
-//     windows are taken with a CAS on the slot's (taken | n) word, slots and prefetched tile-list
-//     entries with atomics, so a tile's slowest window never holds up the others;
+// mbarrier per slot, with the tile's survivor list copied next to it) and every warp works on
+// its own batch of up to 32 windows -- fresh stage-s0 windows of any loaded tiles, one lane per
+// window, so the stump records stay warp-uniform (parameter bank / generated code):
+//   * after each stage the warp compacts its survivors (ballot + rank) and goes on with them; a
+//     batch of at most FD_DQ_GROUP windows runs GL = 2^lg lanes per window (the largest with
+//     cnt * GL <= 32) that share the stage's stumps, so a thinning batch keeps its lanes busy and
+//     its latency short;
+//   * windows entering stage s_tail leave for k_tail's queue (one warp per window there): the
+//     long chains of the last stages would otherwise hold their tile's slot;
+//   * when its batch is empty the warp takes fresh windows (a CAS on the slot's taken | n word)
+//     or claims a prefetched tile into a free slot; there is no CTA barrier after the start and
+//     no lock, so a tile's slowest window never holds up the others;
 //   * a slot is reloaded once every window of its tile has finished (per-slot alive count).
 // Windows of different tiles share a batch (each lane addresses its own slot's plane).  Decisions,
-// scores and outputs are the definition's: lane-per-window sequential fp32 sums (oracle c7/c8).
+// scores and outputs are the definition's: sequential fp32 stage sums in stump order, or tree
+// sums whose decision is certified against their rounding bound (oracle c7/c8).
 #pragma once
 
 namespace fdk {
 
+#ifndef FD_JIT_DEEPQ
+#define FD_JIT_DEEPQ 0       // run-time specialised kernel: stages [1, FD_JIT_DEEPQ) are generated code
+#endif
 #ifndef FD_DQ_NPF
 #define FD_DQ_NPF 4             // tile-list entries prefetched per CTA
 #endif
-#ifndef FD_DQ_KEEP
-#define FD_DQ_KEEP 24           // a batch thinner than this is parked when fuller work exists
+#ifndef FD_DQ_GROUP
+#define FD_DQ_GROUP 16          // batches of at most this many windows run GL > 1 lanes per window
 #endif
+
+// Compact evaluators (one stump per loop iteration, the corner count padded to 9 or 12 with zero
+// corners): every warp of the SM runs its own stage, so the code they execute together must stay
+// inside the instruction caches (L0 ~6 KB, L1.5 32 KB per SM) -- unrolled variants per corner count
+// made k_deepq's warps wait on instruction fetch more than on anything else.
+template <int MC, class R>
+__device__ __forceinline__ float dq_stage_mc(const uint32_t* __restrict__ T, int b, float nf, const R& rec, int first,
+                                         int n) {
+    float sum = 0.0f;
+#pragma unroll 1
+    for (int j = first; j < first + n; ++j) sum = __fadd_rn(sum, eval_stump_mc<MC>(T, b, nf, rec, j));
+    return sum;
+}
+template <class R>
+__device__ __forceinline__ float dq_stage(const uint32_t* __restrict__ T, int b, float nf, const R& rec, int first, int n,
+                                          int mc) {
+    return mc <= 9 ? dq_stage_mc<9>(T, b, nf, rec, first, n) : dq_stage_mc<MAX_CORNERS>(T, b, nf, rec, first, n);
+}
+// GL = 2^lg lanes per window: lane q takes stumps q, q + GL, ...; sum and sum of magnitudes of its
+// leaves, then the group's butterfly (k_common.cuh group_stage_tree, without its unrolling)
+template <int MC>
+__device__ __forceinline__ float2 dq_group_mc(const uint32_t* __restrict__ T, int b, float nf, const uint4* __restrict__ st,
+                                          int first, int n, int lg, bool act, int lane) {
+    const int gl = 1 << lg, q = lane & (gl - 1);
+    const GlobalRec rec{st};
+    float acc = 0.0f, aacc = 0.0f;
+    if (act) {
+#pragma unroll 1
+        for (int j = q; j < n; j += gl) {
+            const float l = eval_stump_mc<MC>(T, b, nf, rec, first + j);
+            acc = __fadd_rn(acc, l);
+            aacc = __fadd_rn(aacc, fabsf(l));
+        }
+    }
+    for (int o = gl >> 1; o > 0; o >>= 1) {
+        acc = __fadd_rn(acc, __shfl_xor_sync(0xffffffffu, acc, o));
+        aacc = __fadd_rn(aacc, __shfl_xor_sync(0xffffffffu, aacc, o));
+    }
+    return make_float2(acc, aacc);
+}
 
 template <int STEP, bool DEPTH>
 __global__ void __launch_bounds__(DQ_THREADS, 1) k_deepq(const __grid_constant__ CascadeParams p) {
     using G = TileGeoQ<STEP>;
     constexpr int TX = k2_tx(STEP), TW = tile_w(STEP), PBUF = G::PBUF, PLANE = tile_w(STEP) * tile_h(STEP);
-    constexpr int NS = G::NS, NQ = DQ_NQ, QC = DQ_QC, NPF = FD_DQ_NPF;
+    constexpr int NS = G::NS, NPF = FD_DQ_NPF, CAPF = DQ_CAPF;
     constexpr unsigned ALL = (NS == 32) ? 0xffffffffu : ((1u << NS) - 1u);
     constexpr unsigned FULL = 0xffffffffu;
-    static_assert(NQ <= 32 && NPF <= 32 && (QC & (QC - 1)) == 0, "one lane per ring / entry; QC a power of two");
+    static_assert(NPF <= 32, "one lane per prefetch entry");
     extern __shared__ __align__(1024) uint8_t smem_raw[];
     const uint32_t* planes = reinterpret_cast<const uint32_t*>(smem_raw);
-    volatile uint2* ent = reinterpret_cast<volatile uint2*>(smem_raw + G::OFF_Q);     // [NQ][QC] {loc, nf bits}
-    volatile int* seq = reinterpret_cast<volatile int*>(smem_raw + G::OFF_SEQ);        // [NQ][QC]
+    uint2* flist = reinterpret_cast<uint2*>(smem_raw + G::OFF_F);                  // [NS][CAPF] {window, nf bits}
     uint2* stg = reinterpret_cast<uint2*>(smem_raw + G::OFF_STG) + (threadIdx.x >> 5) * 32;   // this warp's
     __shared__ __align__(8) uint64_t mbar[NS];
     __shared__ int s_frame[NS], s_lvl[NS], s_wx0[NS], s_wy0[NS];
     __shared__ int s_alive[NS];             // windows of the slot's tile not finished yet
     __shared__ unsigned s_fw[NS];           // fresh windows: taken << 16 | n (taken == n: none left)
-    __shared__ int s_foff[NS];              // the tile's survivors: p.surv[foff, foff + n)
+    __shared__ int s_foff[NS];              // the tile's survivors: p.surv[foff, foff + n), first CAPF in flist
     __shared__ int s_wpar[NS];              // mbarrier parity of the slot's current load
     __shared__ unsigned s_free;
-    __shared__ int s_head[NQ], s_tail[NQ];  // ring q: windows entering stage s0 + 1 + q
     __shared__ int s_pfst[NPF];             // prefetched tile-list entries: 0 filling, 1 owned, 2 ready, 3 none left
     __shared__ int4 s_pf0[NPF], s_pf1[NPF]; // {tile, off, n, -}, {g, k, wx0, wy0}
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -58,8 +101,6 @@ __global__ void __launch_bounds__(DQ_THREADS, 1) k_deepq(const __grid_constant__
     const ParamRec prec{p};
     const GlobalRec grec{p.stumps};
     const WinOut<STEP, DEPTH> out{p, s_frame, s_lvl, s_wx0, s_wy0};
-    volatile int* vhead = s_head;
-    volatile int* vtail = s_tail;
     volatile int* vpfst = s_pfst;
     volatile unsigned* vfw = s_fw;
     volatile unsigned* vfree = &s_free;
@@ -89,68 +130,12 @@ __global__ void __launch_bounds__(DQ_THREADS, 1) k_deepq(const __grid_constant__
         s_fw[tid] = 0u;
         s_wpar[tid] = 0;
     }
-    if (tid < NQ) s_head[tid] = s_tail[tid] = 0;
-    for (int c = tid; c < NQ * QC; c += DQ_THREADS) seq[c] = c & (QC - 1);   // cell free for lap 0
     if (tid < NPF) s_pfst[tid] = 0;
     __syncthreads();
     if (lane == 0 && warp < NPF) refill(warp);
 
-    // ring j: pop up to k (at least kmin) entries into lanes [dst, dst + got); warp-uniform result
-    auto ring_pop = [&](int j, int k, int kmin, int dst, uint32_t& loc, float& nf) -> int {
-        int base = 0, got = 0;
-        if (lane == 0) {
-            for (;;) {
-                const int hd = vhead[j], tl = vtail[j];
-                const int t = min(k, tl - hd);
-                if (t < kmin || t <= 0) break;
-                if (atomicCAS(&s_head[j], hd, hd + t) == hd) {
-                    base = hd;
-                    got = t;
-                    break;
-                }
-            }
-        }
-        got = __shfl_sync(FULL, got, 0);
-        base = __shfl_sync(FULL, base, 0);
-        if (lane >= dst && lane < dst + got) {
-            const int pos = base + lane - dst, cell = j * QC + (pos & (QC - 1));
-            while (seq[cell] != pos + 1) {}                  // the pusher's entry has landed
-            __threadfence_block();
-            const uint2 e = make_uint2(ent[cell].x, ent[cell].y);
-            loc = e.x;
-            nf = __uint_as_float(e.y);
-            __threadfence_block();
-            seq[cell] = pos + QC;                            // free for the next lap
-        }
-        return got;
-    };
-    // ring j: push lanes [0, c); false (nothing written) when the ring has no room
-    auto ring_push = [&](int j, int c, uint32_t loc, float nf) -> bool {
-        int base = -1;
-        if (lane == 0) {
-            for (;;) {
-                const int tl = vtail[j], hd = vhead[j];
-                if (tl - hd + c > QC) break;
-                if (atomicCAS(&s_tail[j], tl, tl + c) == tl) {
-                    base = tl;
-                    break;
-                }
-            }
-        }
-        base = __shfl_sync(FULL, base, 0);
-        if (base < 0) return false;
-        if (lane < c) {
-            const int pos = base + lane, cell = j * QC + (pos & (QC - 1));
-            while (seq[cell] != pos) {}                      // the previous lap's reader is done
-            ent[cell].x = loc;
-            ent[cell].y = __float_as_uint(nf);
-            __threadfence_block();
-            seq[cell] = pos + 1;
-        }
-        return true;
-    };
     // fresh windows of slot sl into lanes [dst, dst + got), at most k; warp-uniform result
-    auto take_fresh = [&](int sl, int k, int dst, uint32_t& loc, int& fidx) -> int {
+    auto take_fresh = [&](int sl, int k, int dst, uint32_t& loc, float& nf) -> int {
         int t0 = 0, got = 0;
         if (lane == 0) {
             for (;;) {
@@ -169,12 +154,15 @@ __global__ void __launch_bounds__(DQ_THREADS, 1) k_deepq(const __grid_constant__
         t0 = __shfl_sync(FULL, t0, 0);
         if (lane >= dst && lane < dst + got) {
             __threadfence_block();
-            loc = (uint32_t)sl << 16;
-            fidx = *reinterpret_cast<volatile int*>(&s_foff[sl]) + t0 + (lane - dst);
+            const int j = t0 + lane - dst;
+            const uint2 v = j < CAPF ? flist[sl * CAPF + j] : p.surv[*reinterpret_cast<volatile int*>(&s_foff[sl]) + j];
+            loc = ((uint32_t)sl << 16) | v.x;
+            nf = __uint_as_float(v.y);
         }
         return got;
     };
-    // claim a prefetched tile into a free slot (TMA of its ii plane); the slot index or -1
+    // claim a prefetched tile into a free slot (TMA of its ii plane, its survivor list copied by
+    // the warp); the slot index or -1.  Warp-collective.
     auto claim = [&]() -> int {
         int sl = -1, pf = -1;
         if (lane == 0) {
@@ -207,13 +195,23 @@ __global__ void __launch_bounds__(DQ_THREADS, 1) k_deepq(const __grid_constant__
                     mbar_expect_tx(&mbar[sl], PLANE * 4);
                     tma_load_4d(const_cast<uint32_t*>(planes) + sl * PBUF, p.tmaps + b.y, b.z * STEP, b.w * STEP, 0,
                                 b.x, &mbar[sl]);
-                    __threadfence_block();
-                    vfw[sl] = (unsigned)a.z;                 // publish: 0 taken of n
-                    refill(pf);
                 }
             }
         }
-        return __shfl_sync(FULL, sl, 0);
+        sl = __shfl_sync(FULL, sl, 0);
+        pf = __shfl_sync(FULL, pf, 0);
+        if (sl >= 0) {
+            __syncwarp();
+            const int off = s_foff[sl], n = s_alive[sl];     // written by lane 0 above
+            for (int j = lane; j < min(n, CAPF); j += 32) flist[sl * CAPF + j] = p.surv[off + j];
+            __syncwarp();
+            if (lane == 0) {
+                __threadfence_block();
+                vfw[sl] = (unsigned)n;                       // publish: 0 taken of n
+                refill(pf);
+            }
+        }
+        return sl;
     };
 
     int cnt = 0, s = s0;          // this warp's batch: lanes [0, cnt) hold windows entering stage s
@@ -221,66 +219,35 @@ __global__ void __launch_bounds__(DQ_THREADS, 1) k_deepq(const __grid_constant__
     float nf = 1.0f;
     int backoff = 64;
     for (;;) {
-        if (cnt < 32) {
-            // ---------------- scheduling: every lane reads one ring / slot / prefetch entry
-            const int qn = lane < NQ ? vtail[lane] - vhead[lane] : 0;
-            const unsigned fullm = __ballot_sync(FULL, qn >= 32);
-            const unsigned nonem = __ballot_sync(FULL, qn > 0);
+        if (cnt == 0) {
+            // ---------------- new batch: fresh windows of loaded tiles, else a new tile
             const unsigned fw = lane < NS ? vfw[lane] : 0u;
             const unsigned freshm = __ballot_sync(FULL, (fw >> 16) < (fw & 0xffffu));
             const unsigned pfm = __ballot_sync(FULL, lane < NPF && vpfst[lane] == 2);
             const unsigned endm = __ballot_sync(FULL, lane < NPF && vpfst[lane] == 3);
-            // every control decision below must be warp-uniform (the helpers are warp-collective):
-            // shared words that other warps change are read once, by lane 0, and broadcast
+            // every control decision must be warp-uniform (the helpers are warp-collective): shared
+            // words that other warps change are read once, by lane 0, and broadcast
             const unsigned freem = __shfl_sync(FULL, lane == 0 ? *vfree : 0u, 0);
             const bool can_claim = pfm && freem;
-            const int qi = s - (s0 + 1);
-            const bool ring_s = cnt > 0 && qi >= 0 && qi < NQ;
-            if (ring_s && (nonem >> qi) & 1u) cnt += ring_pop(qi, 32 - cnt, 1, cnt, loc, nf);
-            if (ring_s && cnt < FD_DQ_KEEP && ((fullm & ~(1u << qi)) || freshm || can_claim)) {
-                if (ring_push(qi, cnt, loc, nf)) cnt = 0;      // parked; take fuller work
+            int got = 0;
+            unsigned fm = freshm;
+            for (int tries = 0; tries < 3 && got < 32 && (fm || can_claim); ++tries) {
+                const int sl = fm ? __ffs(fm) - 1 : claim();
+                if (sl < 0) break;
+                fm &= ~(1u << sl);
+                got += take_fresh(sl, 32 - got, got, loc, nf);
             }
-            int fidx = -1;
-            if (cnt == 0) {
-                int got = 0;
-                if (fullm) {
-                    const int j = 31 - __clz(fullm);
-                    got = ring_pop(j, 32, 32, 0, loc, nf);
-                    s = s0 + 1 + j;
-                }
-                if (!got && (freshm || can_claim)) {
-                    unsigned fm = freshm;
-                    for (int tries = 0; tries < 3 && got < 32; ++tries) {
-                        int sl = fm ? __ffs(fm) - 1 : claim();
-                        if (sl < 0) break;
-                        fm &= ~(1u << sl);
-                        got += take_fresh(sl, 32 - got, got, loc, fidx);
-                        if (!fm && got < 32 && !can_claim) break;
-                    }
-                    s = s0;
-                }
-                if (!got && nonem) {
-                    const int j = 31 - __clz(nonem);
-                    got = ring_pop(j, 32, 1, 0, loc, nf);
-                    s = s0 + 1 + j;
-                }
-                if (!got) {
-                    const unsigned fr2 = __shfl_sync(FULL, lane == 0 ? *vfree : 0u, 0);
-                    if (endm == (NPF == 32 ? FULL : (1u << NPF) - 1u) && fr2 == ALL && !nonem) break;   // all done
-                    __nanosleep(backoff);
-                    backoff = min(2 * backoff, 2048);
-                    continue;
-                }
-                backoff = 64;
-                cnt = got;
+            if (!got) {
+                if (endm == (NPF == 32 ? FULL : (1u << NPF) - 1u) && freem == ALL) break;   // all done
+                __nanosleep(backoff);
+                backoff = min(2 * backoff, 2048);
+                continue;
             }
-            if (fidx >= 0) {                               // fresh window: index and nf from k_stage1's list
-                const uint2 v = p.surv[fidx];
-                loc |= v.x;
-                nf = __uint_as_float(v.y);
-            }
+            backoff = 64;
+            cnt = got;
+            s = s0;
         }
-        // ---------------- one stage for the batch, lane per window
+        // ---------------- one stage for the batch
         const bool act = lane < cnt;
         const int sl = (int)(loc >> 16), idx = (int)(loc & 0xffffu);
         if (act && s == s0) mbar_wait(&mbar[sl], (uint32_t)(s_wpar[sl] ^ 1));   // the tile's plane has landed
@@ -294,38 +261,71 @@ __global__ void __launch_bounds__(DQ_THREADS, 1) k_deepq(const __grid_constant__
             sd = p.stages[s];
         }
         if (lane == 0 && p.stage_counts) atomicAdd(p.stage_counts + s, (unsigned long long)cnt);
+        const bool last = s == N - 1;
         float sum = 0.0f;
-        if (act) {
-            const int b = sl * PBUF + (idx / TX) * STEP * TW + (idx % TX) * STEP;
-#if FD_JIT_DEEP > 0
-            if (s < FD_JIT_DEEP)
-                sum = jit_deep(s, planes + b, nf);
-            else
+        bool pass;
+#ifndef FD_PACKED_WORDS
+        if (cnt <= FD_DQ_GROUP) {
+            // thin batch: GL = 2^lg lanes per window share the stage's stumps (records warp-uniform
+            // per stump index); the leaves are added as a tree and the decision certified against
+            // its rounding bound (k_common.cuh certify) -- the group leader re-adds them in stump
+            // order for near ties and for output scores
+            int lg = 1;
+            while (lg < 5 && (cnt << (lg + 1)) <= 32) ++lg;
+            const int e = lane >> lg;
+            const bool gact = e < cnt;
+            const uint32_t gloc = __shfl_sync(FULL, loc, e & 31);
+            const float gnf = __shfl_sync(FULL, nf, e & 31);
+            const int gsl = (int)(gloc >> 16), gidx = (int)(gloc & 0xffffu);
+            if (gact && s == s0) mbar_wait(&mbar[gsl], (uint32_t)(s_wpar[gsl] ^ 1));
+            const int gb = gsl * PBUF + (gidx / TX) * STEP * TW + (gidx % TX) * STEP;
+            const float2 t = sd.mc <= 9 ? dq_group_mc<9>(planes, gb, gnf, p.stumps, sd.first, sd.n, lg, gact, lane)
+                                        : dq_group_mc<MAX_CORNERS>(planes, gb, gnf, p.stumps, sd.first, sd.n, lg, gact, lane);
+            int dec = certify(t.x, t.y, sd.n, (sd.n + (1 << lg) - 1) / (1 << lg) - 1 + lg, sd.T);
+            float gsum = t.x;
+            if (gact && (lane & ((1 << lg) - 1)) == 0 && (dec < 0 || (dec == 1 && last) || (DEPTH && dec == 0))) {
+                gsum = dq_stage(planes, gb, gnf, grec, sd.first, sd.n, sd.mc);
+                dec = gsum >= sd.T ? 1 : 0;
+            }
+            sum = __shfl_sync(FULL, gsum, (lane << lg) & 31);    // back to one lane per window
+            dec = __shfl_sync(FULL, dec, (lane << lg) & 31);
+            pass = act && dec == 1;
+        } else
+#endif
+        {
+            if (act) {
+                const int b = sl * PBUF + (idx / TX) * STEP * TW + (idx % TX) * STEP;
+#if FD_JIT_DEEPQ > 0
+                if (s < FD_JIT_DEEPQ)
+                    sum = jit_deepq(s, planes + b, nf);
+                else
 #endif
 #ifdef FD_PACKED_WORDS
-                sum = eval_stage_packed<STEP>(planes, b, nf, sd.first, sd.n);
+                    sum = eval_stage_packed<STEP>(planes, b, nf, sd.first, sd.n);
 #else
-                sum = sd.first + sd.n <= p.n_pstumps ? eval_stage(planes, b, nf, prec, sd.first, sd.n, sd.mc)
-                                                     : eval_stage(planes, b, nf, grec, sd.first, sd.n, sd.mc);
+                    sum = sd.first + sd.n <= p.n_pstumps ? dq_stage(planes, b, nf, prec, sd.first, sd.n, sd.mc)
+                                                         : dq_stage(planes, b, nf, grec, sd.first, sd.n, sd.mc);
 #endif
+            }
+            pass = act && sum >= sd.T;
         }
-        const bool pass = act && sum >= sd.T;
-        const bool last = s == N - 1;
         if (act && !pass) out.reject(sl, idx, s, sum);
         if (pass && last) out.emit(sl, idx, sum);
-        const bool fin = act && (!pass || last);
-        const unsigned finm = __ballot_sync(FULL, fin);
-        if (fin) {
-            // per-slot alive counts; the window that finishes a tile frees its slot
-            const unsigned peers = __match_any_sync(finm, sl);
-            if (lane == __ffs(peers) - 1) {
-                const int k = __popc(peers);
-                if (atomicSub(&s_alive[sl], k) == k) {
-                    __threadfence_block();
-                    atomicOr(&s_free, 1u << sl);
+        // windows that finish here, and (below) windows handed to k_tail, release their slot
+        auto release = [&](bool fin, int fsl) {
+            const unsigned fm = __ballot_sync(FULL, fin);
+            if (fin) {
+                const unsigned peers = __match_any_sync(fm, fsl);
+                if (lane == __ffs(peers) - 1) {
+                    const int k = __popc(peers);
+                    if (atomicSub(&s_alive[fsl], k) == k) {  // the tile's last window: free its slot
+                        __threadfence_block();
+                        atomicOr(&s_free, 1u << fsl);
+                    }
                 }
             }
-        }
+        };
+        release(act && (!pass || last), sl);
         const unsigned m = __ballot_sync(FULL, pass && !last);
         if (pass && !last) stg[__popc(m & ((1u << lane) - 1u))] = make_uint2(loc, __float_as_uint(nf));
         __syncwarp();
@@ -337,6 +337,38 @@ __global__ void __launch_bounds__(DQ_THREADS, 1) k_deepq(const __grid_constant__
         }
         __syncwarp();
         s += 1;
+        if (p.tail_q && cnt > 0 && s >= p.s_tail) {
+            // long chains leave the pool: windows entering stage s_tail go to k_tail's queue (one warp
+            // per window there), so their tile's slot is not held for the rest of the cascade
+            int pos = 0;
+            if (lane == 0) pos = (int)atomicAdd(p.tail_count, (unsigned)cnt);
+            pos = __shfl_sync(FULL, pos, 0);
+            const bool hand = lane < cnt && pos + lane < p.tail_cap;
+            const int sl2 = (int)(loc >> 16), idx2 = (int)(loc & 0xffffu);
+            if (hand) {
+                uint4 q;
+                q.x = ((unsigned)s_lvl[sl2] << 8) | (unsigned)s;
+                q.y = ((unsigned)(s_wy0[sl2] + idx2 / TX) << 16) | (unsigned)(s_wx0[sl2] + idx2 % TX);
+                q.z = __float_as_uint(nf);
+                q.w = (unsigned)(s_frame[sl2] - p.frame_base);
+                p.tail_q[pos + lane] = q;
+            }
+            const unsigned hm = __ballot_sync(FULL, hand);
+            if (hm) {
+                if (lane == 0 && p.stage_counts) atomicAdd(p.stage_counts + s, (unsigned long long)__popc(hm));
+                release(hand, sl2);
+                const int h = __popc(hm);               // the handed lanes are the lowest ones
+                if (lane >= h && lane < cnt) stg[lane - h] = make_uint2(loc, __float_as_uint(nf));
+                __syncwarp();
+                cnt -= h;
+                if (lane < cnt) {
+                    const uint2 e = stg[lane];
+                    loc = e.x;
+                    nf = __uint_as_float(e.y);
+                }
+                __syncwarp();
+            }
+        }
     }
 }
 

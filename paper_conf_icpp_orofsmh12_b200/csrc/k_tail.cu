@@ -98,12 +98,10 @@ __global__ void __launch_bounds__(TAIL_THREADS, 4) k_tail(const __grid_constant_
         // leaf of stump c0 + lane of stage sd (0 beyond the stage); MC >= the stage's largest
         // corner count (unused corner slots are offset 0, coefficient 0), so the corner loads do
         // not wait for the stump's own count
-        auto leaf_mc = [&](const StageDev& sd, int c0, auto mc_tag) -> float {
+        // (the shared-memory and global record paths are separate so each compiles to its own
+        // address space: 32-bit LDS, or LDG through the read-only path)
+        auto leaf_rec = [&](const uint32_t* t, int ws, auto mc_tag) -> float {
             constexpr int MC = decltype(mc_tag)::value;
-            if (c0 + lane >= sd.n) return 0.0f;
-            const bool shared = sd.first >= p.j0 && sd.first + sd.n <= p.j0 + p.nsm;   // stage-uniform
-            const uint32_t* t = shared ? srec + (sd.first - p.j0 + c0 + lane) : p.trec + sd.first + c0 + lane;
-            const size_t ws = shared ? (size_t)p.nsm : (size_t)p.ns;
             uint32_t f = 0;
 #pragma unroll
             for (int c = 0; c < MC; ++c) {
@@ -112,6 +110,22 @@ __global__ void __launch_bounds__(TAIL_THREADS, 4) k_tail(const __grid_constant_
             }
             const float tt = __fmul_rn(__int_as_float((int)t[ws]), nf);
             return (__int2float_rn((int)f) < tt) ? __int_as_float((int)t[2 * ws]) : __int_as_float((int)t[3 * ws]);
+        };
+        auto leaf_mc = [&](const StageDev& sd, int c0, auto mc_tag) -> float {
+            constexpr int MC = decltype(mc_tag)::value;
+            if (c0 + lane >= sd.n) return 0.0f;
+            if (sd.first >= p.j0 && sd.first + sd.n <= p.j0 + p.nsm)     // stage-uniform
+                return leaf_rec(srec + (sd.first - p.j0 + c0 + lane), p.nsm, IntC<MC>{});
+            const uint32_t* __restrict__ g = p.trec + sd.first + c0 + lane;
+            uint32_t f = 0;
+#pragma unroll
+            for (int c = 0; c < MC; ++c) {
+                const uint32_t w = __ldg(g + (size_t)(4 + c) * p.ns);
+                f += (uint32_t)((int)w >> 16) * R[w & 0xffffu];
+            }
+            const float tt = __fmul_rn(__int_as_float((int)__ldg(g + p.ns)), nf);
+            return (__int2float_rn((int)f) < tt) ? __int_as_float((int)__ldg(g + 2 * (size_t)p.ns))
+                                                 : __int_as_float((int)__ldg(g + 3 * (size_t)p.ns));
         };
         auto leaf_of = [&](const StageDev& sd, int c0) -> float {
             if (sd.mc <= 6) return leaf_mc(sd, c0, IntC<6>{});

@@ -136,6 +136,10 @@ K2_SCHEDULES = {
     "deepq_s0_1": {"FD_DEEPQ": "1", "FD_S0": "1"},
     "deepq_two_slot": {"FD_DEEPQ": "1", "FD_GROUP_FRAMES": "1"},
     "deepq_2_slots": {"FD_DEEPQ": "1", "FD_DQ_SLOTS": "2", "FD_DQ_WARPS": "4"},   # slot reuse / pinning pressure (JIT only)
+    "deepq_tail_3": {"FD_DEEPQ": "1", "FD_DQ_TAIL": "3"},   # windows entering stage 3 go to k_tail
+    "deepq_no_tail": {"FD_DEEPQ": "1", "FD_DQ_TAIL": "255"},     # k_deepq finishes every window
+    "deepq_lane_only": {"FD_DEEPQ": "1", "FD_DQ_GROUP": "0"},    # no GL > 1 lane groups
+    "deepq_group_all": {"FD_DEEPQ": "1", "FD_DQ_GROUP": "32", "FD_JIT_DEEPQ_STUMPS": "0"},   # every batch in lane groups
     "deep1_no_tail": {"FD_DEEPQ": "0", "FD_TAIL": "0"},     # k_deep1 finishes every window
     "deep1_split_stump": {"FD_DEEPQ": "0", "FD_DEEP_SPLIT": "64"},   # deep stages <= 64 windows split-stump
     "deep1_2warps": {"FD_DEEPQ": "0", "FD_K2D_THREADS": "64"},       # two-warp k_deep1 blocks
@@ -155,7 +159,8 @@ K2_SCHEDULES = {
 
 
 # variables read when a cascade's specialised program is generated (once per fd.Cascade)
-JIT_GEOMETRY_ENV = {"FD_DQ_SLOTS", "FD_DQ_WARPS", "FD_K2D_THREADS", "FD_K2D_CTAS", "FD_K2_CTAS", "FD_F1_CTAS"}
+JIT_GEOMETRY_ENV = {"FD_DQ_SLOTS", "FD_DQ_WARPS", "FD_DQ_GROUP", "FD_JIT_DEEPQ_STUMPS", "FD_K2D_THREADS", "FD_K2D_CTAS",
+                    "FD_K2_CTAS", "FD_F1_CTAS"}
 
 
 @pytest.mark.parametrize("jit", ["1", "0"])
