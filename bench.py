@@ -399,9 +399,9 @@ def run_ours(args):
     else:
         s0 = int(os.environ.get("FD_S0", "2"))
         roof_main = roof(f"k_stage1 (K2, stages [0, {s0}))", t_casc, n_casc, 0, s0, True, traffic_key="k_stage1")
-        dq = os.environ.get("FD_DEEPQ", "1") != "0"
-        roof_other = roof(f"{'k_deepq' if dq else 'k_deep1+k_tail'} (K2, stages [{s0}, N))", t_deep + t_tail, n_casc,
-                          s0, ns, False, traffic_key="k_deepq" if dq else "k_deep1")
+        dname = "k_deep1" if os.environ.get("FD_DEEPQ", "1") == "0" else "k_deepq"
+        roof_other = roof(f"{dname}{'+k_tail' if t_tail else ''} (K2, stages [{s0}, N))", t_deep + t_tail, n_casc,
+                          s0, ns, False, traffic_key=dname)
         if roof_other["per_launch_ms"] > roof_main["per_launch_ms"]:
             roof_main, roof_other = roof_other, roof_main
     k1_names = ("level",) if f1 else ("colsum", "carry", "band")

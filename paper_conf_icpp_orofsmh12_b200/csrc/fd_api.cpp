@@ -702,12 +702,12 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     const bool f1_split = f1 && env_int("FD_F1_SPLIT", 1) != 0;
     const bool split = !queue && !f1 && env_int("FD_K2_SPLIT", 1) != 0;
     const bool surv = split || f1_split;
-    // split K2 deep stages: k_deep1 (CTA per tile, stage-synchronous) + k_tail, or FD_DEEPQ=1:
-    // k_deepq (warp-autonomous batches over a per-SM tile pool, no tail hand-off)
-    const bool deepq = split && env_int("FD_DEEPQ", 0) != 0;
-    // k_deepq hands every window that enters stage FD_DQ_TAIL to k_tail (long chains would hold
-    // their tile's slot); 255 = never
-    const int dq_tail = std::max(1, env_int("FD_DQ_TAIL", 7));
+    // split K2 deep stages: k_deepq (default: warp-autonomous batches over a per-SM pool of tiles)
+    // or FD_DEEPQ=0: k_deep1 (a 4-warp CTA per tile, stage-synchronous) + k_tail
+    const bool deepq = split && env_int("FD_DEEPQ", 1) != 0;
+    // FD_DQ_TAIL=s: k_deepq hands every window that enters stage s to k_tail (default 255: never --
+    // measured best for c3; stage 9 is close for the OpenCV-shaped c6)
+    const int dq_tail = std::max(1, env_int("FD_DQ_TAIL", 255));
     // tail queue (k_tail): FD_TAIL=0 keeps every window inside K2; FD_TAIL_N = windows left in a
     // batch at which it hands them over; FD_TAIL_CAP = queue entries (16 B each) per group
     const bool use_tail = !queue && env_int("FD_TAIL", 1) != 0 && (!deepq || dq_tail < (int)c->stages.size());

@@ -265,7 +265,7 @@ __global__ void __launch_bounds__(DQ_THREADS, 1) k_deepq(const __grid_constant__
         float sum = 0.0f;
         bool pass;
 #ifndef FD_PACKED_WORDS
-        if (cnt <= FD_DQ_GROUP) {
+        if (cnt <= (FD_DQ_GROUP < 16 ? FD_DQ_GROUP : 16)) {      // (GL >= 2 needs cnt <= 16)
             // thin batch: GL = 2^lg lanes per window share the stage's stumps (records warp-uniform
             // per stump index); the leaves are added as a tree and the decision certified against
             // its rounding bound (k_common.cuh certify) -- the group leader re-adds them in stump

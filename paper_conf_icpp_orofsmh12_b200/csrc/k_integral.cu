@@ -20,44 +20,45 @@ namespace fdk {
 // (k_marg / k_tile compiled for 6 resident CTAs per SM -- 40 registers -- measured no faster)
 
 // ---------------------------------------------------------------- scaling (reading R2)
+// The taps are addressed from one corner: (x0, y0) and (x0 + 1, y0 + 1).  Where reading R2 clamps
+// x1 = x0 = W - 1 (the sample lies past the last pixel centre), the corner moves to W - 2 with
+// weight a_x = 256 instead: p00 (256 - 256) + p01 * 256 = p[W-1] * 256 = p[W-1] (256 - a) + p[W-1] a,
+// the same integer; likewise for rows.  So every tap is the corner address + {0, 1, pitch,
+// pitch + 1} (two 64-bit addresses per pixel, immediate offsets for the rest).  Needs W, H >= 2.
 struct RowSample {
-    const uint8_t* r0;
-    const uint8_t* r1;
+    const uint8_t* r0;      // row y0 (its successor is r0 + pitch)
     int ay;
 };
 
 __device__ __forceinline__ RowSample row_sample(const uint8_t* frame, int pitch, int H, int r16, int y) {
     const long long sy = ((2LL * y + 1) * (long long)r16 - 65536) >> 1;
-    int y0 = (int)(sy >> 16);
-    y0 = y0 < H - 1 ? y0 : H - 1;
-    const int y1 = y0 + 1 < H ? y0 + 1 : H - 1;
+    const int y0 = (int)(sy >> 16);
     RowSample s;
-    s.r0 = frame + (size_t)y0 * pitch;
-    s.r1 = frame + (size_t)y1 * pitch;
-    s.ay = (int)((sy >> 8) & 255);
+    s.ay = y0 < H - 1 ? (int)((sy >> 8) & 255) : 256;
+    s.r0 = frame + (size_t)(y0 < H - 1 ? y0 : H - 2) * pitch;
     return s;
 }
 
 struct ColSample {
-    int x0, x1, ax;
+    int x0, ax;
 };
 
 __device__ __forceinline__ ColSample col_sample(int W, int r16, int x) {
     const long long sx = ((2LL * x + 1) * (long long)r16 - 65536) >> 1;
-    int x0 = (int)(sx >> 16);
-    x0 = x0 < W - 1 ? x0 : W - 1;
+    const int x0 = (int)(sx >> 16);
     ColSample c;
-    c.x0 = x0;
-    c.x1 = x0 + 1 < W ? x0 + 1 : W - 1;
-    c.ax = (int)((sx >> 8) & 255);
+    c.x0 = x0 < W - 1 ? x0 : W - 2;
+    c.ax = x0 < W - 1 ? (int)((sx >> 8) & 255) : 256;
     return c;
 }
 
 // p = (p00(256-ax)(256-ay) + p01 ax(256-ay) + p10(256-ax)ay + p11 ax ay + 2^15) >> 16,
 // evaluated as two horizontal lerps then one vertical (identical in exact integer arithmetic).
-__device__ __forceinline__ uint32_t bilinear(const RowSample& r, const ColSample& c) {
-    const int p00 = __ldg(r.r0 + c.x0), p01 = __ldg(r.r0 + c.x1);
-    const int p10 = __ldg(r.r1 + c.x0), p11 = __ldg(r.r1 + c.x1);
+__device__ __forceinline__ uint32_t bilinear(const RowSample& r, int pitch, const ColSample& c) {
+    const uint8_t* a = r.r0 + c.x0;
+    const uint8_t* b = a + pitch;
+    const int p00 = __ldg(a), p01 = __ldg(a + 1);
+    const int p10 = __ldg(b), p11 = __ldg(b + 1);
     const int h0 = p00 * (256 - c.ax) + p01 * c.ax;
     const int h1 = p10 * (256 - c.ax) + p11 * c.ax;
     return (uint32_t)((h0 * (256 - r.ay) + h1 * r.ay + 32768) >> 16);
@@ -67,7 +68,7 @@ __device__ __forceinline__ uint32_t level_pixel(const uint8_t* frame, int pitch,
                                                 int x, int y) {
     if (r16 == 65536) return __ldg(frame + (size_t)y * pitch + x);   // level 0: identity
     const RowSample r = row_sample(frame, pitch, srcH, r16, y);
-    return bilinear(r, col_sample(srcW, r16, x));
+    return bilinear(r, pitch, col_sample(srcW, r16, x));
 }
 
 // The 4 level pixels of row y at columns x .. x+3 (0 at or beyond the level width).  Identity
@@ -91,7 +92,7 @@ __device__ __forceinline__ void tile_row_pixels(const uint8_t* frame, const Plan
     const RowSample rs = row_sample(frame, p.pitch, p.H, L.r16, y);
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-        const uint32_t v = bilinear(rs, cs[j]);
+        const uint32_t v = bilinear(rs, p.pitch, cs[j]);
         pv[j] = x + j < L.W ? v : 0u;
     }
 }

@@ -128,18 +128,20 @@ def test_depth_maps_generic_k2(monkeypatch):
 
 # K2 schedules (fd_api.cpp run_groups): every one computes the same depth maps and detections
 K2_SCHEDULES = {
-    "split_default": {},                                    # K1 -> k_stage1 -> k_deep1 -> k_tail
+    "split_default": {},                                    # K1 -> k_stage1 -> k_deepq
     "split_s0_1": {"FD_S0": "1"},                           # k_stage1 stage 1 only
     "split_two_slot": {"FD_GROUP_FRAMES": "1"},             # 3 frame groups over 2 slots/streams
     "split_one_slot": {"FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
-    "deepq": {"FD_DEEPQ": "1"},                             # K1 -> k_stage1 -> k_deepq
+    "deepq_tail_9": {"FD_DEEPQ": "1", "FD_DQ_TAIL": "9"},   # windows entering stage 9 go to k_tail
     "deepq_s0_1": {"FD_DEEPQ": "1", "FD_S0": "1"},
     "deepq_two_slot": {"FD_DEEPQ": "1", "FD_GROUP_FRAMES": "1"},
     "deepq_2_slots": {"FD_DEEPQ": "1", "FD_DQ_SLOTS": "2", "FD_DQ_WARPS": "4"},   # slot reuse / pinning pressure (JIT only)
     "deepq_tail_3": {"FD_DEEPQ": "1", "FD_DQ_TAIL": "3"},   # windows entering stage 3 go to k_tail
-    "deepq_no_tail": {"FD_DEEPQ": "1", "FD_DQ_TAIL": "255"},     # k_deepq finishes every window
     "deepq_lane_only": {"FD_DEEPQ": "1", "FD_DQ_GROUP": "0"},    # no GL > 1 lane groups
-    "deepq_group_all": {"FD_DEEPQ": "1", "FD_DQ_GROUP": "32", "FD_JIT_DEEPQ_STUMPS": "0"},   # every batch in lane groups
+    "deepq_generic": {"FD_DEEPQ": "1", "FD_JIT_DEEPQ_STUMPS": "0"},   # no generated deep stages
+    "deepq_group_all": {"FD_DEEPQ": "1", "FD_DQ_GROUP": "32"},   # the group bound clamps to 16 windows
+    "deep1": {"FD_DEEPQ": "0"},                             # K1 -> k_stage1 -> k_deep1 -> k_tail
+    "deep1_two_slot": {"FD_DEEPQ": "0", "FD_GROUP_FRAMES": "1"},
     "deep1_no_tail": {"FD_DEEPQ": "0", "FD_TAIL": "0"},     # k_deep1 finishes every window
     "deep1_split_stump": {"FD_DEEPQ": "0", "FD_DEEP_SPLIT": "64"},   # deep stages <= 64 windows split-stump
     "deep1_2warps": {"FD_DEEPQ": "0", "FD_K2D_THREADS": "64"},       # two-warp k_deep1 blocks
@@ -466,12 +468,13 @@ def test_all_pass_and_all_reject():
     assert len(fd.fd_detect(allrej, torch.from_numpy(fr).cuda(), 24, s, 1)) == 0
 
 
-@pytest.mark.parametrize("env", [{}, {"FD_DEEPQ": "1"}, {"FD_DEEPQ": "1", "FD_JIT": "0"},
-                                 {"FD_DEEPQ": "1", "FD_DQ_SLOTS": "2", "FD_DQ_WARPS": "4"}])
+@pytest.mark.parametrize("env", [{}, {"FD_DEEPQ": "0"}, {"FD_JIT": "0"}, {"FD_DQ_TAIL": "4"},
+                                 {"FD_DQ_SLOTS": "2", "FD_DQ_WARPS": "4"}])
 def test_all_pass_deep(env, monkeypatch):
-    """Every window survives every stage of a 7-stage cascade: k_deepq's queues overflow (2048
-    windows per tile), batches stay full through every deep stage, slots are reused only after
-    all of their windows are emitted.  Detections and depth maps equal the oracle's."""
+    """Every window survives every stage of a 7-stage cascade: k_deepq's batches stay full through
+    every deep stage (2048 windows per tile, more than a slot's shared-memory survivor list), slots
+    are reused only after all of their windows are emitted or handed to k_tail.  Detections and
+    depth maps equal the oracle's."""
     for k, v in env.items():
         monkeypatch.setenv(k, v)
     st = ([(1, 1, 10, 10, -1), (1, 1, 5, 10, 2)], 0.1, 0.5, 0.25)
