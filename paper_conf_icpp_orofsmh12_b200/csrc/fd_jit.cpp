@@ -195,10 +195,11 @@ static int jit_ctas() {
 
 std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages, const std::vector<uint32_t>* pk16) {
     // k_deep1 runs its specialised stages one lane per window even when few windows are left, so
-    // it gets the first ~60 stumps; k_deepq's warps each run their own stage, so only the code of
-    // its busiest stage (s0 = 2) is generated -- more straight-line code thrashes the I-caches
+    // it gets the first ~60 stumps; k_deepq's warps each run their own stage, so its generated
+    // stages are bounded at ~150 stumps (c3: stages 1-6, ~20 KB of code next to the compact
+    // generic loop; measured 43.4 / 42.2 / 41.7 / 41.0 ms per 512 frames at 32 / 60 / 100 / 150)
     const int k_end = jit_deep_end(st, n_stages, "FD_JIT_DEEP_STUMPS", 60);
-    const int k_endq = jit_deep_end(st, n_stages, "FD_JIT_DEEPQ_STUMPS", n_stages > 2 ? st[1].n + st[2].n : 0);
+    const int k_endq = jit_deep_end(st, n_stages, "FD_JIT_DEEPQ_STUMPS", 150);
     std::string pre;
     if (pk16 && !pk16->empty()) {
         // the records are data of this program (its own __constant__ bank); a digest of them in the
