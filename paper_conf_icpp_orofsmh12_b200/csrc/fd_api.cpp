@@ -703,8 +703,10 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     const bool split = !queue && !f1 && env_int("FD_K2_SPLIT", 1) != 0;
     const bool surv = split || f1_split;
     // split K2 deep stages: k_deepq (default: warp-autonomous batches over a per-SM pool of tiles)
-    // or FD_DEEPQ=0: k_deep1 (a 4-warp CTA per tile, stage-synchronous) + k_tail
-    const bool deepq = split && env_int("FD_DEEPQ", 1) != 0;
+    // or FD_DEEPQ=0: k_deep1 (a 4-warp CTA per tile, stage-synchronous) + k_tail.  Compressed (f3)
+    // cascades default to k_deep1: k_deepq has no lane-group path for the packed records and ran
+    // c6q at 970 vs 1890 frames/s
+    const bool deepq = split && env_int("FD_DEEPQ", c->compressed ? 0 : 1) != 0;
     // FD_DQ_TAIL=s: k_deepq hands every window that enters stage s to k_tail (default 255: never --
     // measured best for c3; stage 9 is close for the OpenCV-shaped c6)
     const int dq_tail = std::max(1, env_int("FD_DQ_TAIL", 255));
