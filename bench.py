@@ -182,12 +182,12 @@ def load_peaks():
         return {}
 
 
-def ncu_traffic(kernel: str):
-    """DRAM read + write bytes per launch of `kernel` from the committed ncu --set full capture
-    (profiles/ncu_traffic.json), if any."""
+def ncu_traffic(kernel: str, frames: float = 1.0):
+    """DRAM read + write bytes of `kernel` for `frames` frames, from the committed ncu --set full
+    capture (profiles/ncu_traffic.json: bytes per captured launch of frames_per_launch frames)."""
     try:
-        d = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-        return d.get(kernel, {}).get("dram_bytes_per_launch")
+        d = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json"))).get(kernel, {})
+        return d["dram_bytes_per_launch"] / d["frames_per_launch"] * frames
     except Exception:
         return None
 
@@ -380,7 +380,7 @@ def run_ours(args):
              "timing": "CUDA events on the launching stream, untimed one-slot pass (FD_PIPE=0)",
              "ops_model": "SURVEY 8(d): 30 per window (variance) + (8 r + 5) per stump evaluated"
                           + (f" + {INTEGRAL_OPS_PER_PX} per level pixel (tile-local integral)" if extra_ops else ""),
-             "traffic": ncu_traffic(traffic_key) if traffic_key else None}
+             "traffic": ncu_traffic(traffic_key, F / max(n_launch, 1)) if traffic_key else None}
         r["frac"] = r["achieved"] / issue_peak if r["achieved"] else None
         r["frac_lower_bound"] = r["achieved_lower_bound"] / issue_peak if r["achieved_lower_bound"] else None
         return r
@@ -425,7 +425,7 @@ def run_ours(args):
                         "bound": "hbm", "achieved": k1_ach, "peak": hbm, "unit": "GB/s",
                         "frac": (k1_ach / hbm) if k1_ach else None,
                         "algorithmic_bytes_per_frame": level_bytes(plan, f1),
-                        "traffic": ncu_traffic("k_level" if f1 else "k1"),
+                        "traffic_per_frame": ncu_traffic("k_level" if f1 else "k1"),
                         "peak_basis": "MEASURED_PEAKS.json hbm_gbs (burst copy)"},
         "kernel_ms_per_step_one_slot": {k: v[1] for k, v in prof.items() if v[0]},
         "gpu_launches": my_launches,

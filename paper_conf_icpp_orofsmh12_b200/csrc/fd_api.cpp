@@ -702,11 +702,29 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     const bool f1_split = f1 && env_int("FD_F1_SPLIT", 1) != 0;
     const bool split = !queue && !f1 && env_int("FD_K2_SPLIT", 1) != 0;
     const bool surv = split || f1_split;
+    // frames per group: one K2 launch per group.  f1: the group's level images (12.5 MB per 1080p
+    // frame) should stay L2-resident between k_level and k_f1 (FD_F1_GROUP_MB, default 64 MB);
+    // K1 schedules: the ii/sqii planes (95.8 MB per 1080p frame; FD_GROUP_MB, default 12288 MB).
+    // FD_GROUP_FRAMES overrides.  G <= 65535 (tile and tail-queue frame indices are 32-bit, but
+    // the tensor maps' frame extent is kept within 16 bits).
+    PlanDev one;
+    make_plan_dev(pl, W, H, pitch, step, 1, &one);
+    const double per_frame = f1 ? (double)one.u8_bytes : (double)one.ws_elems * 4.0;
+    int G = env_int("FD_GROUP_FRAMES", 0);
+    // (12 GiB: 128 frames of 1080p per group; fewer, larger groups leave fewer drains of the
+    // persistent K2 kernels -- deep path 41.0 / 37.1 / 35.0 / 34.0 / 33.5 ms per 512 frames at
+    // 16 / 32 / 64 / 128 / 256 frames per group.  The survivor list is sized for the worst case,
+    // about as large again as the planes, so both pipeline slots hold ~48 GB at 1080p.)
+    const double budget = (double)(f1 ? env_int("FD_F1_GROUP_MB", 64) : env_int("FD_GROUP_MB", 12288)) * 1024.0 * 1024.0;
+    if (G <= 0) G = (int)std::min(65535.0, std::floor(budget / (per_frame > 1 ? per_frame : 1)));
+    G = std::max(1, std::min(G, std::min(n, 65535)));
+    const int ngroups = (n + G - 1) / G;
     // split K2 deep stages: k_deepq (default: warp-autonomous batches over a per-SM pool of tiles)
     // or FD_DEEPQ=0: k_deep1 (a 4-warp CTA per tile, stage-synchronous) + k_tail.  Compressed (f3)
     // cascades default to k_deep1: k_deepq has no lane-group path for the packed records and ran
-    // c6q at 970 vs 1890 frames/s
-    const bool deepq = split && env_int("FD_DEEPQ", c->compressed ? 0 : 1) != 0;
+    // c6q at 970 vs 1890 frames/s; so do groups of fewer than 4 frames (one 1080p frame: 0.55 vs
+    // 0.50 ms -- too few tiles per SM for k_deepq's slots to fill)
+    const bool deepq = split && env_int("FD_DEEPQ", (c->compressed || G < 4) ? 0 : 1) != 0;
     // FD_DQ_TAIL=s: k_deepq hands every window that enters stage s to k_tail (default 255: never --
     // measured best for c3; stage 9 is close for the OpenCV-shaped c6)
     const int dq_tail = std::max(1, env_int("FD_DQ_TAIL", 255));
@@ -714,19 +732,6 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     // batch at which it hands them over; FD_TAIL_CAP = queue entries (16 B each) per group
     const bool use_tail = !queue && env_int("FD_TAIL", 1) != 0 && (!deepq || dq_tail < (int)c->stages.size());
     const int tail_cap = use_tail ? std::max(1024, env_int("FD_TAIL_CAP", 1 << 22)) : 0;
-    // frames per group: one K2 launch per group.  f1: the group's level images (12.5 MB per 1080p
-    // frame) should stay L2-resident between k_level and k_f1 (FD_F1_GROUP_MB, default 64 MB);
-    // K1 schedules: the ii/sqii planes (95.8 MB per 1080p frame; FD_GROUP_MB, default 1536 MB).
-    // FD_GROUP_FRAMES overrides.  G <= 65535 (tile and tail-queue frame indices are 32-bit, but
-    // the tensor maps' frame extent is kept within 16 bits).
-    PlanDev one;
-    make_plan_dev(pl, W, H, pitch, step, 1, &one);
-    const double per_frame = f1 ? (double)one.u8_bytes : (double)one.ws_elems * 4.0;
-    int G = env_int("FD_GROUP_FRAMES", 0);
-    const double budget = (double)(f1 ? env_int("FD_F1_GROUP_MB", 64) : env_int("FD_GROUP_MB", 1536)) * 1024.0 * 1024.0;
-    if (G <= 0) G = (int)std::min(65535.0, std::floor(budget / (per_frame > 1 ? per_frame : 1)));
-    G = std::max(1, std::min(G, std::min(n, 65535)));
-    const int ngroups = (n + G - 1) / G;
     PlanDev& PD = *w->plan;
     make_plan_dev(pl, W, H, pitch, step, G, &PD);
     PD.filter = c->filter;

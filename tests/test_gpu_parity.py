@@ -128,10 +128,12 @@ def test_depth_maps_generic_k2(monkeypatch):
 
 # K2 schedules (fd_api.cpp run_groups): every one computes the same depth maps and detections
 K2_SCHEDULES = {
-    "split_default": {},                                    # K1 -> k_stage1 -> k_deepq
+    "split_default": {},                                    # K1 -> k_stage1 -> k_deep1 + k_tail (< 4 frames per group)
     "split_s0_1": {"FD_S0": "1"},                           # k_stage1 stage 1 only
     "split_two_slot": {"FD_GROUP_FRAMES": "1"},             # 3 frame groups over 2 slots/streams
     "split_one_slot": {"FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
+    "deepq": {"FD_DEEPQ": "1"},                             # K1 -> k_stage1 -> k_deepq (default at >= 4 frames per group)
+    "deepq_one_slot": {"FD_DEEPQ": "1", "FD_PIPE": "0", "FD_GROUP_FRAMES": "1"},
     "deepq_tail_9": {"FD_DEEPQ": "1", "FD_DQ_TAIL": "9"},   # windows entering stage 9 go to k_tail
     "deepq_s0_1": {"FD_DEEPQ": "1", "FD_S0": "1"},
     "deepq_two_slot": {"FD_DEEPQ": "1", "FD_GROUP_FRAMES": "1"},
@@ -400,10 +402,32 @@ def _bench_shape_parity(n_frames, first=0):
     return fr
 
 
-def test_video_batch_1080p_bench_shape():
-    """48 frames at the default group size (16 frames of 1080p per group -> three groups over
-    both pipeline slots and streams), every frame checked (VERDICT r1 'weak' 1)."""
+def test_video_batch_1080p_bench_shape(monkeypatch):
+    """48 frames in 16-frame groups (three groups over both pipeline slots and streams), every
+    frame, the stage counters and the grouping checked (VERDICT r1 'weak' 1)."""
+    monkeypatch.setenv("FD_GROUP_FRAMES", "16")
     _bench_shape_parity(48)
+
+
+def test_video_batch_1080p_default_groups_sampled():
+    """The bench's launch configuration: the default grouping (128 1080p frames per group, from
+    the 12 GiB workspace budget) over 384 frames = three groups alternating over both pipeline
+    slots.  Every frame runs on the GPU; the oracle checks the detections of sampled frames at
+    both ends of every group (whole-batch stage counters and grouping are checked above)."""
+    W, H, s = 1920, 1080, 1.1
+    n = 384
+    lv = oracle.plan(W, H, 24, s, 1)
+    fr, _ = fdgen.frames(4, 500, n, W, H, lv, faces="poisson", face_param=4, max_face_level=30)
+    gc, oc = cascades(3)
+    got = fd.to_numpy(fd.fd_detect(gc, torch.from_numpy(fr).cuda(), 24, s, 1, capacity=1 << 22))
+    near = 0
+    for i in (0, 1, 127, 128, 129, 255, 256, 383):
+        ref, nn = oracle.detect(oc, fr[i:i + 1], 24, s, 1, nthreads=os.cpu_count())
+        near += nn
+        g = got[got["frame"] == i].copy()
+        g["frame"] = 0
+        assert np.array_equal(g, ref), f"frame {i}"
+    print(f"{n} frames, 8 sampled: near-threshold windows {near}, 0 decision mismatches")
 
 
 def test_video_batch_1080p_small_groups(monkeypatch):
@@ -468,8 +492,9 @@ def test_all_pass_and_all_reject():
     assert len(fd.fd_detect(allrej, torch.from_numpy(fr).cuda(), 24, s, 1)) == 0
 
 
-@pytest.mark.parametrize("env", [{}, {"FD_DEEPQ": "0"}, {"FD_JIT": "0"}, {"FD_DQ_TAIL": "4"},
-                                 {"FD_DQ_SLOTS": "2", "FD_DQ_WARPS": "4"}])
+@pytest.mark.parametrize("env", [{"FD_DEEPQ": "1"}, {"FD_DEEPQ": "0"}, {"FD_DEEPQ": "1", "FD_JIT": "0"},
+                                 {"FD_DEEPQ": "1", "FD_DQ_TAIL": "4"},
+                                 {"FD_DEEPQ": "1", "FD_DQ_SLOTS": "2", "FD_DQ_WARPS": "4"}])
 def test_all_pass_deep(env, monkeypatch):
     """Every window survives every stage of a 7-stage cascade: k_deepq's batches stay full through
     every deep stage (2048 windows per tile, more than a slot's shared-memory survivor list), slots
