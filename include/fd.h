@@ -131,8 +131,11 @@ fd_status fd_integral(const uint8_t* d_img, int n, int W, int H, int pitch, uint
  * Synchronises `stream` once (to read the count); the records in d_out are complete when
  * `stream` next completes.
  * Schedules (identical results): default K1 (global ii/sqii) -> k_stage1 ->
- * k_deep1 -> k_tail; environment FD_F1=1 selects SURVEY 8(f) f1 (k_level -> k_f1 with tile-local
- * integrals in shared memory -> k_deep1<F1> -> k_tail; no global integral image). */
+ * k_deepq (frame groups of >= 4 frames, uncompressed cascades) or k_deep1 -> k_tail (otherwise,
+ * or environment FD_DEEPQ=0); environment FD_F1=1 selects SURVEY 8(f) f1 (k_level -> k_f1 with
+ * tile-local integrals in shared memory -> k_deep1<F1> -> k_tail; no global integral image).
+ * Frames are processed in groups of up to 128 1080p frames (FD_GROUP_MB workspace budget,
+ * default 12 GiB: ~48 GB of device memory over the two pipeline slots at 1080p). */
 fd_status fd_detect(fd_cascade c, const uint8_t* d_frames, int n, int W, int H, int pitch,
                     int min_size, double scale_factor, int step, fd_detection* d_out,
                     int64_t capacity, int64_t* n_out, void* stream);
@@ -193,12 +196,12 @@ fd_status fd_detect_group_host(fd_cascade c, const uint8_t* h_frames, int n, int
  * since the last fd_profile_reset and, if time_kernels != 0, their summed device time
  * measured with CUDA events recorded on the launching stream around each launch.
  * FD_K_SORT is the CUB radix sort (library code, counted as one call).  Default detection
- * path (f1): FD_K_LEVEL (k_level: the group's level images) and FD_K_CASCADE (k_f1: tile-local
- * integral + every stage).  K1 (fd_integral, soft cascades, the FD_F1=0 schedule) is
- * FD_K_COLSUM (k_marg: resampling + per-tile marginals), FD_K_CARRY (k_carry + k_corner) and
- * FD_K_BAND (k_tile: ii / sqii); its cascade kernels are FD_K_CASCADE (k_stage1, k_cascade or
- * k_soft) and FD_K_DEEP (k_deep1).  FD_K_TAIL is k_tail (the few windows left per tile, one warp
- * per window).  FD_K_DEPTH_HIST is fd_depth_histogram. */
+ * path: K1 is FD_K_COLSUM (k_marg: resampling + per-tile marginals), FD_K_CARRY (k_carry +
+ * k_corner) and FD_K_BAND (k_tile: ii / sqii); the cascade kernels are FD_K_CASCADE (k_stage1,
+ * k_cascade or k_soft) and FD_K_DEEP (k_deepq or k_deep1).  FD_K_TAIL is k_tail (windows handed
+ * over one warp per window).  The f1 schedule (FD_F1=1): FD_K_LEVEL (k_level: the group's level
+ * images) and FD_K_CASCADE (k_f1: tile-local integral + stages 1-2).  FD_K_DEPTH_HIST is
+ * fd_depth_histogram. */
 typedef enum {
     FD_K_COLSUM = 0, FD_K_CARRY = 1, FD_K_BAND = 2, FD_K_CASCADE = 3,
     FD_K_SORT = 4, FD_K_DETS = 5, FD_K_GROUP = 6, FD_K_PYRAMID = 7, FD_K_TAIL = 8,
