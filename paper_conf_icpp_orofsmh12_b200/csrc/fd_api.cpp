@@ -689,8 +689,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     fd_status s = get_packed(c, step, &pk);
     if (s != FD_OK) return s;
     // Schedules (all under the same parity tests, tests/test_gpu_parity.py K2_SCHEDULES):
-    //   default for hard cascades: K1 -> k_stage1 -> k_deep1 -> k_tail (FD_K2_SPLIT=0: K1 ->
-    //            fused k_cascade -> k_tail);
+    //   default for hard cascades: K1 -> k_stage1 -> k_deepq, or k_deep1 -> k_tail (below);
     //   FD_F1=1: k_level -> k_f1 -> k_deep1<F1> -> k_tail, no global integral
     //            (FD_F1_SPLIT=0: k_f1 runs every stage);
     //   soft cascades (R8b) and FD_K2_QUEUE=1: K1 -> k_soft (one lane per window, running sums).
@@ -700,7 +699,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
     // f1 split (default): k_f1 runs stages 0-1, k_deep1 the rest from rebuilt tile integrals
     // (FD_F1_SPLIT=0: k_f1 runs every stage itself)
     const bool f1_split = f1 && env_int("FD_F1_SPLIT", 1) != 0;
-    const bool split = !queue && !f1 && env_int("FD_K2_SPLIT", 1) != 0;
+    const bool split = !queue && !f1;
     const bool surv = split || f1_split;
     // frames per group: one K2 launch per group.  f1: the group's level images (12.5 MB per 1080p
     // frame) should stay L2-resident between k_level and k_f1 (FD_F1_GROUP_MB, default 64 MB);
@@ -858,7 +857,6 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         CK(cudaStreamWaitEvent(w->side, w->ev_fork, 0));
         sts[1] = w->side;
     }
-    const int grid = cascade_grid(depth, step);
     for (int gi = 0; gi < ngroups; ++gi) {
         // group gi runs on slot gi % nslots; the slot's stream orders it after group gi - nslots,
         // the previous user of the slot's buffers
@@ -891,7 +889,6 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         P.tile_list = deepq ? sl.tlist.as<uint4>() : nullptr;
         P.surv = surv ? sl.surv.as<uint2>() : nullptr;
         P.tile_rec = surv ? sl.tilerec.as<uint2>() : nullptr;
-        const int gr = grid < P.total_tiles ? grid : P.total_tiles;
         if (queue) {
             LAUNCH(FD_K_CASCADE, gs, launch_soft(P, depth, step, soft, gs));
         } else if (jit) {
@@ -899,7 +896,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
             cudaError_t e;
             {
                 ProfScope ps(FD_K_CASCADE, gs);
-                e = jit_k2_launch(jit, P, depth, f1 ? JIT_F1 : (split ? JIT_STAGE1 : JIT_FUSED), gs, &err);
+                e = jit_k2_launch(jit, P, depth, f1 ? JIT_F1 : JIT_STAGE1, gs, &err);
             }
             if (e == cudaSuccess && surv) {
                 ProfScope ps(FD_K_DEEP, gs);
@@ -910,14 +907,12 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         } else if (f1) {
             LAUNCH(FD_K_CASCADE, gs, launch_f1(P, depth, step, gs));
             if (f1_split) LAUNCH(FD_K_DEEP, gs, launch_deep1(P, depth, step, true, gs));
-        } else if (split) {
+        } else {
             LAUNCH(FD_K_CASCADE, gs, launch_stage1(P, depth, step, gs));
             if (deepq)
                 LAUNCH(FD_K_DEEP, gs, launch_deepq(P, depth, step, gs));
             else
                 LAUNCH(FD_K_DEEP, gs, launch_deep1(P, depth, step, false, gs));
-        } else {
-            LAUNCH(FD_K_CASCADE, gs, launch_cascade(P, depth, step, gr, gs));
         }
         if (use_tail) {
             TP.q = P.tail_q;

@@ -53,8 +53,8 @@ __host__ __device__ constexpr int tile_h(int step) { return (k2_ty(step) - 1) * 
 __host__ __device__ constexpr int k2_pbuf(int step) { return (tile_w(step) * tile_h(step) + 31) & ~31; }
 
 
-// Fused K2 (k_cascade) shared memory: the tile's ii plane, then its sqii plane -- which, once
-// stage 1 has taken every window's variance from it, holds the stage-1 survivor pool
+// k_soft (and the former fused K2) shared memory: the tile's ii plane, then its sqii plane -- which,
+// once stage 1 has taken every window's variance from it, holds the stage-1 survivor pool
 // (nf f32[NW], window u16[NW]) and the two per-stage lists (u16[2][NW]).
 template <int STEP>
 struct TileGeo {
@@ -69,9 +69,6 @@ struct TileGeo {
     static constexpr size_t OFF_RED = OFF_Q + (size_t)QBUF * 4;
     static constexpr size_t SMEM = OFF_RED + (size_t)k2_threads(STEP) * 8;   // + split-stump partial sums
 };
-#ifndef FD_K2_CTAS
-#define FD_K2_CTAS 4                        // fused K2: resident CTAs per SM the launch bounds target
-#endif
 
 // k_stage1 (K2a): two ii planes (the current tile's and the prefetched next tile's), one sqii
 // plane (dead once the variance is taken, so the next tile's sqii lands in it during stages 1-2)
@@ -312,7 +309,6 @@ cudaError_t launch_k1_tiles_canonical(const uint8_t* img, const PlanDev& plan, i
                                       uint32_t* ii, uint64_t* sqii, int out_pitch, cudaStream_t st);
 cudaError_t launch_pyramid(const uint8_t* frames, const PlanDev& plan, int n, uint8_t* levels,
                            long long frame_stride, const long long* lvl_off_host, cudaStream_t st);
-cudaError_t launch_cascade(const CascadeParams& p, bool depth_mode, int step, int grid, cudaStream_t st);
 // f1: level images of a frame group (u8, level-major, pitch PB) and the fused tile-local kernel
 cudaError_t launch_levels(const uint8_t* frames, const PlanDev& plan, int g_frames, uint8_t* out, cudaStream_t st);
 cudaError_t launch_f1(const CascadeParams& p, bool depth_mode, int step, cudaStream_t st);
@@ -324,8 +320,6 @@ cudaError_t launch_deepq(const CascadeParams& p, bool depth_mode, int step, cuda
 cudaError_t launch_soft(const CascadeParams& p, bool depth_mode, int step, bool soft, cudaStream_t st);  // k_soft.cu (R8b)
 cudaError_t launch_depth_hist(const uint8_t* depth, int n, long long win_per_frame, const long long* d_win0,
                               int n_levels, int n_stages, long long* hist, int max_span, cudaStream_t st);
-int cascade_grid(bool depth_mode, int step);       // persistent grid size (SMs x resident CTAs)
-size_t cascade_smem(int step);
 cudaError_t launch_keys_to_dets(const unsigned long long* keys, const float* scores, long long n,
                                 const double* f_levels_dev, int n_stages, fd_detection* out, cudaStream_t st);
 cudaError_t sort_pairs(void* tmp, size_t& tmp_bytes, const unsigned long long* kin, unsigned long long* kout,

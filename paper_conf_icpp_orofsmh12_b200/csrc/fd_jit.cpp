@@ -187,11 +187,6 @@ static int jit_dq_warps() {
     return v < 1 ? 1 : (v > 32 ? 32 : v);
 }
 
-// resident CTAs per SM targeted by the fused kernel's launch bounds (FD_K2_CTAS, 2..6)
-static int jit_ctas() {
-    const int c = env_or("FD_K2_CTAS", FD_K2_CTAS);
-    return c < 2 ? 2 : (c > 6 ? 6 : c);
-}
 
 std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_stages, const std::vector<uint32_t>* pk16) {
     // k_deep1 runs its specialised stages one lane per window even when few windows are left, so
@@ -212,7 +207,6 @@ std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_sta
     std::string src = pre + "#define FD_K2D_CTAS " + std::to_string(env_or("FD_K2D_CTAS", FD_K2D_CTAS)) +
                       "\n#define FD_K2D_THREADS " + std::to_string(jit_deep_threads()) +
                       "\n#define FD_F1_CTAS " + std::to_string(env_or("FD_F1_CTAS", FD_F1_CTAS)) +
-                      "\n#define FD_K2_CTAS " + std::to_string(jit_ctas()) +
                       "\n#define FD_DQ_SLOTS " + std::to_string(jit_dq_slots()) +
                       "\n#define FD_DQ_WARPS " + std::to_string(jit_dq_warps()) +
                       "\n#define FD_DQ_GROUP " + std::to_string(env_or("FD_DQ_GROUP", 16)) +
@@ -227,7 +221,6 @@ std::string jit_program(const uint32_t* rec_words, const StageDev* st, int n_sta
 
 static std::string jit_name(int kind, bool depth) {
     const std::string d = depth ? "true" : "false";
-    if (kind == JIT_FUSED) return "fdk::k_cascade<1, " + d + ">";
     if (kind == JIT_STAGE1) return "fdk::k_stage1<1, " + d + ">";
     if (kind == JIT_DEEP1) return "fdk::k_deep1<1, " + d + ", false>";
     if (kind == JIT_DEEP1_F1) return "fdk::k_deep1<1, " + d + ", true>";
@@ -238,7 +231,6 @@ static std::string jit_name(int kind, bool depth) {
 static KindGeo jit_kind_geo(int kind) {
     KindGeo g;
     g.threads = (kind == JIT_DEEP1 || kind == JIT_DEEP1_F1) ? jit_deep_threads() : k2_threads(JIT_STEP);
-    if (kind == JIT_FUSED) g.smem = TileGeo<JIT_STEP>::SMEM;
     if (kind == JIT_STAGE1) g.smem = TileGeoA<JIT_STEP>::SMEM;
     if (kind == JIT_DEEP1) g.smem = TileGeoD<JIT_STEP, false>::SMEM;
     if (kind == JIT_DEEP1_F1) g.smem = TileGeoD<JIT_STEP, true>::SMEM;

@@ -8,9 +8,9 @@
 namespace fdk {
 
 struct JitK2;
-// kernels of the specialised program: split k_stage1 + k_deep1 (default), fused k_cascade, and
-// the f1 kernels k_f1 + k_deep1<F1> (tile integrals rebuilt from level images)
-enum { JIT_FUSED = 0, JIT_STAGE1 = 1, JIT_DEEP1 = 2, JIT_F1 = 3, JIT_DEEP1_F1 = 4, JIT_DEEPQ = 5, JIT_KINDS = 6 };
+// kernels of the specialised program: k_stage1 + k_deepq or k_deep1, and the f1 kernels k_f1 +
+// k_deep1<F1> (tile integrals rebuilt from level images)
+enum { JIT_STAGE1 = 0, JIT_DEEP1 = 1, JIT_F1 = 2, JIT_DEEP1_F1 = 3, JIT_DEEPQ = 4, JIT_KINDS = 5 };
 // CUDA source of the generated first stage (stage index `first`..first+n of the packed step-1
 // records, REC_WORDS u32 per stump)
 std::string jit_stage1_source(const uint32_t* rec_words, int first, int n);

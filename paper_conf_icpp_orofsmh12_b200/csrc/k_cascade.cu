@@ -20,8 +20,9 @@
 //     (one stump per lane) and the leaves are added in stump order;
 //   * fp32 arithmetic matches the oracle bit for bit: __fmul_rn/__fadd_rn (no FMA
 //     contraction), __int2float_rn, __ll2float_rn, IEEE __fsqrt_rn.
-// Kernels: k_stage1 + k_deep1 (default schedule, split at stage 2), k_cascade (fused, all stages
-// in one CTA), k_f1 (+ k_deep1<F1>: SURVEY 8(f) f1, tile-local integrals built in shared memory).
+// Kernels: k_stage1 + k_deepq (k_deepq.cuh) or k_deep1 (split at stage 2), k_f1 (+ k_deep1<F1>:
+// SURVEY 8(f) f1, tile-local integrals built in shared memory).  (A fused kernel running every
+// stage of a tile in one CTA was measured slower in rounds 1-2 and removed.)
 // This file is also compiled at run time by NVRTC with the cascade's specialised stages
 // (fd_jit.cpp: FD_JIT_STAGE1, FD_JIT_DEEP, FD_PACKED_WORDS).
 #include "k_common.cuh"
@@ -485,136 +486,6 @@ __device__ __forceinline__ TileAt tile_at(const CascadeParams& p, int tn) {
     t.x = t.wx0 * STEP;
     t.y = t.wy0 * STEP;
     return t;
-}
-
-// Fused K2: one CTA per tile at a time, persistent over every (frame, level, tile) of the
-// group.  One TMA brings the tile's ii and sqii planes; stage 1 runs densely (WPT windows per
-// thread down a column, nf from the variance, oracle c5); its survivors go into a pool that
-// reuses the sqii buffer (dead once every nf is taken), and deep_phase runs the deeper stages
-// over the pool.  40 KB of shared memory per CTA keeps FD_K2_CTAS CTAs resident per SM, so
-// the latency-bound deep phase of one tile overlaps the dense stage 1 of the others.
-template <int STEP, bool DEPTH>
-__global__ void __launch_bounds__(k2_threads(STEP), FD_K2_CTAS) k_cascade(const __grid_constant__ CascadeParams p) {
-    using G = TileGeo<STEP>;
-    constexpr int TW = tile_w(STEP), TX = k2_tx(STEP), TY = k2_ty(STEP), WPT = k2_wpt(STEP), CP = G::CP;
-    constexpr int WARPS_X = TX / 32, PLANE = tile_w(STEP) * tile_h(STEP);
-    extern __shared__ __align__(1024) uint8_t smem_raw[];
-    uint32_t* T = reinterpret_cast<uint32_t*>(smem_raw);                      // ii plane
-    uint32_t* Q = reinterpret_cast<uint32_t*>(smem_raw + G::OFF_Q);           // sqii plane (mod 2^32)
-    float* pnf = reinterpret_cast<float*>(smem_raw + G::OFF_NF);              // pool, over Q after stage 1
-    uint16_t* ploc = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LOC);
-    uint16_t* lists = reinterpret_cast<uint16_t*>(smem_raw + G::OFF_LIST);
-    __shared__ __align__(8) uint64_t mbar;
-    __shared__ int s_tile;
-    __shared__ int s_frame[1], s_lvl[1], s_wx0[1], s_wy0[1];
-    __shared__ int s_cnt[3];
-    __shared__ int s_tpos;
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const StageDev& st0 = p.pstages[0];     // parameter bank: warp-uniform (n_pstages >= 1)
-    const ParamRec prec{p};
-    const GlobalRec grec{p.stumps};
-    const WinOut<STEP, DEPTH> out{p, s_frame, s_lvl, s_wx0, s_wy0};
-    if (tid == 0) {
-        mbar_init(&mbar, 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    uint32_t phase = 0;
-    for (;;) {
-        __syncthreads();                          // buffers and s_* free
-        if (tid == 0) {
-            s_cnt[0] = 0;
-            s_cnt[1] = 0;
-            s_cnt[2] = 0;
-            const int tn = (int)atomicAdd(p.tile_counter, 1u);
-            s_tile = tn;
-            if (tn < p.total_tiles) {
-                const TileAt t = tile_at<STEP>(p, tn);
-                s_frame[0] = p.frame_base + t.g;
-                s_lvl[0] = t.k;
-                s_wx0[0] = t.wx0;
-                s_wy0[0] = t.wy0;
-                // generic-proxy accesses of the buffers are ordered before the async-proxy writes
-                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                mbar_expect_tx(&mbar, 2 * PLANE * 4);
-                tma_load_4d(T, p.tmaps + t.k, t.x, t.y, 0, t.g, &mbar);
-                tma_load_4d(Q, p.tmaps + t.k, t.x, t.y, 1, t.g, &mbar);
-            }
-        }
-        __syncthreads();
-        if (s_tile >= p.total_tiles) break;
-#ifdef FD_K2_TIMING
-        const long long tm0 = clock64();
-#endif
-        mbar_wait(&mbar, phase);
-        phase ^= 1;
-#ifdef FD_K2_TIMING
-        const long long tm1 = clock64();
-#endif
-        const int k = s_lvl[0];
-        const int nx = __ldg(&p.lv[k].nx), ny = __ldg(&p.lv[k].ny);
-        const int wx0 = s_wx0[0], wy0 = s_wy0[0];
-        const int lx = lane + 32 * (warp % WARPS_X);
-        const int ly0 = (warp / WARPS_X) * WPT;
-        const int base = ly0 * STEP * TW + lx * STEP;
-        const bool colok = wx0 + lx < nx;
-        float nf[WPT], sm[WPT];
-#pragma unroll
-        for (int i = 0; i < WPT; ++i) {
-            const int b = base + i * STEP * TW;
-            const uint32_t S = T[b + WIN * TW + WIN] - T[b + WIN] - T[b + WIN * TW] + T[b];
-            const uint32_t q = Q[b + WIN * TW + WIN] - Q[b + WIN] - Q[b + WIN * TW] + Q[b];
-            const long long v = 576LL * (long long)q - (long long)S * (long long)S;
-            nf[i] = v > 0 ? __fsqrt_rn(__ll2float_rn(v)) : 1.0f;
-            sm[i] = 0.0f;
-        }
-#ifdef FD_JIT_STAGE1
-        // run-time specialised first stage (fd_jit.cpp): corner offsets, coefficients and
-        // thresholds are immediates and each (column, row) value is loaded once per thread
-        jit_stage1(T + base, nf, sm);
-#else
-        if (st0.first + st0.n <= p.n_pstumps)
-            dense_stage<WPT, STEP * TW>(T, base, nf, sm, prec, st0.first, st0.n);
-        else
-            dense_stage<WPT, STEP * TW>(T, base, nf, sm, grec, st0.first, st0.n);
-#endif
-        __syncthreads();                          // every sqii read done: the buffer becomes the pool
-        // stage-1 survivors into the pool (or out, for a one-stage cascade)
-#pragma unroll
-        for (int i = 0; i < WPT; ++i) {
-            const int wy = wy0 + ly0 + i;
-            const bool valid = colok && wy < ny;
-            const bool pass = valid && (sm[i] >= st0.T);
-            const int idx = (ly0 + i) * TX + lx;
-            if (DEPTH && valid && !pass) out.reject(0, idx, 0, sm[i]);
-            if (p.n_stages == 1) {
-                if (pass) out.emit(0, idx, sm[i]);
-                continue;
-            }
-            const unsigned m = __ballot_sync(0xffffffffu, pass);
-            if (m) {
-                int pos = 0;
-                if (lane == 0) pos = atomicAdd(&s_cnt[1], __popc(m));
-                pos = __shfl_sync(0xffffffffu, pos, 0);
-                if (pass) {
-                    const int at = pos + __popc(m & ((1u << lane) - 1u));
-                    ploc[at] = (uint16_t)idx;
-                    pnf[at] = nf[i];
-                }
-            }
-        }
-        if (tid == 0 && p.stage_counts)
-            atomicAdd(p.stage_counts, (unsigned long long)min(TX, nx - wx0) * (unsigned long long)min(TY, ny - wy0));
-#ifdef FD_K2_TIMING
-        if (tid == 0) {
-            atomicAdd(&g_k2_timing[0], 1ull);
-            atomicAdd(&g_k2_timing[1], (unsigned long long)(tm1 - tm0));
-            atomicAdd(&g_k2_timing[2], (unsigned long long)(clock64() - tm1));
-        }
-#endif
-        __syncthreads();                          // pool complete
-        deep_phase<STEP, DEPTH, CP>(p, 1, T, pnf, ploc, lists, s_cnt, s_tpos, out,
-                                    reinterpret_cast<float2*>(smem_raw + G::OFF_RED));
-    }
 }
 
 // ======================================================================== split K2, kernel a
@@ -1202,26 +1073,6 @@ namespace fdk {
 // instantiates only its own step's kernels (StepLaunch<FD_KC_STEP>), and the step-1 object also
 // holds the dispatchers over the step.  Without FD_KC_STEP every step is instantiated here.
 template <int STEP, bool DEPTH>
-static cudaError_t launch_one(const CascadeParams& p, int grid, cudaStream_t st) {
-    const size_t smem = TileGeo<STEP>::SMEM;
-    cudaError_t e = cudaFuncSetAttribute(k_cascade<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    k_cascade<STEP, DEPTH><<<grid, k2_threads(STEP), smem, st>>>(p);
-    return cudaGetLastError();
-}
-
-template <int STEP, bool DEPTH>
-static int grid_step() {
-    const size_t smem = TileGeo<STEP>::SMEM;
-    cudaFuncSetAttribute(k_cascade<STEP, DEPTH>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    int dev = 0, sms = 0, per = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_cascade<STEP, DEPTH>, k2_threads(STEP), smem);
-    return sms * (per > 0 ? per : 1);
-}
-
-template <int STEP, bool DEPTH>
 static cudaError_t launch_stage1_t(const CascadeParams& p, cudaStream_t st) {
     static int grid = 0;
     const size_t smem = TileGeoA<STEP>::SMEM;
@@ -1294,10 +1145,6 @@ static cudaError_t launch_f1_t(const CascadeParams& p, cudaStream_t st) {
 
 template <int STEP>
 struct StepLaunch {
-    static cudaError_t cascade(const CascadeParams& p, bool d, int grid, cudaStream_t st) {
-        return d ? launch_one<STEP, true>(p, grid, st) : launch_one<STEP, false>(p, grid, st);
-    }
-    static int grid(bool d) { return d ? grid_step<STEP, true>() : grid_step<STEP, false>(); }
     static cudaError_t stage1(const CascadeParams& p, bool d, cudaStream_t st) {
         return d ? launch_stage1_t<STEP, true>(p, st) : launch_stage1_t<STEP, false>(p, st);
     }
@@ -1332,25 +1179,6 @@ extern template struct StepLaunch<4>;
         default: return cudaErrorInvalidValue;        \
     }
 
-size_t cascade_smem(int step) {
-    switch (step) {
-        case 1: return TileGeo<1>::SMEM;
-        case 2: return TileGeo<2>::SMEM;
-        case 3: return TileGeo<3>::SMEM;
-        default: return TileGeo<4>::SMEM;
-    }
-}
-int cascade_grid(bool depth, int step) {
-    switch (step) {
-        case 1: return StepLaunch<1>::grid(depth);
-        case 2: return StepLaunch<2>::grid(depth);
-        case 3: return StepLaunch<3>::grid(depth);
-        default: return StepLaunch<4>::grid(depth);
-    }
-}
-cudaError_t launch_cascade(const CascadeParams& p, bool depth, int step, int grid, cudaStream_t st) {
-    FD_STEP_SWITCH(step, cascade(p, depth, grid, st))
-}
 cudaError_t launch_stage1(const CascadeParams& p, bool depth, int step, cudaStream_t st) {
     FD_STEP_SWITCH(step, stage1(p, depth, st))
 }

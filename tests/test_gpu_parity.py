@@ -148,7 +148,6 @@ K2_SCHEDULES = {
     "deep1_split_stump": {"FD_DEEPQ": "0", "FD_DEEP_SPLIT": "64"},   # deep stages <= 64 windows split-stump
     "deep1_2warps": {"FD_DEEPQ": "0", "FD_K2D_THREADS": "64"},       # two-warp k_deep1 blocks
     "deep1_s_tail_3": {"FD_DEEPQ": "0", "FD_S_TAIL": "3"},  # every window alive at stage 3 through k_tail
-    "fused_k1": {"FD_K2_SPLIT": "0"},                       # K1 -> k_cascade -> k_tail
     "f1": {"FD_F1": "1"},                                   # k_level -> k_f1 -> k_deep1<F1> -> k_tail
     "f1_no_tail": {"FD_F1": "1", "FD_TAIL": "0"},
     "f1_tail_early": {"FD_F1": "1", "FD_TAIL_N": "200"},    # most deep windows through k_tail (u8 rebuild)
@@ -164,7 +163,7 @@ K2_SCHEDULES = {
 
 # variables read when a cascade's specialised program is generated (once per fd.Cascade)
 JIT_GEOMETRY_ENV = {"FD_DQ_SLOTS", "FD_DQ_WARPS", "FD_DQ_GROUP", "FD_JIT_DEEPQ_STUMPS", "FD_K2D_THREADS", "FD_K2D_CTAS",
-                    "FD_K2_CTAS", "FD_F1_CTAS"}
+                    "FD_F1_CTAS"}
 
 
 @pytest.mark.parametrize("jit", ["1", "0"])
