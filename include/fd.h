@@ -169,7 +169,9 @@ fd_status fd_depth_histogram(const uint8_t* d_depth, int n, int W, int H, int mi
                              int step, int n_stages, int64_t* d_hist, void* stream);
 
 /* End-to-end entry with HOST buffers: copies h_frames to the device, runs fd_detect, copies
- * the detections back to h_out (capacity elements).  Synchronises `stream`. */
+ * the detections back to h_out (capacity elements).  Synchronises `stream`.  The frames are
+ * copied one frame group at a time on that group's pipeline stream, so the copy of a group
+ * overlaps the kernels of the previous one (pinned h_frames make the copies asynchronous). */
 fd_status fd_detect_host(fd_cascade c, const uint8_t* h_frames, int n, int W, int H, int pitch,
                          int min_size, double scale_factor, int step, fd_detection* h_out,
                          int64_t capacity, int64_t* n_out, void* stream);
@@ -184,8 +186,9 @@ fd_status fd_group(const fd_detection* d_in, int64_t n, double eyes_thresh, int 
                    fd_detection* d_out, int64_t capacity, int64_t* n_out, void* stream);
 
 /* fd_detect + fd_group end to end with HOST buffers (the user-facing e2e call): copies
- * h_frames to the device, detects, groups (eyes_thresh, min_neighbors as fd_group) and copies
- * the grouped detections to h_out.  *n_raw (may be NULL) = detections before grouping.
+ * h_frames to the device (group by group, overlapped with the previous group's kernels, as
+ * fd_detect_host), detects, groups (eyes_thresh, min_neighbors as fd_group) and copies the
+ * grouped detections to h_out.  *n_raw (may be NULL) = detections before grouping.
  * Synchronises `stream`. */
 fd_status fd_detect_group_host(fd_cascade c, const uint8_t* h_frames, int n, int W, int H, int pitch,
                                int min_size, double scale_factor, int step, double eyes_thresh,

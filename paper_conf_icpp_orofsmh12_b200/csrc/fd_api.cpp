@@ -683,7 +683,8 @@ fd_status check_frames(const void* d, int n, int W, int H, int pitch) {
 // core of fd_detect / fd_detect_depth: the hot path for every frame group.
 fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int n, int W, int H, int pitch,
                      const fd_plan& pl, int step, bool depth, uint8_t* d_depth, float* d_score, long long det_cap,
-                     unsigned long long* d_stage_counts, cudaStream_t st) {
+                     unsigned long long* d_stage_counts, cudaStream_t st,
+                     const uint8_t* h_frames = nullptr) {
     if (step > MAX_STEP) return fail(FD_EINVAL, "step %d not supported (1..%d)", step, MAX_STEP);
     const Packed* pk = nullptr;
     fd_status s = get_packed(c, step, &pk);
@@ -866,6 +867,11 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
         const int f0 = gi * G, gf = (n - f0) < G ? (n - f0) : G;
         const uint8_t* fr = d_frames + (size_t)f0 * H * pitch;
         const cudaStream_t ks = gs;               // K1's stream
+        // host frames (fd_detect_host, fd_detect_group_host): each group's frames are copied on its
+        // own slot's stream, so the copy of group g+1 overlaps the kernels of group g
+        if (h_frames)
+            CK(cudaMemcpyAsync(const_cast<uint8_t*>(fr), h_frames + (size_t)f0 * H * pitch, (size_t)gf * H * pitch,
+                               cudaMemcpyHostToDevice, ks));
         if (f1) {
             LAUNCH(FD_K_LEVEL, ks, launch_levels(fr, PD, gf, sl.ws.as<uint8_t>(), ks));
         } else {
@@ -932,7 +938,7 @@ fd_status run_groups(fd_cascade_s* c, Workspace* w, const uint8_t* d_frames, int
 
 fd_status detect_impl(fd_cascade c, const uint8_t* d_frames, int n, int W, int H, int pitch, int min_size, double s,
                       int step, fd_detection* d_out, int64_t capacity, int64_t* n_out, int64_t* d_stage_counts,
-                      cudaStream_t st) {
+                      cudaStream_t st, const uint8_t* h_frames = nullptr) {
     if (!c) return fail(FD_EINVAL, "cascade is NULL");
     if (!n_out) return fail(FD_EINVAL, "n_out is NULL");
     if (capacity < 0) return fail(FD_EINVAL, "capacity < 0");
@@ -952,7 +958,7 @@ fd_status detect_impl(fd_cascade c, const uint8_t* d_frames, int n, int W, int H
     }
     const long long cap = capacity > 0 ? capacity : 1;
     r = run_groups(c, w, d_frames, n, W, H, pitch, pl, step, false, nullptr, nullptr, cap,
-                   reinterpret_cast<unsigned long long*>(d_stage_counts), st);
+                   reinterpret_cast<unsigned long long*>(d_stage_counts), st, h_frames);
     if (r != FD_OK) return r;
     CK(cudaMemcpyAsync(w->h_pinned, w->ctl.p, 8, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -1178,9 +1184,8 @@ fd_status fd_detect_host(fd_cascade c, const uint8_t* h_frames, int n, int W, in
         CK(w->outbuf.ensure((size_t)(capacity > 0 ? capacity : 1) * sizeof(fd_detection)));
         d_fr = w->frames.as<uint8_t>();
         d_out = w->outbuf.as<fd_detection>();
-        CK(cudaMemcpyAsync(d_fr, h_frames, (size_t)n * H * pitch, cudaMemcpyHostToDevice, st));
     }
-    r = detect_impl(c, d_fr, n, W, H, pitch, min_size, scale_factor, step, d_out, capacity, n_out, nullptr, st);
+    r = detect_impl(c, d_fr, n, W, H, pitch, min_size, scale_factor, step, d_out, capacity, n_out, nullptr, st, h_frames);
     if (r != FD_OK) return r;
     if (*n_out > 0) CK(cudaMemcpyAsync(h_out, d_out, (size_t)*n_out * sizeof(fd_detection), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
@@ -1237,7 +1242,6 @@ fd_status fd_detect_group_host(fd_cascade c, const uint8_t* h_frames, int n, int
         std::lock_guard<std::mutex> lk(w->mu);
         CK(w->frames.ensure((size_t)n * H * pitch));
         d_fr = w->frames.as<uint8_t>();
-        CK(cudaMemcpyAsync(d_fr, h_frames, (size_t)n * H * pitch, cudaMemcpyHostToDevice, st));
     }
     int64_t cnt = 0;
     for (int attempt = 0; attempt < 2; ++attempt) {
@@ -1250,7 +1254,9 @@ fd_status fd_detect_group_host(fd_cascade c, const uint8_t* h_frames, int n, int
             }
             d_raw = w->outbuf.as<fd_detection>();
         }
-        r = detect_impl(c, d_fr, n, W, H, pitch, min_size, scale_factor, step, d_raw, raw_cap, &cnt, nullptr, st);
+        // the frames are copied group by group inside the first attempt (and are resident for a retry)
+        r = detect_impl(c, d_fr, n, W, H, pitch, min_size, scale_factor, step, d_raw, raw_cap, &cnt, nullptr, st,
+                        attempt == 0 ? h_frames : nullptr);
         if (r == FD_ECAPACITY && attempt == 0) {
             std::lock_guard<std::mutex> lk(w->mu);
             CK(w->outbuf.ensure((size_t)cnt * sizeof(fd_detection)));

@@ -1,12 +1,5 @@
 mkdir -p gpurun_out
-run() { # tag env... (extra bench args in BARGS)
-  tag=$1; shift
-  env "$@" timeout 400 python bench.py --steps 10 --warmup 3 --no-cpu --no-e2e $BARGS > gpurun_out/b_$tag.json 2>gpurun_out/b_$tag.err; tail -2 gpurun_out/b_$tag.err
-  python -c "import json;d=json.load(open('gpurun_out/b_$tag.json'));k=d.get('kernel_ms_per_step_one_slot');print('$tag',round(d['value'],1),round(k['deep'],1),round(k.get('tail',0),1))"
-}
-run base
-run t9 FD_DQ_TAIL=9
-run t12 FD_DQ_TAIL=12
-BARGS="--cascade c6" run c6
-BARGS="--cascade c6" run c6t9 FD_DQ_TAIL=9
-BARGS="--cascade c6" run c6d1 FD_DEEPQ=0
+timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_dist.py -m gpu -q -k "host or group or smoke or dist or rank or bench_shape" > gpurun_out/t_h2d.log 2>&1; tail -2 gpurun_out/t_h2d.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; tail -1 gpurun_out/smoke.log
+timeout 600 python bench.py --steps 20 --warmup 5 --no-cpu > gpurun_out/b_h2d.json 2>gpurun_out/b_h2d.err; tail -2 gpurun_out/b_h2d.err
+python -c "import json;d=json.load(open('gpurun_out/b_h2d.json'));print('h2d',round(d['value'],1),d['e2e'])"
